@@ -1,0 +1,399 @@
+"""bench.py — Game of Life cell-updates/s and % HBM roofline on 1..8 B200.
+
+Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` (torchrun
+for N > 1) prints ONE JSON line on rank 0.
+
+* step      = one ``mapsm_iterate(grid, n)`` call: n generations (BASELINE.json
+              configs[2]: 200) of the whole hot path over the row-slab-
+              partitioned grid — boundary rows, halo exchange (N > 1),
+              interior, buffer swap — with the grid resident in HBM.
+* value     = w*h*n*K / max-over-ranks device time of the K timed steps
+              (CUDA events on the library's compute stream; L2 is flushed
+              between steps, outside the events).
+* e2e       = the same metric through the public C ABI with HOST buffers:
+              per step mapsm_bind (pinned u8 host rows -> device, packed),
+              mapsm_iterate(n), mapsm_read (device -> pinned host u8).
+* roofline  = the dominant kernel (life_step_kernel): 0.25 B/cell-update
+              algorithmic (1 bit in + 1 bit out), per launch, vs the measured
+              HBM copy bandwidth (MEASURED_PEAKS.json hbm_gbs).
+* cpu_baseline = the CPU oracle (oracle/oracle.c, OpenMP) timed on a bounded
+              sample of the same workload on rank 0 only.
+``--impl reference`` times only the oracle (this tier's reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+import numpy as np  # noqa: E402
+
+WORKLOADS = {
+    # name: (op, w, h_total_at_1gpu, radius, boundary, n per step, seed field, seed weights, scaling)
+    "life64k": dict(op="life", w=65536, h=65536, r=1, b="wrap", n=200, seed=0x5EED0003, wseed=None,
+                    scaling="strong", bcell=0.25,
+                    label="Game of Life 65536x65536 WRAP, random p=0.5 (splitmix64 seed 0x5EED0003), "
+                          "200 generations per step (BASELINE configs[2])"),
+    "life8k": dict(op="life", w=8192, h=8192, r=1, b="wrap", n=1000, seed=0x5EED0002, wseed=None,
+                   scaling="strong", bcell=0.25,
+                   label="Game of Life 8192x8192 WRAP, random p=0.5 (seed 0x5EED0002), 1000 generations per step "
+                         "(BASELINE configs[1]; L2-resident)"),
+    "conv5": dict(op="conv", w=16384, h=16384, r=2, b="clamp", n=500, seed=0x5EED0004, wseed=0x5EED0044,
+                  scaling="strong", bcell=8.0,
+                  label="fp32 5x5 window convolution 16384x16384 CLAMP, 500 iterations per step (BASELINE configs[3])"),
+    "conv9": dict(op="conv", w=32768, h=4096, r=4, b="zero", n=100, seed=0x5EED0005, wseed=0x5EED0055,
+                  scaling="weak", bcell=8.0,
+                  label="fp32 9x9 (r=4) window stencil, 32768 wide x 4096 rows per GPU, ZERO, 100 iterations per "
+                        "step (BASELINE configs[4], weak scaling)"),
+}
+
+
+def load_peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, copy)"
+    return 6650.0, "fallback (B200_PROFILING.md 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device_index: int):
+        self.dev = device_index
+        self.proc = None
+        self.lines = []
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                                          "-lms", "100", "-i", str(self.dev)], stdout=subprocess.PIPE,
+                                         stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+        except Exception:
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def stop(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        self.t.join(timeout=2)
+        sm, smax, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        for ln in self.lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 6:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                smax.append(float(parts[1]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, parts[2:6]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+                "reasons": sorted(reasons), "samples": len(sm)}
+
+
+def cpu_baseline(wl, budget_s=12.0):
+    """Time the oracle (as it stands) on a bounded sample of the workload."""
+    import mapsm_inputs as mi
+    import oracle
+
+    w = wl["w"]
+    rows = 512 if wl["op"] == "life" else 256
+    if wl["op"] == "life":
+        g0 = mi.life_u8(wl["seed"], w, rows)
+        run = lambda n: oracle.life(g0, n, wl["b"])
+    else:
+        g0 = mi.field_f32(wl["seed"], w, rows)
+        W = mi.weights_f32(wl["wseed"], wl["r"])
+        run = lambda n: oracle.conv(g0, W, n, wl["b"])
+    t0 = time.perf_counter()
+    run(1)
+    t1 = time.perf_counter() - t0
+    n = max(1, min(wl["n"], int(budget_s / max(t1, 1e-6))))
+    t0 = time.perf_counter()
+    run(n)
+    dt = time.perf_counter() - t0
+    return {"value": w * rows * n / dt, "unit": "cell-updates/s", "cores": oracle.num_threads(), "kind": "oracle",
+            "sample": f"{w} x {rows} rows of the same {wl['op']} workload ({wl['b']} boundary on the sample), "
+                      f"{n} iterations, {dt:.1f} s wall (oracle.c, OpenMP, byte/cell Life or fmaf-chain conv)"}
+
+
+def run_reference(args, wl, rank, world):
+    """Reference arm of this tier: the oracle as it stands, on the host cores,
+    rank 0 only; each step is a bounded sample (full width, 512 or 256 rows,
+    k iterations) of the same workload, sized so W+K steps take ~1 minute."""
+    if rank != 0:
+        return
+    import mapsm_inputs as mi
+    import oracle
+
+    w = wl["w"]
+    rows = 512 if wl["op"] == "life" else 256
+    if wl["op"] == "life":
+        g0 = mi.life_u8(wl["seed"], w, rows)
+        run = lambda k: oracle.life(g0, k, wl["b"])
+    else:
+        g0 = mi.field_f32(wl["seed"], w, rows)
+        W = mi.weights_f32(wl["wseed"], wl["r"])
+        run = lambda k: oracle.conv(g0, W, k, wl["b"])
+    t0 = time.perf_counter()
+    run(1)
+    t1 = time.perf_counter() - t0
+    per_step = max(1, min(wl["n"], int(60.0 / max(1, args.steps + args.warmup) / max(t1, 1e-6))))
+    for _ in range(args.warmup):
+        run(per_step)
+    t0 = time.perf_counter()
+    for _ in range(args.steps):
+        run(per_step)
+    dt = time.perf_counter() - t0
+    value = w * rows * per_step * args.steps / dt
+    cb = {"value": value, "unit": "cell-updates/s", "cores": oracle.num_threads(), "kind": "oracle",
+          "sample": f"per step: {w} x {rows} rows, {per_step} iterations of the same workload "
+                    f"({wl['b']} boundary on the sample); {args.steps} timed steps, {dt:.1f} s"}
+    metric = "Game of Life cell-updates/s" if wl["op"] == "life" else f"fp32 {2*wl['r']+1}x{2*wl['r']+1} window-conv cell-updates/s"
+    line = {"impl": "reference", "metric": metric, "value": value, "unit": "cell-updates/s",
+            "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
+            "higher_is_better": True, "scaling": wl["scaling"], "vs_baseline": None,
+            "dtype": "u8" if wl["op"] == "life" else "f32", "data": "synthetic",
+            "config": {"workload": wl["label"]}, "cpu_baseline": cb,
+            "e2e": {"value": value, "unit": "cell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=10)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="mapsm", choices=["mapsm", "reference"])
+    ap.add_argument("--workload", default="life64k", choices=sorted(WORKLOADS))
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--graph-iters", type=int, default=0)
+    args = ap.parse_args()
+    wl = dict(WORKLOADS[args.workload])
+
+    rank = int(os.environ.get("RANK", "0"))
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.impl == "reference":
+        run_reference(args, wl, rank, world)
+        return
+
+    import torch
+    import torch.distributed as dist
+
+    import mapsm_inputs as mi
+    from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.current_stream()
+    uid = None
+    if world > 1:
+        obj = [M.mapsm_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    ctx = M.mapsm_ctx_create(rank, world, local_rank, uid, stream.cuda_stream)
+
+    w = wl["w"]
+    h = wl["h"] * (world if wl["scaling"] == "weak" else 1)
+    n = wl["n"]
+    W = mi.weights_f32(wl["wseed"], wl["r"]) if wl["op"] == "conv" else None
+    grid = M.Grid(ctx, w, h, wl["op"], wl["r"], wl["b"], W)
+    if args.graph_iters:
+        grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
+    y0, rows = grid.local_rows()
+    host_dtype = torch.uint8 if wl["op"] == "life" else torch.float32
+    # pinned host rows of this rank (input and result buffers for e2e)
+    h_in = torch.empty((rows, w), dtype=host_dtype, pin_memory=True)
+    if wl["op"] == "life":
+        mi.life_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
+    else:
+        mi.field_f32(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
+    h_out = torch.empty_like(h_in, pin_memory=True)
+    grid.bind(h_in)
+    info0 = grid.info()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local_rank])
+        torch.cuda.synchronize()
+
+    # warm-up (graph capture, NCCL connections, clocks)
+    for _ in range(args.warmup):
+        grid.iterate(n)
+    barrier()
+
+    # timed region: K steps, L2 flushed between steps outside the events
+    sampler = ClockSampler(local_rank)
+    sampler.start()
+    launches0 = grid.info().launches
+    total_ms = 0.0
+    barrier()
+    for _ in range(args.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        grid.iterate(n)
+        e1.record(stream)
+        e1.synchronize()
+        total_ms += e0.elapsed_time(e1)
+    barrier()
+    clocks = sampler.stop()
+    launches = grid.info().launches - launches0
+    used_graphs = bool(grid.info().used_graphs)
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    tl = torch.tensor([launches], dtype=torch.int64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        dist.all_reduce(tl, op=dist.ReduceOp.SUM)
+    total_ms = float(t.item())
+    total_launches = int(tl.item())
+    cells_per_step = w * h * n
+    value = cells_per_step * args.steps / (total_ms / 1e3)
+    ms_per_step = total_ms / args.steps
+
+    # Dominant-kernel timing: CUDA events around every bulk launch on the
+    # launching stream (direct launches, same kernels/config) for one step.
+    grid.set_option(M.OPT_TIMING, 1)
+    grid.iterate(n)
+    bulk_ms, bulk_n, bnd_ms, bnd_n = M.mapsm_get_timing(grid.handle)
+    grid.set_option(M.OPT_TIMING, 0)
+    peak_gbs, peak_src = load_peaks()
+    bcell = wl["bcell"]
+    slab_cells = rows * w
+    if world == 1:
+        # whole step = back-to-back bulk launches: region time / launches, measured over the timed region
+        per_launch_s = (total_ms / 1e3) / max(1, launches)
+        achieved_region = bcell * slab_cells / per_launch_s / 1e9
+    else:
+        achieved_region = None
+    bulk_rows = rows if bnd_n == 0 else rows - 2 * wl["r"]
+    per_kernel_s = (bulk_ms / 1e3) / max(1, bulk_n)
+    achieved_kernel = bcell * bulk_rows * w / per_kernel_s / 1e9
+    achieved = achieved_region if achieved_region is not None else achieved_kernel
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tfile):
+        try:
+            traffic = json.load(open(tfile)).get(args.workload)
+        except Exception:
+            traffic = None
+    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak_gbs, "unit": "GB/s",
+                "frac": achieved / peak_gbs, "traffic": traffic,
+                "kernel": "life_step_kernel" if wl["op"] == "life" else "conv_step_kernel",
+                "bytes_per_cell_update": bcell, "algorithmic_bytes_per_launch": bcell * slab_cells,
+                "peak_source": peak_src, "achieved_events_per_launch_GBps": achieved_kernel,
+                "kernel_ms_per_launch": per_kernel_s * 1e3,
+                "frac_vs_8TBps_spec": achieved / 8000.0}
+    if wl["op"] == "conv":
+        # 9x9 is FP32-FMA bound; report the FMA-pipe fraction alongside
+        fma_per_cell = (2 * wl["r"] + 1) ** 2
+        sm_mhz = clocks.get("sm_mhz") or 1965.0
+        fma_peak = 148 * 128 * sm_mhz * 1e6
+        roofline["fma_frac_at_sampled_clock"] = (bulk_rows * w * fma_per_cell / per_kernel_s) / fma_peak
+
+    # halo-exchange exposure (N > 1): same steps without the exchange
+    exposure = None
+    if world > 1:
+        grid.set_option(M.OPT_NO_EXCHANGE, 1)
+        grid.iterate(n)
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        grid.iterate(n)
+        e1.record(stream)
+        barrier()
+        tt = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
+        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
+        grid.set_option(M.OPT_NO_EXCHANGE, 0)
+        exposure = {"ms_per_step_no_exchange": float(tt.item()),
+                    "exposed_pct": 100.0 * (ms_per_step - float(tt.item())) / ms_per_step}
+
+    # e2e: host buffers through the public API, copies inside the timed region
+    e2e_ms = 0.0
+    barrier()
+    for _ in range(args.e2e_steps):
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        barrier()
+        e0.record(stream)
+        grid.bind(h_in)
+        grid.iterate(n)
+        M.mapsm_read(grid.handle, h_out)
+        e1.record(stream)
+        e1.synchronize()
+        e2e_ms += e0.elapsed_time(e1)
+    te = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_value = cells_per_step * args.e2e_steps / (float(te.item()) / 1e3)
+    elem = 1 if wl["op"] == "life" else 4
+
+    grid.close()
+    M.mapsm_ctx_destroy(ctx)
+
+    if rank == 0:
+        cb = None if args.no_cpu_baseline else cpu_baseline(wl)
+        ws_mib = 2 * (rows + 2 * wl["r"]) * info0.pitch_bytes / 2**20
+        metric = ("Game of Life cell-updates/s" if wl["op"] == "life"
+                  else f"fp32 {2*wl['r']+1}x{2*wl['r']+1} window-conv cell-updates/s")
+        line = {
+            "metric": metric, "value": value, "unit": "cell-updates/s", "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+            "scaling": wl["scaling"], "vs_baseline": None,
+            "dtype": "u32 bit-sliced (1 bit/cell)" if wl["op"] == "life" else "f32",
+            "data": "synthetic",
+            "config": {"workload": wl["label"], "w": w, "h": h, "iterations_per_step": n, "radius": wl["r"],
+                       "boundary": wl["b"], "parallelism": f"row-slab x{world}" + (" + NCCL halo exchange" if world > 1 else ""),
+                       "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU double-buffer "
+                             f"working set {ws_mib:.0f} MiB vs 126 MB L2",
+                       "cuda_graphs": used_graphs},
+            "e2e": {"value": e2e_value, "unit": "cell-updates/s", "h2d_bytes_per_step": h * w * elem,
+                    "d2h_bytes_per_step": h * w * elem,
+                    "how": "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step"},
+            "gpu_launches": total_launches,
+            "roofline": roofline,
+            "clocks": clocks,
+            "cpu_baseline": cb,
+        }
+        if exposure is not None:
+            line["halo_exposure"] = exposure
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier(device_ids=[local_rank])
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

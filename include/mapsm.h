@@ -1,0 +1,230 @@
+/*
+ * mapsm.h — C ABI of libmapsm, the B200-native Window(2D) -> Structured-
+ * Injective stencil path of MAPS-Multi (Ben-Nun, Levy, Rubin, Barak, SC'15).
+ *
+ * Citations: "P:L<n> §<s>" = line n of the paper text, section s.
+ *
+ * What the library does (BASELINE.json north_star; §2.1
+ * §4, Fig 2): an iterated radius-r 2D stencil over a double-
+ * buffered grid ("two matrices are used as input and output buffers in
+ * alternating succession"), row-slab-partitioned over g GPUs ("task
+ * partitioning ... evenly distributing the thread-blocks among the devices",
+ * P:L59), with the r halo rows the Window pattern implies exchanged between
+ * neighbouring slabs every iteration ("two-line boundary exchanges per
+ * iteration").  Two operators:
+ *   - MAPSM_OP_LIFE: Conway's Game of Life, B3/S23 on the 3x3 window (P:L133,
+ *     Gardner [14] P:L619), radius 1, u8 cells on the host (nonzero = alive),
+ *     bit-packed 32 cells per 32-bit word on the device;
+ *   - MAPSM_OP_CONV: fp32 window convolution (Table 1, "N-dimensional
+ *     convolution"), cross-correlation with (2r+1)^2 row-major weights,
+ *     1 <= r <= 4, one fmaf per tap in row-major (dy, dx) order starting from
+ *     +0.0f (reading c11) so results are reproducible bit for bit.
+ * Boundaries (the Window container's "boundary condition management",
+ * P:L115; WRAP is the paper's GoL mode): WRAP = torus on both axes,
+ * CLAMP = replicate the nearest edge cell, ZERO = constant 0 outside.
+ *
+ * Paper API -> this ABI (Table 2):
+ *   Matrix<T> A,B + Bind            -> mapsm_grid_create + mapsm_bind
+ *   Scheduler::AnalyzeCall x2       -> mapsm_window_set (partition + allocate
+ *                                      both buffers with halos)
+ *   Scheduler::Invoke (per iter)    -> mapsm_iterate(n)  (asynchronous)
+ *   Wait / WaitAll                  -> mapsm_sync
+ *   Gather (A if n even, else B)    -> mapsm_gather (always generation n)
+ *
+ * Conventions (all entry points):
+ *   - Every call returns a mapsm_status; MAPSM_OK == 0.  No C++ exception
+ *     crosses the ABI.  mapsm_last_error() gives a thread-local message for
+ *     the most recent failure on the calling thread.
+ *   - Handles are opaque; a ctx must outlive its grids.  A grid owns all of its
+ *     device memory (two slab buffers per local slab, each (rows + 2r) rows).
+ *   - Host pointers are borrowed only for the duration of the call (data is
+ *     copied).  "ptr" arguments accept host memory (pageable or pinned) or
+ *     device memory on the slab's device; the kind is detected with
+ *     cudaPointerGetAttributes.  Row pitches are in bytes.
+ *   - State machine: grid_create -> window_set -> op_set -> bind ->
+ *     (iterate)* -> sync/gather/read -> destroy.  Out-of-order calls return
+ *     MAPSM_ESTATE (e.g. window_set after bind: the allocation depends on r,
+ *     like AnalyzeCall before Invoke).  Re-binding is allowed.
+ *   - Multi-process mode (one process per GPU, NCCL over NVLink): bind,
+ *     iterate, gather are collective — every rank calls them with the same
+ *     arguments (n).  One host thread per ctx; no internal locking.
+ *   - Asynchronous CUDA/NCCL errors surface at mapsm_sync / mapsm_gather /
+ *     mapsm_read.
+ */
+#ifndef MAPSM_H
+#define MAPSM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+    MAPSM_OK = 0,
+    MAPSM_EINVAL = -1,       /* bad argument (sizes, pointers, radius, pitch) */
+    MAPSM_ENOMEM = -2,       /* device or host allocation failed */
+    MAPSM_ECUDA = -3,        /* CUDA runtime / kernel error */
+    MAPSM_ENCCL = -4,        /* NCCL missing or failed */
+    MAPSM_ESTATE = -5,       /* call out of order for this handle */
+    MAPSM_EUNSUPPORTED = -6  /* valid but not supported (dtype/op/radius combo) */
+} mapsm_status;
+
+typedef enum { MAPSM_U8 = 1, MAPSM_F32 = 2 } mapsm_dtype;
+typedef enum { MAPSM_WRAP = 0, MAPSM_CLAMP = 1, MAPSM_ZERO = 2 } mapsm_boundary;
+typedef enum { MAPSM_OP_LIFE = 0, MAPSM_OP_CONV = 1 } mapsm_op;
+
+/* How a slab obtains the r rows just above (top) / below (bottom) its owned
+ * rows — the Segment Location Monitor's answer (Alg 2) for this path. */
+typedef enum {
+    MAPSM_HALO_EXCHANGE = 0,   /* received from a neighbour slab every iteration */
+    MAPSM_HALO_WRAP_LOCAL = 1, /* g == 1 under WRAP: the slab's own far rows (no copy) */
+    MAPSM_HALO_CLAMP = 2,      /* global edge under CLAMP: replicate the edge row (no copy) */
+    MAPSM_HALO_ZERO = 3        /* global edge under ZERO: zero rows written once at bind */
+} mapsm_halo_kind;
+
+typedef struct mapsm_ctx_s* mapsm_ctx;
+typedef struct mapsm_grid_s* mapsm_grid;
+
+/* ------------------------------------------------------------ partition plan
+ * Pure host arithmetic (the Segmenter + Memory Analyzer + static Location
+ * Monitor, Alg 2).  Needs no GPU.
+ * For slab `rank` of g over h rows with radius r:
+ *   rows = floor(h/g) + (rank < h mod g),  y0 = sum_{j<rank} rows_j
+ *   up = (rank-1) mod g, down = (rank+1) mod g (WRAP); -1 at the global edge
+ *   under CLAMP/ZERO.  top halo = global rows [y0-r, y0), bottom halo =
+ *   [y0+rows, y0+rows+r), taken mod h under WRAP.
+ * Requires g >= 1, h >= 1, 0 <= r, and when g > 1: rows_j >= r for all j
+ * (so each halo row has exactly one owner, the neighbour) — else EINVAL.   */
+typedef struct {
+    int64_t y0, rows;              /* owned global rows [y0, y0+rows) */
+    int up, down;                  /* neighbour slab ranks, -1 if none */
+    int top_kind, bottom_kind;     /* mapsm_halo_kind */
+    int64_t top_src_row;           /* global row of the first top-halo row's source (-1 if none) */
+    int64_t bottom_src_row;        /* global row of the first bottom-halo row's source (-1 if none) */
+    int n_send, n_recv;            /* halo messages per iteration (each r rows) */
+    int64_t alloc_rows;            /* rows allocated per buffer = rows + 2r */
+} mapsm_slab_plan;
+
+mapsm_status mapsm_plan_query(int64_t h, int g, int radius, mapsm_boundary boundary, int rank,
+                              mapsm_slab_plan* out);
+
+/* ------------------------------------------------------------------- context */
+
+/* Multi-process mode: one process (rank of world) per GPU.  `nccl_unique_id`
+ * is the 128-byte ncclUniqueId from mapsm_nccl_unique_id() on rank 0,
+ * broadcast by the caller (e.g. torch.distributed); NULL iff world == 1.
+ * `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream().cuda_stream)
+ * becomes the compute stream; NULL -> the library creates its own.  The
+ * exchange runs on a library-owned side stream.                             */
+mapsm_status mapsm_ctx_create(int rank, int world, int device, const void* nccl_unique_id,
+                              void* cuda_stream, mapsm_ctx* out);
+
+/* Single-process mode (the paper's own model: one process driving g devices
+ * with host-initiated peer copies): g slabs on devices[i]
+ * (entries may repeat, e.g. g slabs on one GPU); halos move with
+ * cudaMemcpyAsync peer/device copies instead of NCCL.                       */
+mapsm_status mapsm_ctx_create_local(int nslabs, const int* devices, mapsm_ctx* out);
+
+mapsm_status mapsm_ctx_destroy(mapsm_ctx ctx);
+
+/* Writes a fresh ncclUniqueId (128 bytes) to out128.  ENCCL if NCCL cannot be
+ * loaded (libnccl.so.2, the one torch ships, is dlopen'ed on first use).     */
+mapsm_status mapsm_nccl_unique_id(void* out128);
+
+/* ---------------------------------------------------------------------- grid */
+
+/* Declare a w x h datum.  dtype U8 for Life, F32 for conv.          */
+mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, mapsm_dtype dtype,
+                               mapsm_grid* out);
+
+/* Window(2D) pattern: radius and boundary.  Partitions the rows over
+ * the slabs and allocates both buffers of every local slab with 2r halo rows
+ * (the Memory Analyzer's bounding box after both AnalyzeCalls, P:L167-169,
+ * P:L281).  EUNSUPPORTED: Life with r != 1, conv with r outside 1..4.
+ * EINVAL: a slab would have fewer than r rows (g > 1), or Life with w % 64
+ * != 0.  ENOMEM on allocation failure.                                       */
+mapsm_status mapsm_window_set(mapsm_grid grid, int radius, mapsm_boundary boundary);
+
+/* Operator: LIFE (weights must be NULL, dtype U8) or CONV (weights = (2r+1)^2
+ * fp32 values, row-major over (dy, dx), copied; dtype F32).                  */
+mapsm_status mapsm_op_set(mapsm_grid grid, mapsm_op op, const float* weights);
+
+/* Owned rows of local slab `local_index` (0 in multi-process mode).          */
+mapsm_status mapsm_grid_slab(mapsm_grid grid, int local_index, int64_t* y0, int64_t* rows);
+
+/* Bind: upload this process's rows — global rows
+ * [y0 of its first local slab, end of its last) — from `ptr` (row pitch
+ * `row_pitch_bytes` >= w * elem_size) and fill the halos (one exchange).  Life
+ * bytes: nonzero = alive.  Resets the generation counter to 0.  Collective.  */
+mapsm_status mapsm_bind(mapsm_grid grid, const void* ptr, int64_t row_pitch_bytes);
+
+/* Enqueue n iterations (Invoke, Alg 1) on the compute stream(s)
+ * and return; n == 0 is a no-op.  Collective.                                */
+mapsm_status mapsm_iterate(mapsm_grid grid, int64_t n);
+
+/* Wait for all enqueued work (Wait/WaitAll, Table 2) and report async errors.*/
+mapsm_status mapsm_sync(mapsm_grid grid);
+
+/* Gather: write the full h x w generation-n grid
+ * to `ptr` on rank `root` (other ranks pass NULL).  Life output bytes are
+ * exactly 0/1.  Collective; synchronises.                                    */
+mapsm_status mapsm_gather(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, int root);
+
+/* Copy only this process's own rows (same row range as mapsm_bind) to `ptr`;
+ * not collective; synchronises.                                              */
+mapsm_status mapsm_read(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes);
+
+mapsm_status mapsm_grid_destroy(mapsm_grid grid);
+
+/* ----------------------------------------------------------- introspection */
+
+typedef struct {
+    int64_t w, h;
+    int dtype, op, radius, boundary;
+    int world;               /* g: total slabs over all processes */
+    int local_slabs;         /* slabs owned by this process */
+    int64_t pitch_bytes;     /* device row pitch */
+    int64_t generation;      /* iterations applied since bind */
+    int64_t launches;        /* kernels launched by this grid since bind (all slabs) */
+    int64_t exchanges;       /* halo messages received by this process since bind */
+    int64_t device_bytes;    /* device memory owned by the grid */
+    int used_graphs;         /* 1 if iterate replays CUDA graphs */
+} mapsm_grid_info;
+
+mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
+
+/* Options (set before the first iterate; values are int64):
+ *   MAPSM_OPT_GRAPHS      1 (default) capture iterations in CUDA graphs, 0 = direct launches
+ *   MAPSM_OPT_GRAPH_ITERS iterations per captured graph (even, default 16)
+ *   MAPSM_OPT_NO_EXCHANGE 1 = skip the halo exchange (bench only: measures
+ *                         exchange exposure; results are then WRONG for g > 1)
+ *   MAPSM_OPT_TIMING      1 = record CUDA events around every compute kernel
+ *                         (forces direct launches); read with mapsm_get_timing */
+typedef enum {
+    MAPSM_OPT_GRAPHS = 1,
+    MAPSM_OPT_GRAPH_ITERS = 2,
+    MAPSM_OPT_NO_EXCHANGE = 3,
+    MAPSM_OPT_TIMING = 4
+} mapsm_option;
+
+mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);
+
+/* With MAPSM_OPT_TIMING: summed device time (ms) and count of the bulk
+ * ("interior" / whole-slab) compute kernels and of the boundary-row kernels
+ * of local slab 0 since the option was set.  Synchronises.                   */
+mapsm_status mapsm_get_timing(mapsm_grid grid, double* bulk_ms, int64_t* bulk_launches,
+                              double* boundary_ms, int64_t* boundary_launches);
+
+/* The compute stream of local slab `local_index` (a cudaStream_t).           */
+mapsm_status mapsm_grid_stream(mapsm_grid grid, int local_index, void** stream);
+
+const char* mapsm_status_string(mapsm_status s);
+const char* mapsm_last_error(void);
+const char* mapsm_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* MAPSM_H */

@@ -1,0 +1,12 @@
+"""mapsm — B200-native Window(2D) -> Structured-Injective stencil path of
+MAPS-Multi (SC'15): Game of Life and fp32 window convolution, row-slab
+partitioned over GPUs with per-iteration halo exchange.
+
+The product is ``libmapsm.so`` (C ABI in ``include/mapsm.h``); this package is
+its thin ctypes binding (``mapsm``) and the multi-process bootstrap
+(``dist``).  There is no CPU fallback.
+"""
+from . import mapsm  # noqa: F401
+from .mapsm import Grid, MapsmError  # noqa: F401
+
+__all__ = ["mapsm", "Grid", "MapsmError"]

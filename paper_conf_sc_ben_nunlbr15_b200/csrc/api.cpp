@@ -1,0 +1,949 @@
+// api.cpp — host runtime of libmapsm behind the C ABI of include/mapsm.h.
+//
+// Paper components (§4, Fig 1a) and what replaces them here:
+//   Scheduler + Alg 1  -> mapsm_iterate: per iteration, per slab,
+//       boundary-row kernel -> event -> halo exchange on a side stream, while
+//       the interior kernel runs on the compute stream; the compute stream
+//       waits for the exchange before the next iteration ("segment ready"
+//       events, Alg 1 lines 16/20).  Iterations are captured in CUDA graphs.
+//   Invoker threads        -> one process per GPU (NCCL mode) or one
+//       host thread issuing to per-slab streams (local mode).
+//   Memory Analyzer + Allocator     -> mapsm_window_set (plan.cpp + cudaMalloc
+//       of both buffers with 2r halo rows each, once).
+//   Location Monitor + Alg 2        -> the static halo plan (plan.cpp).
+//   P2P copies      -> ncclSend/ncclRecv over NVLink (NCCL
+//       mode) or cudaMemcpyAsync peer copies (local mode).
+#include <cuda_runtime.h>
+#include <dlfcn.h>
+
+#include <cstdarg>
+#include <cstdint>
+#include <cstdio>
+#include <cstring>
+#include <string>
+#include <vector>
+
+#include "../../include/mapsm.h"
+#include "kernels.h"
+#include "nccl.h"
+
+namespace mapsm {
+mapsm_status compute_plan(int64_t h, int g, int r, mapsm_boundary b, int rank, mapsm_slab_plan* out);
+}
+
+using namespace mapsm;
+
+// ----------------------------------------------------------------- errors
+
+static thread_local std::string g_last_error;
+
+static mapsm_status fail(mapsm_status s, const char* fmt, ...) {
+    char buf[512];
+    va_list ap;
+    va_start(ap, fmt);
+    vsnprintf(buf, sizeof buf, fmt, ap);
+    va_end(ap);
+    g_last_error = buf;
+    return s;
+}
+
+#define CK(expr)                                                                              \
+    do {                                                                                      \
+        cudaError_t e_ = (expr);                                                              \
+        if (e_ != cudaSuccess)                                                                \
+            return fail(e_ == cudaErrorMemoryAllocation ? MAPSM_ENOMEM : MAPSM_ECUDA,         \
+                        "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
+    } while (0)
+
+#define TRY(expr)                          \
+    do {                                   \
+        mapsm_status s_ = (expr);          \
+        if (s_ != MAPSM_OK) return s_;     \
+    } while (0)
+
+// Restores the caller's current device on scope exit (torch relies on it).
+struct DeviceGuard {
+    int prev = -1;
+    DeviceGuard() { cudaGetDevice(&prev); }
+    ~DeviceGuard() {
+        if (prev >= 0) cudaSetDevice(prev);
+    }
+};
+
+// ------------------------------------------------------------------- NCCL
+// Loaded on first use with dlopen("libnccl.so.2"): inside a torch process this
+// resolves to the NCCL torch already loaded (one NCCL per process).
+
+struct NcclApi {
+    void* h = nullptr;
+    decltype(&ncclGetUniqueId) getUniqueId = nullptr;
+    decltype(&ncclCommInitRank) commInitRank = nullptr;
+    decltype(&ncclCommDestroy) commDestroy = nullptr;
+    decltype(&ncclCommAbort) commAbort = nullptr;
+    decltype(&ncclCommGetAsyncError) commGetAsyncError = nullptr;
+    decltype(&ncclSend) send = nullptr;
+    decltype(&ncclRecv) recv = nullptr;
+    decltype(&ncclGroupStart) groupStart = nullptr;
+    decltype(&ncclGroupEnd) groupEnd = nullptr;
+    decltype(&ncclGetErrorString) errStr = nullptr;
+};
+static NcclApi g_nccl;
+
+static mapsm_status nccl_load() {
+    if (g_nccl.h) return MAPSM_OK;
+    void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
+    if (!h) return fail(MAPSM_ENCCL, "dlopen(libnccl.so.2) failed: %s", dlerror());
+#define SYM(field, name)                                                              \
+    g_nccl.field = reinterpret_cast<decltype(g_nccl.field)>(dlsym(h, name));          \
+    if (!g_nccl.field) return fail(MAPSM_ENCCL, "NCCL symbol %s missing", name);
+    SYM(getUniqueId, "ncclGetUniqueId");
+    SYM(commInitRank, "ncclCommInitRank");
+    SYM(commDestroy, "ncclCommDestroy");
+    SYM(commAbort, "ncclCommAbort");
+    SYM(commGetAsyncError, "ncclCommGetAsyncError");
+    SYM(send, "ncclSend");
+    SYM(recv, "ncclRecv");
+    SYM(groupStart, "ncclGroupStart");
+    SYM(groupEnd, "ncclGroupEnd");
+    SYM(errStr, "ncclGetErrorString");
+#undef SYM
+    g_nccl.h = h;
+    return MAPSM_OK;
+}
+
+#define NK(expr)                                                                              \
+    do {                                                                                      \
+        ncclResult_t r_ = (expr);                                                             \
+        if (r_ != ncclSuccess)                                                                \
+            return fail(MAPSM_ENCCL, "%s failed: %s", #expr, g_nccl.errStr(r_));              \
+    } while (0)
+
+// ---------------------------------------------------------------- objects
+
+struct mapsm_ctx_s {
+    bool local = false;            // single-process multi-slab mode
+    int rank = 0, world = 1;       // process rank / count (multi-process mode)
+    int g = 1;                     // total slabs
+    int first_slab = 0;            // global index of local slab 0
+    std::vector<int> devices;      // device per local slab
+    cudaStream_t user_stream = nullptr;
+    ncclComm_t comm = nullptr;
+    int live_grids = 0;
+};
+
+struct TimingPair {
+    cudaEvent_t a, b;
+};
+
+struct Slab {
+    int rank = 0;      // global slab index
+    int device = 0;
+    int num_sms = 148;
+    mapsm_slab_plan plan{};
+    char* base[2] = {nullptr, nullptr};  // allocation base (row -r)
+    cudaStream_t main = nullptr, side = nullptr;
+    bool own_main = false;
+    cudaEvent_t ev_b = nullptr, ev_h = nullptr;
+    cudaGraphExec_t graph[2] = {nullptr, nullptr};
+    int64_t graph_iters = 0;
+    void* staging = nullptr;   // device staging for host bind/gather (Life)
+    int64_t staging_bytes = 0;
+    std::vector<TimingPair> t_bulk, t_bnd;
+    size_t t_bulk_used = 0, t_bnd_used = 0;
+};
+
+enum GridState { ST_CREATED = 0, ST_WINDOW = 1, ST_OP = 2, ST_BOUND = 3 };
+
+struct mapsm_grid_s {
+    mapsm_ctx ctx = nullptr;
+    int64_t w = 0, h = 0;
+    mapsm_dtype dtype = MAPSM_U8;
+    int r = 0;
+    mapsm_boundary boundary = MAPSM_WRAP;
+    mapsm_op op = MAPSM_OP_LIFE;
+    float wt[81] = {0};
+    int state = ST_CREATED;
+    int64_t pitch = 0;
+    int64_t elem = 1;               // host bytes per cell
+    std::vector<Slab> slabs;
+    int cur = 0;                    // buffer holding the current generation
+    int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
+    bool opt_graphs = true, opt_no_exchange = false, opt_timing = false;
+    int64_t opt_graph_iters = 16;
+    bool used_graphs = false;
+};
+
+static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
+    return s.base[b] + (y + g->r) * g->pitch;
+}
+
+static bool has_exchange(const Slab& s) {
+    return s.plan.top_kind == MAPSM_HALO_EXCHANGE || s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+}
+
+static int rowmap_of(int kind) {
+    switch (kind) {
+        case MAPSM_HALO_WRAP_LOCAL: return ROWMAP_WRAP;
+        case MAPSM_HALO_CLAMP: return ROWMAP_CLAMP;
+        default: return ROWMAP_HALO;  // exchanged rows or zeroed rows
+    }
+}
+
+// ------------------------------------------------------------- context API
+
+extern "C" mapsm_status mapsm_nccl_unique_id(void* out128) {
+    if (!out128) return fail(MAPSM_EINVAL, "out128 is NULL");
+    TRY(nccl_load());
+    ncclUniqueId id;
+    NK(g_nccl.getUniqueId(&id));
+    static_assert(sizeof(ncclUniqueId) == 128, "ncclUniqueId size");
+    memcpy(out128, &id, sizeof id);
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_ctx_create(int rank, int world, int device, const void* nccl_unique_id,
+                                         void* cuda_stream, mapsm_ctx* out) {
+    if (!out) return fail(MAPSM_EINVAL, "out is NULL");
+    *out = nullptr;
+    if (world < 1 || rank < 0 || rank >= world) return fail(MAPSM_EINVAL, "bad rank %d / world %d", rank, world);
+    if ((world > 1) != (nccl_unique_id != nullptr))
+        return fail(MAPSM_EINVAL, "nccl_unique_id must be given iff world > 1");
+    int ndev = 0;
+    CK(cudaGetDeviceCount(&ndev));
+    if (device < 0 || device >= ndev) return fail(MAPSM_EINVAL, "device %d out of range (%d devices)", device, ndev);
+    DeviceGuard dg;
+    CK(cudaSetDevice(device));
+    auto* c = new mapsm_ctx_s();
+    c->local = false;
+    c->rank = rank;
+    c->world = world;
+    c->g = world;
+    c->first_slab = rank;
+    c->devices = {device};
+    c->user_stream = static_cast<cudaStream_t>(cuda_stream);
+    if (world > 1) {
+        mapsm_status s = nccl_load();
+        if (s != MAPSM_OK) {
+            delete c;
+            return s;
+        }
+        ncclUniqueId id;
+        memcpy(&id, nccl_unique_id, sizeof id);
+        ncclResult_t r = g_nccl.commInitRank(&c->comm, world, id, rank);
+        if (r != ncclSuccess) {
+            delete c;
+            return fail(MAPSM_ENCCL, "ncclCommInitRank failed: %s", g_nccl.errStr(r));
+        }
+    }
+    *out = c;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_ctx_create_local(int nslabs, const int* devices, mapsm_ctx* out) {
+    if (!out || !devices || nslabs < 1) return fail(MAPSM_EINVAL, "bad arguments");
+    *out = nullptr;
+    int ndev = 0;
+    CK(cudaGetDeviceCount(&ndev));
+    for (int i = 0; i < nslabs; ++i)
+        if (devices[i] < 0 || devices[i] >= ndev) return fail(MAPSM_EINVAL, "device %d out of range", devices[i]);
+    DeviceGuard dg;
+    // Peer access between distinct devices (host-initiated P2P copies).
+    for (int i = 0; i < nslabs; ++i)
+        for (int j = 0; j < nslabs; ++j) {
+            if (devices[i] == devices[j]) continue;
+            int can = 0;
+            CK(cudaDeviceCanAccessPeer(&can, devices[i], devices[j]));
+            if (can) {
+                CK(cudaSetDevice(devices[i]));
+                cudaError_t e = cudaDeviceEnablePeerAccess(devices[j], 0);
+                if (e != cudaSuccess && e != cudaErrorPeerAccessAlreadyEnabled)
+                    return fail(MAPSM_ECUDA, "cudaDeviceEnablePeerAccess: %s", cudaGetErrorString(e));
+                cudaGetLastError();
+            }
+        }
+    auto* c = new mapsm_ctx_s();
+    c->local = true;
+    c->g = nslabs;
+    c->devices.assign(devices, devices + nslabs);
+    *out = c;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_ctx_destroy(mapsm_ctx c) {
+    if (!c) return fail(MAPSM_EINVAL, "ctx is NULL");
+    if (c->live_grids > 0) return fail(MAPSM_ESTATE, "ctx still has %d grids", c->live_grids);
+    if (c->comm) g_nccl.commDestroy(c->comm);
+    delete c;
+    return MAPSM_OK;
+}
+
+// ---------------------------------------------------------------- grid API
+
+extern "C" mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, mapsm_dtype dtype,
+                                          mapsm_grid* out) {
+    if (!ctx || !out) return fail(MAPSM_EINVAL, "NULL argument");
+    *out = nullptr;
+    if (w < 1 || h < 1) return fail(MAPSM_EINVAL, "grid must be at least 1x1 (w=%lld h=%lld)", (long long)w, (long long)h);
+    if (dtype != MAPSM_U8 && dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "dtype %d", (int)dtype);
+    auto* g = new mapsm_grid_s();
+    g->ctx = ctx;
+    g->w = w;
+    g->h = h;
+    g->dtype = dtype;
+    g->elem = dtype == MAPSM_U8 ? 1 : 4;
+    g->op = dtype == MAPSM_U8 ? MAPSM_OP_LIFE : MAPSM_OP_CONV;
+    ctx->live_grids++;
+    *out = g;
+    return MAPSM_OK;
+}
+
+static void free_slab(Slab& s) {
+    cudaSetDevice(s.device);
+    for (int b = 0; b < 2; ++b)
+        if (s.base[b]) cudaFree(s.base[b]);
+    if (s.staging) cudaFree(s.staging);
+    for (int b = 0; b < 2; ++b)
+        if (s.graph[b]) cudaGraphExecDestroy(s.graph[b]);
+    for (auto& t : s.t_bulk) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
+    for (auto& t : s.t_bnd) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
+    if (s.ev_b) cudaEventDestroy(s.ev_b);
+    if (s.ev_h) cudaEventDestroy(s.ev_h);
+    if (s.side) cudaStreamDestroy(s.side);
+    if (s.own_main && s.main) cudaStreamDestroy(s.main);
+    s = Slab();
+}
+
+extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundary boundary) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "window_set after bind (allocation depends on r)");
+    if (boundary != MAPSM_WRAP && boundary != MAPSM_CLAMP && boundary != MAPSM_ZERO)
+        return fail(MAPSM_EINVAL, "boundary %d", (int)boundary);
+    if (g->dtype == MAPSM_U8) {
+        if (radius != 1) return fail(MAPSM_EUNSUPPORTED, "Life (u8) needs radius 1, got %d", radius);
+        if (g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
+    } else {
+        if (radius < 1 || radius > 4) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..4, got %d", radius);
+    }
+    mapsm_ctx c = g->ctx;
+    // validate the partition for every slab before allocating anything
+    for (int k = 0; k < c->g; ++k) {
+        mapsm_slab_plan p;
+        if (compute_plan(g->h, c->g, radius, boundary, k, &p) != MAPSM_OK)
+            return fail(MAPSM_EINVAL, "cannot split %lld rows over %d slabs with radius %d (need >= r rows each)",
+                        (long long)g->h, c->g, radius);
+    }
+    DeviceGuard dg;
+    for (auto& s : g->slabs) free_slab(s);
+    g->slabs.clear();
+    g->device_bytes = 0;
+    g->r = radius;
+    g->boundary = boundary;
+    const int64_t row_bytes = g->dtype == MAPSM_U8 ? g->w / 8 : g->w * 4;
+    const int64_t align = row_bytes >= 128 ? 128 : 16;
+    g->pitch = (row_bytes + align - 1) / align * align;
+    const int nloc = c->local ? c->g : 1;
+    g->slabs.resize(nloc);
+    for (int i = 0; i < nloc; ++i) {
+        Slab& s = g->slabs[i];
+        s.rank = c->local ? i : c->first_slab;
+        s.device = c->devices[c->local ? i : 0];
+        compute_plan(g->h, c->g, radius, boundary, s.rank, &s.plan);
+        CK(cudaSetDevice(s.device));
+        CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
+        const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
+        for (int b = 0; b < 2; ++b) {
+            cudaError_t e = cudaMalloc(&s.base[b], bytes);
+            if (e != cudaSuccess) {
+                cudaGetLastError();
+                for (auto& t : g->slabs) free_slab(t);
+                g->slabs.clear();
+                g->state = ST_CREATED;
+                return fail(MAPSM_ENOMEM, "cudaMalloc(%zu) on device %d: %s", bytes, s.device, cudaGetErrorString(e));
+            }
+            CK(cudaMemset(s.base[b], 0, bytes));  // ZERO halos are written once, here
+            g->device_bytes += (int64_t)bytes;
+        }
+        if (!c->local && c->user_stream) {
+            s.main = c->user_stream;
+            s.own_main = false;
+        } else {
+            CK(cudaStreamCreateWithFlags(&s.main, cudaStreamNonBlocking));
+            s.own_main = true;
+        }
+        CK(cudaStreamCreateWithFlags(&s.side, cudaStreamNonBlocking));
+        CK(cudaEventCreateWithFlags(&s.ev_b, cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&s.ev_h, cudaEventDisableTiming));
+    }
+    CK(cudaDeviceSynchronize());
+    g->state = ST_WINDOW;
+    if (g->dtype == MAPSM_U8) g->state = ST_OP;  // Life is the only u8 operator; op_set optional
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* weights) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    if (g->state < ST_WINDOW) return fail(MAPSM_ESTATE, "op_set before window_set");
+    if (op == MAPSM_OP_LIFE) {
+        if (g->dtype != MAPSM_U8) return fail(MAPSM_EUNSUPPORTED, "Life needs dtype U8");
+        if (weights) return fail(MAPSM_EINVAL, "Life takes no weights");
+    } else if (op == MAPSM_OP_CONV) {
+        if (g->dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "conv needs dtype F32");
+        if (!weights) return fail(MAPSM_EINVAL, "conv needs (2r+1)^2 weights");
+        const int k = 2 * g->r + 1;
+        memcpy(g->wt, weights, sizeof(float) * k * k);
+    } else {
+        return fail(MAPSM_EUNSUPPORTED, "op %d", (int)op);
+    }
+    g->op = op;
+    for (auto& s : g->slabs)
+        for (int b = 0; b < 2; ++b)
+            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+    if (g->state < ST_OP) g->state = ST_OP;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_grid_slab(mapsm_grid g, int i, int64_t* y0, int64_t* rows) {
+    if (!g || !y0 || !rows) return fail(MAPSM_EINVAL, "NULL argument");
+    if (g->state < ST_WINDOW) return fail(MAPSM_ESTATE, "grid_slab before window_set");
+    if (i < 0 || i >= (int)g->slabs.size()) return fail(MAPSM_EINVAL, "local slab %d out of range", i);
+    *y0 = g->slabs[i].plan.y0;
+    *rows = g->slabs[i].plan.rows;
+    return MAPSM_OK;
+}
+
+// ------------------------------------------------------------ halo exchange
+
+// Local mode: slab i pulls its halos of buffer b from its neighbours with
+// device/peer copies on its side stream, after the neighbours' ev_b.
+static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events) {
+    const int64_t bytes = (int64_t)g->r * g->pitch;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
+            Slab& u = g->slabs[s.plan.up];
+            if (wait_events) CK(cudaStreamWaitEvent(s.side, u.ev_b, 0));
+            CK(cudaMemcpyAsync(row_ptr(g, s, b, -g->r), row_ptr(g, u, b, u.plan.rows - g->r), bytes,
+                               cudaMemcpyDefault, s.side));
+            g->exchanges++;
+        }
+        if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
+            Slab& d = g->slabs[s.plan.down];
+            if (wait_events) CK(cudaStreamWaitEvent(s.side, d.ev_b, 0));
+            CK(cudaMemcpyAsync(row_ptr(g, s, b, s.plan.rows), row_ptr(g, d, b, 0), bytes, cudaMemcpyDefault,
+                               s.side));
+            g->exchanges++;
+        }
+        CK(cudaEventRecord(s.ev_h, s.side));
+    }
+    return MAPSM_OK;
+}
+
+// NCCL mode: one group per iteration, issued on the side stream in the fixed
+// order send-up, send-down, recv-bottom (from down), recv-top (from up): with
+// g == 2 under WRAP both neighbours are the same peer, and this order makes
+// the peer's first recv (its bottom halo) match my first send (my top rows).
+static mapsm_status exchange_nccl(mapsm_grid_s* g, int b) {
+    Slab& s = g->slabs[0];
+    const size_t bytes = (size_t)g->r * (size_t)g->pitch;
+    NK(g_nccl.groupStart());
+    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
+        NK(g_nccl.send(row_ptr(g, s, b, 0), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
+    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
+        NK(g_nccl.send(row_ptr(g, s, b, s.plan.rows - g->r), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
+    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
+        NK(g_nccl.recv(row_ptr(g, s, b, s.plan.rows), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
+    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
+        NK(g_nccl.recv(row_ptr(g, s, b, -g->r), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
+    NK(g_nccl.groupEnd());
+    g->exchanges += s.plan.n_recv;
+    return MAPSM_OK;
+}
+
+// ------------------------------------------------------------- compute step
+
+static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk) {
+    StencilGeom geom;
+    geom.in = row_ptr(g, s, b_in, 0);
+    geom.out = row_ptr(g, s, b_in ^ 1, 0);
+    geom.pitch = g->pitch;
+    geom.rows = s.plan.rows;
+    geom.w = g->w;
+    geom.top_map = rowmap_of(s.plan.top_kind);
+    geom.bot_map = rowmap_of(s.plan.bottom_kind);
+    geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+    TimingPair* tp = nullptr;
+    if (g->opt_timing && &s == &g->slabs[0]) {
+        auto& vec = bulk ? s.t_bulk : s.t_bnd;
+        size_t& used = bulk ? s.t_bulk_used : s.t_bnd_used;
+        if (used == vec.size()) {
+            TimingPair t;
+            CK(cudaEventCreate(&t.a));
+            CK(cudaEventCreate(&t.b));
+            vec.push_back(t);
+        }
+        tp = &vec[used++];
+        CK(cudaEventRecord(tp->a, s.main));
+    }
+    cudaError_t e;
+    if (g->op == MAPSM_OP_LIFE)
+        e = launch_life_step(geom, bands, s.num_sms, s.main);
+    else
+        e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main);
+    if (e != cudaSuccess) return fail(MAPSM_ECUDA, "stencil launch: %s", cudaGetErrorString(e));
+    if (tp) CK(cudaEventRecord(tp->b, s.main));
+    g->launches++;
+    return MAPSM_OK;
+}
+
+// Output-row bands: rows sent to neighbours (boundary) and the rest (interior).
+static void split_bands(const mapsm_grid_s* g, const Slab& s, RowBands& bnd, RowBands& inner) {
+    const int64_t rows = s.plan.rows, r = g->r;
+    const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+    bnd.nbands = inner.nbands = 0;
+    if (rows <= 2 * r) {  // tiny slab: everything is boundary
+        bnd.begin[0] = 0; bnd.end[0] = rows; bnd.nbands = 1;
+        return;
+    }
+    if (top) { bnd.begin[bnd.nbands] = 0; bnd.end[bnd.nbands] = r; bnd.nbands++; }
+    if (bot) { bnd.begin[bnd.nbands] = rows - r; bnd.end[bnd.nbands] = rows; bnd.nbands++; }
+    inner.begin[0] = top ? r : 0;
+    inner.end[0] = bot ? rows - r : rows;
+    inner.nbands = 1;
+}
+
+// One iteration for all local slabs, reading buffer b_in.
+static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
+    mapsm_ctx c = g->ctx;
+    const bool exch = !g->opt_no_exchange;
+    bool any_exchange = false;
+    for (auto& s : g->slabs) any_exchange |= has_exchange(s);
+    if (!any_exchange) {
+        for (auto& s : g->slabs) {
+            CK(cudaSetDevice(s.device));
+            RowBands all;
+            all.nbands = 1;
+            all.begin[0] = 0;
+            all.end[0] = s.plan.rows;
+            TRY(launch_step(g, s, b_in, all, true));
+        }
+        return MAPSM_OK;
+    }
+    std::vector<RowBands> inner(g->slabs.size());
+    // 1. boundary rows first (they are what the neighbours wait for)
+    for (size_t i = 0; i < g->slabs.size(); ++i) {
+        Slab& s = g->slabs[i];
+        CK(cudaSetDevice(s.device));
+        RowBands bnd;
+        split_bands(g, s, bnd, inner[i]);
+        TRY(launch_step(g, s, b_in, bnd, false));
+        CK(cudaEventRecord(s.ev_b, s.main));
+    }
+    // 2. halo exchange of the freshly computed rows on the side streams
+    if (exch) {
+        if (c->local) {
+            TRY(exchange_local(g, b_in ^ 1, true));
+        } else {
+            Slab& s = g->slabs[0];
+            CK(cudaStreamWaitEvent(s.side, s.ev_b, 0));
+            TRY(exchange_nccl(g, b_in ^ 1));
+            CK(cudaEventRecord(s.ev_h, s.side));
+        }
+    }
+    // 3. interior rows overlap the exchange; then join before the next step
+    for (size_t i = 0; i < g->slabs.size(); ++i) {
+        Slab& s = g->slabs[i];
+        CK(cudaSetDevice(s.device));
+        if (inner[i].nbands > 0 && inner[i].end[0] > inner[i].begin[0]) TRY(launch_step(g, s, b_in, inner[i], true));
+        if (exch) CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
+    }
+    return MAPSM_OK;
+}
+
+static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters) {
+    CK(cudaSetDevice(s.device));
+    const int64_t l0 = g->launches, x0 = g->exchanges;
+    CK(cudaStreamBeginCapture(s.main, cudaStreamCaptureModeThreadLocal));
+    mapsm_status st = MAPSM_OK;
+    int cur = start_cur;
+    for (int64_t k = 0; k < iters && st == MAPSM_OK; ++k) {
+        st = iterate_once(g, cur);
+        cur ^= 1;
+    }
+    cudaGraph_t graph = nullptr;
+    cudaError_t e = cudaStreamEndCapture(s.main, &graph);
+    g->launches = l0;
+    g->exchanges = x0;
+    if (st != MAPSM_OK) {
+        if (graph) cudaGraphDestroy(graph);
+        return st;
+    }
+    if (e != cudaSuccess) return fail(MAPSM_ECUDA, "graph capture: %s", cudaGetErrorString(e));
+    e = cudaGraphInstantiate(&s.graph[start_cur], graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) return fail(MAPSM_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
+    s.graph_iters = iters;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "iterate before bind");
+    if (n < 0) return fail(MAPSM_EINVAL, "n < 0");
+    if (n == 0) return MAPSM_OK;
+    DeviceGuard dg;
+    // CUDA graphs for the single-stream-per-process modes (g == 1 and NCCL);
+    // local multi-slab mode issues directly (it is the single-GPU test vehicle).
+    const bool graphs = g->opt_graphs && !g->opt_timing && !g->ctx->local;
+    int64_t done = 0;
+    if (graphs) {
+        Slab& s = g->slabs[0];
+        int64_t gi = g->opt_graph_iters;
+        if (gi < 2) gi = 2;
+        if (gi % 2) gi++;
+        if (s.graph_iters != gi) {
+            for (int b = 0; b < 2; ++b)
+                if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+        }
+        int64_t per_graph_launches = 0, per_graph_exch = 0;
+        {
+            // launches per iteration (for the counters; graphs replay them)
+            RowBands bnd, inner;
+            split_bands(g, s, bnd, inner);
+            per_graph_launches = has_exchange(s) ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0)) : 1;
+            per_graph_exch = (has_exchange(s) && !g->opt_no_exchange) ? s.plan.n_recv : 0;
+        }
+        while (n - done >= gi) {
+            if (!s.graph[g->cur]) TRY(capture_graph(g, s, g->cur, gi));
+            CK(cudaSetDevice(s.device));
+            CK(cudaGraphLaunch(s.graph[g->cur], s.main));
+            done += gi;
+            g->launches += per_graph_launches * gi;
+            g->exchanges += per_graph_exch * gi;
+            g->gen += gi;
+            g->used_graphs = true;
+            // gi is even: cur unchanged
+        }
+    }
+    for (; done < n; ++done) {
+        TRY(iterate_once(g, g->cur));
+        g->cur ^= 1;
+        g->gen++;
+    }
+    return MAPSM_OK;
+}
+
+static mapsm_status check_async(mapsm_grid_s* g) {
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaStreamSynchronize(s.main));
+        CK(cudaStreamSynchronize(s.side));
+    }
+    if (g->ctx->comm) {
+        ncclResult_t ar = ncclSuccess;
+        NK(g_nccl.commGetAsyncError(g->ctx->comm, &ar));
+        if (ar != ncclSuccess) return fail(MAPSM_ENCCL, "NCCL async error: %s", g_nccl.errStr(ar));
+    }
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_sync(mapsm_grid g) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    DeviceGuard dg;
+    return check_async(g);
+}
+
+// ------------------------------------------------------------- bind / read
+
+static bool is_device_ptr(const void* p, int* dev) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+        *dev = a.device;
+        return true;
+    }
+    return false;
+}
+
+static mapsm_status ensure_staging(Slab& s, int64_t bytes) {
+    if (s.staging_bytes >= bytes) return MAPSM_OK;
+    if (s.staging) cudaFree(s.staging);
+    s.staging = nullptr;
+    s.staging_bytes = 0;
+    CK(cudaMalloc(&s.staging, (size_t)bytes));
+    s.staging_bytes = bytes;
+    return MAPSM_OK;
+}
+
+static const int64_t kStagingBytes = 64ll << 20;
+
+extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch) {
+    if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
+    if (g->state < ST_OP) return fail(MAPSM_ESTATE, "bind before window_set/op_set");
+    if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch %lld < row bytes", (long long)pitch);
+    DeviceGuard dg;
+    int pdev = -1;
+    const bool on_dev = is_device_ptr(ptr, &pdev);
+    const int64_t y_first = g->slabs[0].plan.y0;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        for (int b = 0; b < 2; ++b)
+            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+        const char* src = static_cast<const char*>(ptr) + (s.plan.y0 - y_first) * pitch;
+        const int64_t rows = s.plan.rows;
+        if (g->dtype == MAPSM_F32) {
+            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->pitch, src, pitch, g->w * 4, rows, cudaMemcpyDefault,
+                                 s.main));
+        } else if (on_dev && pdev == s.device) {
+            CK(launch_pack_life(reinterpret_cast<const uint8_t*>(src), pitch, row_ptr(g, s, 0, 0), g->pitch, rows,
+                                g->w, s.main));
+        } else {
+            const int64_t spitch = (g->w + 15) / 16 * 16;
+            int64_t chunk = kStagingBytes / spitch;
+            if (chunk < 1) chunk = 1;
+            if (chunk > rows) chunk = rows;
+            TRY(ensure_staging(s, chunk * spitch));
+            for (int64_t y = 0; y < rows; y += chunk) {
+                const int64_t nr = (rows - y < chunk) ? rows - y : chunk;
+                CK(cudaMemcpy2DAsync(s.staging, spitch, src + y * pitch, pitch, g->w, nr, cudaMemcpyDefault, s.main));
+                CK(launch_pack_life(static_cast<const uint8_t*>(s.staging), spitch, row_ptr(g, s, 0, y), g->pitch, nr,
+                                    g->w, s.main));
+            }
+        }
+    }
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaStreamSynchronize(s.main));
+    }
+    g->cur = 0;
+    g->gen = 0;
+    g->launches = 0;
+    g->exchanges = 0;
+    g->state = ST_BOUND;
+    // Fill the halos of the current buffer once (the first exchange).
+    bool any = false;
+    for (auto& s : g->slabs) any |= has_exchange(s);
+    if (any) {
+        if (g->ctx->local) {
+            TRY(exchange_local(g, 0, false));
+        } else {
+            TRY(exchange_nccl(g, 0));
+        }
+        g->exchanges = 0;
+    }
+    return check_async(g);
+}
+
+// Copy owned rows of the current buffer of slab s to dst (pitch dpitch).
+static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitch, bool dst_on_dev) {
+    const int64_t rows = s.plan.rows;
+    if (g->dtype == MAPSM_F32) {
+        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->pitch, g->w * 4, rows, cudaMemcpyDefault,
+                             s.main));
+        return MAPSM_OK;
+    }
+    if (dst_on_dev) {
+        CK(launch_unpack_life(row_ptr(g, s, g->cur, 0), g->pitch, reinterpret_cast<uint8_t*>(dst), dpitch, rows, g->w,
+                              s.main));
+        return MAPSM_OK;
+    }
+    const int64_t spitch = (g->w + 15) / 16 * 16;
+    int64_t chunk = kStagingBytes / spitch;
+    if (chunk < 1) chunk = 1;
+    if (chunk > rows) chunk = rows;
+    TRY(ensure_staging(s, chunk * spitch));
+    for (int64_t y = 0; y < rows; y += chunk) {
+        const int64_t nr = (rows - y < chunk) ? rows - y : chunk;
+        CK(launch_unpack_life(row_ptr(g, s, g->cur, y), g->pitch, static_cast<uint8_t*>(s.staging), spitch, nr, g->w,
+                              s.main));
+        CK(cudaMemcpy2DAsync(dst + y * dpitch, dpitch, s.staging, spitch, g->w, nr, cudaMemcpyDefault, s.main));
+    }
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_read(mapsm_grid g, void* ptr, int64_t pitch) {
+    if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
+    if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "read before bind");
+    if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch too small");
+    DeviceGuard dg;
+    int pdev = -1;
+    const bool on_dev = is_device_ptr(ptr, &pdev);
+    const int64_t y_first = g->slabs[0].plan.y0;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        char* dst = static_cast<char*>(ptr) + (s.plan.y0 - y_first) * pitch;
+        TRY(read_slab(g, s, dst, pitch, on_dev && pdev == s.device));
+    }
+    return check_async(g);
+}
+
+extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int root) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "gather before bind");
+    mapsm_ctx c = g->ctx;
+    if (root < 0 || root >= c->world) return fail(MAPSM_EINVAL, "root %d", root);
+    if (c->world == 1) {
+        if (!ptr) return fail(MAPSM_EINVAL, "ptr is NULL");
+        return mapsm_read(g, ptr, pitch);
+    }
+    if (c->rank == root && (!ptr || pitch < g->w * g->elem)) return fail(MAPSM_EINVAL, "root needs ptr and pitch");
+    DeviceGuard dg;
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    TRY(check_async(g));
+    const int64_t slab_bytes_row = g->pitch;
+    if (c->rank != root) {
+        NK(g_nccl.send(row_ptr(g, s, g->cur, 0), (size_t)(s.plan.rows * slab_bytes_row), ncclUint8, root, c->comm,
+                       s.main));
+        return check_async(g);
+    }
+    int pdev = -1;
+    const bool on_dev = is_device_ptr(ptr, &pdev) && pdev == s.device;
+    // Root: receive each slab into a temporary buffer, then unpack / copy out.
+    mapsm_slab_plan pk;
+    compute_plan(g->h, c->g, g->r, g->boundary, 0, &pk);
+    const int64_t max_rows = pk.rows;  // slab 0 is never shorter than any other
+    char* tmp = nullptr;
+    CK(cudaMalloc(&tmp, (size_t)(max_rows * slab_bytes_row)));
+    mapsm_status st = MAPSM_OK;
+    for (int k = 0; k < c->world && st == MAPSM_OK; ++k) {
+        compute_plan(g->h, c->g, g->r, g->boundary, k, &pk);
+        char* dst = static_cast<char*>(ptr) + pk.y0 * pitch;
+        if (k == root) {
+            st = read_slab(g, s, dst, pitch, on_dev);
+            continue;
+        }
+        ncclResult_t r = g_nccl.recv(tmp, (size_t)(pk.rows * slab_bytes_row), ncclUint8, k, c->comm, s.main);
+        if (r != ncclSuccess) {
+            st = fail(MAPSM_ENCCL, "gather recv from %d: %s", k, g_nccl.errStr(r));
+            break;
+        }
+        // Reuse read_slab's copy-out path on a view of the received rows.
+        Slab view = s;
+        view.plan = pk;
+        view.base[g->cur] = tmp - (int64_t)g->r * g->pitch;
+        view.staging = s.staging;
+        view.staging_bytes = s.staging_bytes;
+        st = read_slab(g, view, dst, pitch, on_dev);
+        s.staging = view.staging;  // staging may have been (re)allocated
+        s.staging_bytes = view.staging_bytes;
+        view.staging = nullptr;
+        view.graph[0] = view.graph[1] = nullptr;
+        cudaError_t e = cudaStreamSynchronize(s.main);
+        if (e != cudaSuccess && st == MAPSM_OK) st = fail(MAPSM_ECUDA, "gather: %s", cudaGetErrorString(e));
+    }
+    cudaStreamSynchronize(s.main);
+    cudaFree(tmp);
+    if (st != MAPSM_OK) return st;
+    return check_async(g);
+}
+
+extern "C" mapsm_status mapsm_grid_destroy(mapsm_grid g) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    DeviceGuard dg;
+    for (auto& s : g->slabs) {
+        cudaSetDevice(s.device);
+        cudaStreamSynchronize(s.main);
+        cudaStreamSynchronize(s.side);
+        free_slab(s);
+    }
+    g->ctx->live_grids--;
+    delete g;
+    return MAPSM_OK;
+}
+
+// ----------------------------------------------------------- introspection
+
+extern "C" mapsm_status mapsm_get_info(mapsm_grid g, mapsm_grid_info* o) {
+    if (!g || !o) return fail(MAPSM_EINVAL, "NULL argument");
+    o->w = g->w;
+    o->h = g->h;
+    o->dtype = g->dtype;
+    o->op = g->op;
+    o->radius = g->r;
+    o->boundary = g->boundary;
+    o->world = g->ctx->g;
+    o->local_slabs = (int)g->slabs.size();
+    o->pitch_bytes = g->pitch;
+    o->generation = g->gen;
+    o->launches = g->launches;
+    o->exchanges = g->exchanges;
+    o->device_bytes = g->device_bytes;
+    o->used_graphs = g->used_graphs ? 1 : 0;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t v) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    switch (opt) {
+        case MAPSM_OPT_GRAPHS: g->opt_graphs = v != 0; break;
+        case MAPSM_OPT_GRAPH_ITERS:
+            if (v < 2) return fail(MAPSM_EINVAL, "graph iters must be >= 2");
+            g->opt_graph_iters = v;
+            break;
+        case MAPSM_OPT_NO_EXCHANGE: g->opt_no_exchange = v != 0; break;
+        case MAPSM_OPT_TIMING:
+            g->opt_timing = v != 0;
+            for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;
+            break;
+        default: return fail(MAPSM_EINVAL, "unknown option %d", (int)opt);
+    }
+    for (auto& s : g->slabs)
+        for (int b = 0; b < 2; ++b)
+            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_get_timing(mapsm_grid g, double* bulk_ms, int64_t* bulk_n, double* bnd_ms,
+                                         int64_t* bnd_n) {
+    if (!g || !bulk_ms || !bulk_n || !bnd_ms || !bnd_n) return fail(MAPSM_EINVAL, "NULL argument");
+    if (g->slabs.empty()) return fail(MAPSM_ESTATE, "no slabs");
+    DeviceGuard dg;
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    CK(cudaStreamSynchronize(s.main));
+    double t = 0;
+    for (size_t i = 0; i < s.t_bulk_used; ++i) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, s.t_bulk[i].a, s.t_bulk[i].b));
+        t += ms;
+    }
+    *bulk_ms = t;
+    *bulk_n = (int64_t)s.t_bulk_used;
+    t = 0;
+    for (size_t i = 0; i < s.t_bnd_used; ++i) {
+        float ms = 0;
+        CK(cudaEventElapsedTime(&ms, s.t_bnd[i].a, s.t_bnd[i].b));
+        t += ms;
+    }
+    *bnd_ms = t;
+    *bnd_n = (int64_t)s.t_bnd_used;
+    s.t_bulk_used = s.t_bnd_used = 0;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_grid_stream(mapsm_grid g, int i, void** stream) {
+    if (!g || !stream) return fail(MAPSM_EINVAL, "NULL argument");
+    if (i < 0 || i >= (int)g->slabs.size()) return fail(MAPSM_EINVAL, "local slab %d out of range", i);
+    *stream = g->slabs[i].main;
+    return MAPSM_OK;
+}
+
+extern "C" const char* mapsm_status_string(mapsm_status s) {
+    switch (s) {
+        case MAPSM_OK: return "MAPSM_OK";
+        case MAPSM_EINVAL: return "MAPSM_EINVAL";
+        case MAPSM_ENOMEM: return "MAPSM_ENOMEM";
+        case MAPSM_ECUDA: return "MAPSM_ECUDA";
+        case MAPSM_ENCCL: return "MAPSM_ENCCL";
+        case MAPSM_ESTATE: return "MAPSM_ESTATE";
+        case MAPSM_EUNSUPPORTED: return "MAPSM_EUNSUPPORTED";
+    }
+    return "MAPSM_UNKNOWN";
+}
+
+extern "C" const char* mapsm_last_error(void) { return g_last_error.c_str(); }
+
+extern "C" const char* mapsm_version(void) { return "mapsm 0.1 (sm_100a)"; }

@@ -1,0 +1,51 @@
+// kernels.h — launch interface between the host runtime (api.cpp) and the
+// sm_100a device kernels (life.cu, conv.cu).  Internal to libmapsm.
+#pragma once
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+namespace mapsm {
+
+// How a kernel maps an input row index y outside [0, rows) of its slab
+// (see mapsm_halo_kind in include/mapsm.h).
+enum RowMap : int {
+    ROWMAP_HALO = 0,   // read the slab buffer's halo row (exchanged, or zeroed for ZERO)
+    ROWMAP_WRAP = 1,   // g == 1 WRAP: y mod rows (no halo copy needed)
+    ROWMAP_CLAMP = 2   // global edge under CLAMP: nearest owned edge row
+};
+
+// Column boundary == the grid's boundary (columns are never split).
+enum ColMode : int { COL_WRAP = 0, COL_CLAMP = 1, COL_ZERO = 2 };
+
+// One stencil launch over a slab.  `in`/`out` point at owned row 0 of the
+// input/output slab buffers; halo rows live at rows -r..-1 and rows..rows+r-1.
+struct StencilGeom {
+    const void* in;
+    void* out;
+    int64_t pitch;   // bytes between rows (same for in and out)
+    int64_t rows;    // owned rows of the slab
+    int64_t w;       // columns (cells)
+    int top_map, bot_map, col_mode;
+};
+
+// Output-row bands computed by one launch (1 band = all rows or interior;
+// 2 bands = the boundary rows [0,r) and [rows-r,rows)).
+struct RowBands {
+    int64_t begin[2], end[2];
+    int nbands;
+};
+
+// Life (bit-packed: bit j of 32-bit word m of a row = column 32m + j).
+// `resident_warps` = warps the device keeps resident for this kernel
+// (persistent-style row chunking); 0 = compute from the occupancy API.
+cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s);
+cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, int64_t dst_pitch,
+                             int64_t rows, int64_t w, cudaStream_t s);
+cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst, int64_t dst_pitch,
+                               int64_t rows, int64_t w, cudaStream_t s);
+
+// fp32 window convolution, radius r in 1..4, weights (2r+1)^2 row-major.
+cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
+                             int num_sms, cudaStream_t s);
+
+}  // namespace mapsm

@@ -1,0 +1,310 @@
+"""Thin ctypes binding of libmapsm (include/mapsm.h) — argument marshalling only.
+
+Every function here has the name of the C entry point it wraps and raises
+``MapsmError`` on a non-OK status.  All compute happens in libmapsm's sm_100a
+kernels; there is no Python or CPU fallback: if ``libmapsm.so`` is missing
+the import fails loudly (build it with ``python -m
+paper_conf_sc_ben_nunlbr15_b200.build``).
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import numpy as np
+
+_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libmapsm.so")
+
+# enums (include/mapsm.h)
+OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
+U8, F32 = 1, 2
+WRAP, CLAMP, ZERO = 0, 1, 2
+OP_LIFE, OP_CONV = 0, 1
+HALO_EXCHANGE, HALO_WRAP_LOCAL, HALO_CLAMP, HALO_ZERO = 0, 1, 2, 3
+OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING = 1, 2, 3, 4
+
+BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO}
+
+EXPORTED = [
+    "mapsm_plan_query", "mapsm_ctx_create", "mapsm_ctx_create_local", "mapsm_ctx_destroy",
+    "mapsm_nccl_unique_id", "mapsm_grid_create", "mapsm_window_set", "mapsm_op_set", "mapsm_grid_slab",
+    "mapsm_bind", "mapsm_iterate", "mapsm_sync", "mapsm_gather", "mapsm_read", "mapsm_grid_destroy",
+    "mapsm_get_info", "mapsm_set_option", "mapsm_get_timing", "mapsm_grid_stream", "mapsm_status_string",
+    "mapsm_last_error", "mapsm_version",
+]
+
+
+class MapsmError(RuntimeError):
+    def __init__(self, status: int, where: str, detail: str):
+        super().__init__(f"{where}: {status} {detail}")
+        self.status = status
+
+
+class mapsm_slab_plan(ctypes.Structure):
+    _fields_ = [("y0", ctypes.c_int64), ("rows", ctypes.c_int64), ("up", ctypes.c_int), ("down", ctypes.c_int),
+                ("top_kind", ctypes.c_int), ("bottom_kind", ctypes.c_int), ("top_src_row", ctypes.c_int64),
+                ("bottom_src_row", ctypes.c_int64), ("n_send", ctypes.c_int), ("n_recv", ctypes.c_int),
+                ("alloc_rows", ctypes.c_int64)]
+
+
+class mapsm_grid_info(ctypes.Structure):
+    _fields_ = [("w", ctypes.c_int64), ("h", ctypes.c_int64), ("dtype", ctypes.c_int), ("op", ctypes.c_int),
+                ("radius", ctypes.c_int), ("boundary", ctypes.c_int), ("world", ctypes.c_int),
+                ("local_slabs", ctypes.c_int), ("pitch_bytes", ctypes.c_int64), ("generation", ctypes.c_int64),
+                ("launches", ctypes.c_int64), ("exchanges", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
+                ("used_graphs", ctypes.c_int)]
+
+
+_lib = None
+
+
+def lib() -> ctypes.CDLL:
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(_LIB_PATH):
+        raise ImportError(f"{_LIB_PATH} is missing: build it with `python -m paper_conf_sc_ben_nunlbr15_b200.build` "
+                          "(no CPU fallback exists)")
+    L = ctypes.CDLL(_LIB_PATH)
+    i64, ci, vp = ctypes.c_int64, ctypes.c_int, ctypes.c_void_p
+    P = ctypes.POINTER
+    sig = {
+        "mapsm_plan_query": [i64, ci, ci, ci, ci, P(mapsm_slab_plan)],
+        "mapsm_ctx_create": [ci, ci, ci, vp, vp, P(vp)],
+        "mapsm_ctx_create_local": [ci, P(ci), P(vp)],
+        "mapsm_ctx_destroy": [vp],
+        "mapsm_nccl_unique_id": [vp],
+        "mapsm_grid_create": [vp, i64, i64, ci, P(vp)],
+        "mapsm_window_set": [vp, ci, ci],
+        "mapsm_op_set": [vp, ci, vp],
+        "mapsm_grid_slab": [vp, ci, P(i64), P(i64)],
+        "mapsm_bind": [vp, vp, i64],
+        "mapsm_iterate": [vp, i64],
+        "mapsm_sync": [vp],
+        "mapsm_gather": [vp, vp, i64, ci],
+        "mapsm_read": [vp, vp, i64],
+        "mapsm_grid_destroy": [vp],
+        "mapsm_get_info": [vp, P(mapsm_grid_info)],
+        "mapsm_set_option": [vp, ci, i64],
+        "mapsm_get_timing": [vp, P(ctypes.c_double), P(i64), P(ctypes.c_double), P(i64)],
+        "mapsm_grid_stream": [vp, ci, P(vp)],
+    }
+    for name, args in sig.items():
+        f = getattr(L, name)
+        f.argtypes = args
+        f.restype = ci
+    L.mapsm_status_string.argtypes = [ci]
+    L.mapsm_status_string.restype = ctypes.c_char_p
+    L.mapsm_last_error.argtypes = []
+    L.mapsm_last_error.restype = ctypes.c_char_p
+    L.mapsm_version.argtypes = []
+    L.mapsm_version.restype = ctypes.c_char_p
+    _lib = L
+    return L
+
+
+def _check(status: int, where: str) -> None:
+    if status != OK:
+        L = lib()
+        raise MapsmError(status, where, f"{L.mapsm_status_string(status).decode()}: {L.mapsm_last_error().decode()}")
+
+
+def _ptr(buf) -> int:
+    """Address of a numpy array, torch tensor (host or device) or int."""
+    if isinstance(buf, int):
+        return buf
+    if isinstance(buf, np.ndarray):
+        return buf.ctypes.data
+    if hasattr(buf, "data_ptr"):
+        return buf.data_ptr()
+    raise TypeError(f"unsupported buffer type {type(buf)}")
+
+
+def _pitch(buf, default: int) -> int:
+    if isinstance(buf, np.ndarray):
+        return buf.strides[0]
+    if hasattr(buf, "stride") and hasattr(buf, "element_size"):
+        return buf.stride(0) * buf.element_size()
+    return default
+
+
+# ---------------------------------------------------------------- C-named API
+
+def mapsm_plan_query(h: int, g: int, radius: int, boundary: int, rank: int) -> mapsm_slab_plan:
+    p = mapsm_slab_plan()
+    _check(lib().mapsm_plan_query(h, g, radius, boundary, rank, ctypes.byref(p)), "mapsm_plan_query")
+    return p
+
+
+def mapsm_nccl_unique_id() -> bytes:
+    buf = ctypes.create_string_buffer(128)
+    _check(lib().mapsm_nccl_unique_id(buf), "mapsm_nccl_unique_id")
+    return buf.raw
+
+
+def mapsm_ctx_create(rank: int, world: int, device: int, nccl_unique_id: bytes | None = None,
+                     cuda_stream: int | None = None) -> int:
+    out = ctypes.c_void_p()
+    uid = ctypes.create_string_buffer(nccl_unique_id, 128) if nccl_unique_id is not None else None
+    _check(lib().mapsm_ctx_create(rank, world, device, uid, cuda_stream, ctypes.byref(out)), "mapsm_ctx_create")
+    return out.value
+
+
+def mapsm_ctx_create_local(devices) -> int:
+    arr = (ctypes.c_int * len(devices))(*devices)
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_ctx_create_local(len(devices), arr, ctypes.byref(out)), "mapsm_ctx_create_local")
+    return out.value
+
+
+def mapsm_ctx_destroy(ctx: int) -> None:
+    _check(lib().mapsm_ctx_destroy(ctx), "mapsm_ctx_destroy")
+
+
+def mapsm_grid_create(ctx: int, w: int, h: int, dtype: int) -> int:
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_grid_create(ctx, w, h, dtype, ctypes.byref(out)), "mapsm_grid_create")
+    return out.value
+
+
+def mapsm_window_set(grid: int, radius: int, boundary: int) -> None:
+    _check(lib().mapsm_window_set(grid, radius, boundary), "mapsm_window_set")
+
+
+def mapsm_op_set(grid: int, op: int, weights=None) -> None:
+    wptr = None
+    if weights is not None:
+        w = np.ascontiguousarray(weights, dtype=np.float32)
+        wptr = w.ctypes.data
+        _check(lib().mapsm_op_set(grid, op, wptr), "mapsm_op_set")
+        return
+    _check(lib().mapsm_op_set(grid, op, None), "mapsm_op_set")
+
+
+def mapsm_grid_slab(grid: int, local_index: int = 0) -> tuple[int, int]:
+    y0, rows = ctypes.c_int64(), ctypes.c_int64()
+    _check(lib().mapsm_grid_slab(grid, local_index, ctypes.byref(y0), ctypes.byref(rows)), "mapsm_grid_slab")
+    return y0.value, rows.value
+
+
+def mapsm_bind(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
+    _check(lib().mapsm_bind(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_bind")
+
+
+def mapsm_iterate(grid: int, n: int) -> None:
+    _check(lib().mapsm_iterate(grid, n), "mapsm_iterate")
+
+
+def mapsm_sync(grid: int) -> None:
+    _check(lib().mapsm_sync(grid), "mapsm_sync")
+
+
+def mapsm_gather(grid: int, buf, row_pitch_bytes: int | None = None, root: int = 0) -> None:
+    p = None if buf is None else _ptr(buf)
+    pitch = row_pitch_bytes or (0 if buf is None else _pitch(buf, 0))
+    _check(lib().mapsm_gather(grid, p, pitch, root), "mapsm_gather")
+
+
+def mapsm_read(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
+    _check(lib().mapsm_read(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read")
+
+
+def mapsm_grid_destroy(grid: int) -> None:
+    _check(lib().mapsm_grid_destroy(grid), "mapsm_grid_destroy")
+
+
+def mapsm_get_info(grid: int) -> mapsm_grid_info:
+    info = mapsm_grid_info()
+    _check(lib().mapsm_get_info(grid, ctypes.byref(info)), "mapsm_get_info")
+    return info
+
+
+def mapsm_set_option(grid: int, opt: int, value: int) -> None:
+    _check(lib().mapsm_set_option(grid, opt, value), "mapsm_set_option")
+
+
+def mapsm_get_timing(grid: int) -> tuple[float, int, float, int]:
+    a, b = ctypes.c_double(), ctypes.c_int64()
+    c, d = ctypes.c_double(), ctypes.c_int64()
+    _check(lib().mapsm_get_timing(grid, ctypes.byref(a), ctypes.byref(b), ctypes.byref(c), ctypes.byref(d)),
+           "mapsm_get_timing")
+    return a.value, b.value, c.value, d.value
+
+
+def mapsm_grid_stream(grid: int, local_index: int = 0) -> int:
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_grid_stream(grid, local_index, ctypes.byref(out)), "mapsm_grid_stream")
+    return out.value or 0
+
+
+def mapsm_version() -> str:
+    return lib().mapsm_version().decode()
+
+
+# ------------------------------------------------------------ convenience
+
+class Grid:
+    """One datum with its Window(2D) pattern — create -> window_set -> op_set ->
+    bind -> iterate -> gather, as in Fig 2a."""
+
+    def __init__(self, ctx: int, w: int, h: int, op: str = "life", radius: int = 1, boundary: str = "wrap",
+                 weights=None):
+        self.ctx, self.w, self.h = ctx, w, h
+        self.op = op
+        self.dtype = U8 if op == "life" else F32
+        self.handle = mapsm_grid_create(ctx, w, h, self.dtype)
+        try:
+            mapsm_window_set(self.handle, radius, BOUNDARY[boundary] if isinstance(boundary, str) else boundary)
+            if op == "life":
+                mapsm_op_set(self.handle, OP_LIFE, None)
+            else:
+                mapsm_op_set(self.handle, OP_CONV, weights)
+        except Exception:
+            mapsm_grid_destroy(self.handle)
+            raise
+
+    def local_rows(self) -> tuple[int, int]:
+        """(y0, rows) of this process's rows (all local slabs)."""
+        info = mapsm_get_info(self.handle)
+        y0, _ = mapsm_grid_slab(self.handle, 0)
+        ylast, rlast = mapsm_grid_slab(self.handle, info.local_slabs - 1)
+        return y0, ylast + rlast - y0
+
+    def bind(self, buf, pitch: int | None = None):
+        mapsm_bind(self.handle, buf, pitch)
+
+    def iterate(self, n: int):
+        mapsm_iterate(self.handle, n)
+
+    def sync(self):
+        mapsm_sync(self.handle)
+
+    def read(self, out=None):
+        y0, rows = self.local_rows()
+        if out is None:
+            out = np.empty((rows, self.w), dtype=np.uint8 if self.dtype == U8 else np.float32)
+        mapsm_read(self.handle, out)
+        return out
+
+    def gather(self, out=None, root: int = 0, rank: int = 0):
+        if out is None and rank == root:
+            out = np.empty((self.h, self.w), dtype=np.uint8 if self.dtype == U8 else np.float32)
+        mapsm_gather(self.handle, out, None, root)
+        return out
+
+    def info(self) -> mapsm_grid_info:
+        return mapsm_get_info(self.handle)
+
+    def set_option(self, opt: int, value: int):
+        mapsm_set_option(self.handle, opt, value)
+
+    def close(self):
+        if self.handle:
+            mapsm_grid_destroy(self.handle)
+            self.handle = None
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
