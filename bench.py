@@ -214,7 +214,10 @@ def main():
     dev = torch.device("cuda", local_rank)
     if world > 1:
         dist.init_process_group("nccl", device_id=dev)
-    stream = torch.cuda.current_stream()
+    # A dedicated (non-default) stream: libmapsm launches on it, and the CUDA
+    # events of the timed region are recorded on it.
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
     uid = None
     if world > 1:
         obj = [M.mapsm_nccl_unique_id() if rank == 0 else None]

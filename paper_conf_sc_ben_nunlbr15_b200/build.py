@@ -52,27 +52,34 @@ def needs_build() -> bool:
     return any(os.path.getmtime(p) > t for p in _deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and not needs_build():
+def build(force: bool = False, verbose: bool = False, out: str | None = None, csrc: str | None = None,
+          extra: list[str] | None = None) -> str:
+    """Build the library.  ``out``/``csrc``/``extra`` build a tuning variant
+    from another source tree with extra nvcc flags (tools/ only)."""
+    lib_path = out or LIB
+    if out is None and not force and not needs_build():
         return LIB
-    os.makedirs(OBJ, exist_ok=True)
+    src_dir = csrc or CSRC
+    obj_dir = os.path.join(os.path.dirname(lib_path), "_build") if out else OBJ
+    os.makedirs(obj_dir, exist_ok=True)
     nvcc = os.environ.get("NVCC", "nvcc")
-    incs = ["-I", INCLUDE, "-I", CSRC, "-I", _nccl_include()]
+    incs = ["-I", INCLUDE, "-I", src_dir, "-I", _nccl_include()]
     objs = []
-    for src in _sources():
-        obj = os.path.join(OBJ, os.path.basename(src) + ".o")
-        cmd = [nvcc, *ARCH, *NVFLAGS, *incs, "-c", src, "-o", obj]
+    srcs = sorted(glob.glob(os.path.join(src_dir, "*.cu")) + glob.glob(os.path.join(src_dir, "*.cpp")))
+    for src in srcs:
+        obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
+        cmd = [nvcc, *ARCH, *NVFLAGS, *(extra or []), *incs, "-c", src, "-o", obj]
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
         subprocess.check_call(cmd)
         objs.append(obj)
-    tmp = LIB + ".tmp"
+    tmp = lib_path + ".tmp"
     cmd = [nvcc, *ARCH, "-shared", "-o", tmp, *objs, "-ldl", "-lpthread"]
     if verbose:
         print(" ".join(cmd), file=sys.stderr)
     subprocess.check_call(cmd)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib_path)
+    return lib_path
 
 
 if __name__ == "__main__":

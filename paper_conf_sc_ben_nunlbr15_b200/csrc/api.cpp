@@ -23,7 +23,7 @@
 #include <string>
 #include <vector>
 
-#include "../../include/mapsm.h"
+#include "mapsm.h"
 #include "kernels.h"
 #include "nccl.h"
 

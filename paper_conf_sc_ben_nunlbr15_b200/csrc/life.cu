@@ -31,6 +31,18 @@ namespace {
 
 constexpr int kThreads = 256;
 constexpr unsigned kFull = 0xffffffffu;
+#ifndef MAPSM_LIFE_P
+#define MAPSM_LIFE_P 3
+#endif
+constexpr int kLifeP = MAPSM_LIFE_P;  // rows of loads in flight per lane
+#ifndef MAPSM_TMA_NS
+#define MAPSM_TMA_NS 24
+#endif
+constexpr int kTmaNS = MAPSM_TMA_NS;  // pipeline stages (rows in flight per CTA)
+#ifndef MAPSM_TMA_CTAS
+#define MAPSM_TMA_CTAS 0
+#endif
+constexpr int kTmaCtasPerSm = MAPSM_TMA_CTAS;  // 0 = 16 consumer warps per SM
 
 struct LifeParams {
     const uint32_t* in;   // owned row 0 of input
@@ -48,7 +60,8 @@ __device__ __forceinline__ uint32_t maj3(uint32_t a, uint32_t b, uint32_t c) {
     return (a & b) | (a & c) | (b & c);
 }
 
-__device__ __forceinline__ int64_t map_row(const LifeParams& p, int64_t y) {
+template <class Prm>
+__device__ __forceinline__ int64_t map_row(const Prm& p, int64_t y) {
     if (y < 0) {
         if (p.top_map == ROWMAP_WRAP) {
             y %= p.rows;
@@ -89,38 +102,43 @@ __device__ __forceinline__ void store_vec(uint32_t* ptr, const uint32_t (&x)[V])
     }
 }
 
-// Per-lane constants of the column layout.
+// Per-lane constants of the column layout.  Lane l of a warp owns words
+// [vi*V, vi*V+V) of every row; the bit just left of its first word comes from
+// lane l-1 by shuffle (or, on lane 0 / column 0, from its own 4-byte load or
+// the boundary rule), the bit right of its last word likewise from lane l+1.
 struct LaneCols {
-    int64_t vi;          // vector index of this lane within the row
-    bool active;         // vi < nvec
-    bool need_l, need_r; // this lane supplies its own edge word instead of a shuffle
-    int64_t l_idx, r_idx;  // word index of the edge word to load, -1 = synthesise
+    int64_t vi;           // vector index of this lane within the row
+    bool active;          // vi < nvec
+    bool need_l, need_r;  // this lane supplies its own edge word instead of a shuffle
+    bool load_l, load_r;  // ... and loads it (WRAP, or an interior warp edge)
+    bool synth_l, synth_r;  // ... or synthesises it (CLAMP/ZERO at column 0 / w-1)
+    int64_t l_off, r_off;   // word offsets of the loaded edge words within a row
 };
 
 template <int V>
-__device__ __forceinline__ void fetch_row(const LifeParams& p, const LaneCols& c, int64_t y,
-                                          Fetch<V>& f) {
-    const uint32_t* row = p.in + map_row(p, y) * p.pitch_w;
+__device__ __forceinline__ void fetch_row(const LaneCols& c, const uint32_t* row, Fetch<V>& f) {
     if (c.active) {
         load_vec<V>(row + c.vi * V, f.x);
     } else {
 #pragma unroll
         for (int i = 0; i < V; ++i) f.x[i] = 0u;
     }
-    f.le = (c.need_l && c.l_idx >= 0) ? __ldg(row + c.l_idx) : 0u;
-    f.re = (c.need_r && c.r_idx >= 0) ? __ldg(row + c.r_idx) : 0u;
+    f.le = c.load_l ? __ldg(row + c.l_off) : 0u;
+    f.re = c.load_r ? __ldg(row + c.r_off) : 0u;
 }
 
 // Horizontal 3-cell sums of one row: s0 = parity, s1 = carry (L + x + R).
-template <int V>
-__device__ __forceinline__ void row_sums(const LifeParams& p, const LaneCols& c, const Fetch<V>& f,
-                                         uint32_t (&s0)[V], uint32_t (&s1)[V]) {
+template <int V, int CM>
+__device__ __forceinline__ void row_sums(const LaneCols& c, const Fetch<V>& f, uint32_t (&s0)[V],
+                                         uint32_t (&s1)[V]) {
     const uint32_t up = __shfl_up_sync(kFull, f.x[V - 1], 1);
     const uint32_t dn = __shfl_down_sync(kFull, f.x[0], 1);
-    uint32_t lw = c.need_l ? f.le : up;
+    uint32_t lw = c.need_l ? f.le : up;  // ZERO: f.le == 0 on the synthesising lane
     uint32_t rw = c.need_r ? f.re : dn;
-    if (c.l_idx < 0) lw = (p.col_mode == COL_CLAMP) ? (f.x[0] << 31) : 0u;
-    if (c.r_idx < 0) rw = (p.col_mode == COL_CLAMP) ? (f.x[V - 1] >> 31) : 0u;
+    if (CM == COL_CLAMP) {
+        if (c.synth_l) lw = f.x[0] << 31;       // column -1 := column 0
+        if (c.synth_r) rw = f.x[V - 1] >> 31;   // column w := column w-1
+    }
 #pragma unroll
     for (int i = 0; i < V; ++i) {
         const uint32_t ls = (i == 0) ? lw : f.x[i - 1];
@@ -151,7 +169,30 @@ __device__ __forceinline__ uint32_t life_word(uint32_t a0, uint32_t a1, uint32_t
     return C & D;
 }
 
-template <int V, int P>
+template <int V, int CM>
+struct LifeRowState {
+    uint32_t a0[V], a1[V], b0[V], b1[V], alive[V];
+};
+
+// One output row: consume input row y+1 (fetch f), combine with the sums of
+// rows y-1 (a) and y (b), store, rotate.
+template <int V, int CM>
+__device__ __forceinline__ void life_row(const LaneCols& c, const Fetch<V>& f, LifeRowState<V, CM>& st,
+                                         uint32_t* out_row) {
+    uint32_t c0[V], c1[V], o[V];
+    row_sums<V, CM>(c, f, c0, c1);
+#pragma unroll
+    for (int i = 0; i < V; ++i) o[i] = life_word(st.a0[i], st.a1[i], st.b0[i], st.b1[i], c0[i], c1[i], st.alive[i]);
+    if (c.active) store_vec<V>(out_row, o);
+#pragma unroll
+    for (int i = 0; i < V; ++i) {
+        st.a0[i] = st.b0[i]; st.a1[i] = st.b1[i];
+        st.b0[i] = c0[i]; st.b1[i] = c1[i];
+        st.alive[i] = f.x[i];
+    }
+}
+
+template <int V, int P, int CM>
 __global__ void __launch_bounds__(kThreads) life_step_kernel(const __grid_constant__ LifeParams p) {
     const int lane = threadIdx.x & 31;
     const int64_t warp_gid = (int64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
@@ -168,52 +209,325 @@ __global__ void __launch_bounds__(kThreads) life_step_kernel(const __grid_consta
     LaneCols c;
     c.vi = strip * 32 + lane;
     c.active = c.vi < p.nvec;
-    c.need_l = c.active && (lane == 0 || c.vi == 0);
-    c.need_r = c.active && (lane == 31 || c.vi == p.nvec - 1);
-    c.l_idx = (c.vi == 0) ? (p.col_mode == COL_WRAP ? p.nw - 1 : -1) : c.vi * V - 1;
-    c.r_idx = (c.vi == p.nvec - 1) ? (p.col_mode == COL_WRAP ? 0 : -1) : (c.vi + 1) * V;
-    if (!c.need_l) c.l_idx = 0;
-    if (!c.need_r) c.r_idx = 0;
+    const bool first = c.vi == 0, last = c.vi == p.nvec - 1;
+    c.need_l = c.active && (lane == 0 || first);
+    c.need_r = c.active && (lane == 31 || last);
+    c.synth_l = c.need_l && first && CM != COL_WRAP;
+    c.synth_r = c.need_r && last && CM != COL_WRAP;
+    c.load_l = c.need_l && !c.synth_l;
+    c.load_r = c.need_r && !c.synth_r;
+    c.l_off = first ? p.nw - 1 : c.vi * V - 1;
+    c.r_off = last ? 0 : (c.vi + 1) * V;
 
-    // Prologue: rows ys-1 and ys, and the first P rows of the pipeline.
+    // Rows ys..ye-1 lie inside the slab; only rows ys-1 and ye can be halo
+    // rows (or wrapped / clamped rows), so they are resolved once here and
+    // the streaming loop below is branch-free.
+    const uint32_t* row_top = p.in + map_row(p, ys - 1) * p.pitch_w;
+    const uint32_t* row_bot = p.in + map_row(p, ye) * p.pitch_w;
+    const uint32_t* row_ys = p.in + ys * p.pitch_w;
+    auto rowp = [&](int64_t y) { return y < ye ? row_ys + (y - ys) * p.pitch_w : row_bot; };
+
     Fetch<V> fa, fb;
-    fetch_row<V>(p, c, ys - 1, fa);
-    fetch_row<V>(p, c, ys, fb);
+    fetch_row<V>(c, row_top, fa);
+    fetch_row<V>(c, row_ys, fb);
     Fetch<V> ring[P];
 #pragma unroll
-    for (int k = 0; k < P; ++k)
-        if (ys + 1 + k <= ye) fetch_row<V>(p, c, ys + 1 + k, ring[k]);
+    for (int k = 0; k < P; ++k) fetch_row<V>(c, rowp(ys + 1 + k), ring[k]);
 
-    uint32_t a0[V], a1[V], b0[V], b1[V], alive[V];
-    row_sums<V>(p, c, fa, a0, a1);
-    row_sums<V>(p, c, fb, b0, b1);
+    LifeRowState<V, CM> st;
+    row_sums<V, CM>(c, fa, st.a0, st.a1);
+    row_sums<V, CM>(c, fb, st.b0, st.b1);
 #pragma unroll
-    for (int i = 0; i < V; ++i) alive[i] = fb.x[i];
+    for (int i = 0; i < V; ++i) st.alive[i] = fb.x[i];
 
     uint32_t* out_row = p.out + ys * p.pitch_w + c.vi * V;
-    for (int64_t y = ys; y < ye; y += P) {
+    int64_t y = ys;
+    // Steady state: P output rows per trip, P rows of loads always in flight.
+    // Fetches past row ye re-read row ye (harmless, L1/L2 hits).
+    for (; y + P <= ye; y += P) {
 #pragma unroll
         for (int k = 0; k < P; ++k) {
-            const int64_t yy = y + k;
-            if (yy < ye) {
-                Fetch<V> f = ring[k];
-                if (yy + 1 + P <= ye) fetch_row<V>(p, c, yy + 1 + P, ring[k]);
-                uint32_t c0[V], c1[V], o[V];
-                row_sums<V>(p, c, f, c0, c1);
+            const Fetch<V> f = ring[k];
+            fetch_row<V>(c, rowp(y + k + 1 + P), ring[k]);
+            life_row<V, CM>(c, f, st, out_row);
+            out_row += p.pitch_w;
+        }
+    }
+    // Tail: fewer than P rows left; their input rows are already in the ring.
 #pragma unroll
-                for (int i = 0; i < V; ++i)
-                    o[i] = life_word(a0[i], a1[i], b0[i], b1[i], c0[i], c1[i], alive[i]);
-                if (c.active) store_vec<V>(out_row, o);
-                out_row += p.pitch_w;
-#pragma unroll
-                for (int i = 0; i < V; ++i) {
-                    a0[i] = b0[i]; a1[i] = b1[i];
-                    b0[i] = c0[i]; b1[i] = c1[i];
-                    alive[i] = f.x[i];
+    for (int k = 0; k < P; ++k) {
+        if (y + k < ye) {
+            life_row<V, CM>(c, ring[k], st, out_row);
+            out_row += p.pitch_w;
+        }
+    }
+}
+
+// ------------------------------------------------ TMA-bulk pipelined kernel
+// For rows that are a multiple of 128 bits (w % 128 == 0, every BASELINE
+// config): warp-specialised producer/consumer.  One producer warp streams the
+// CTA's strip (NC consumer warps x 512 B) of successive rows into an NS-stage
+// shared-memory ring with cp.async.bulk (TMA bulk copies, completion counted
+// on an mbarrier per stage); the NC consumer warps read their 16 B plus the
+// neighbouring words from shared memory, compute, and store straight to HBM.
+// The data in flight lives in shared memory, not registers, so the pipeline
+// depth (NS rows) is independent of occupancy.  Each stage row carries a
+// 16-byte margin on each side: the neighbouring strip's edge words, or at the
+// row ends the WRAP source (a separate 16-byte bulk copy) — so no shuffles and
+// no per-lane edge loads are needed.
+
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
+                 : "memory");
+}
+
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
+}
+
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+    uint32_t done = 0;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(smem_u32(bar)), "r"(parity)
+            : "memory");
+    } while (!done);
+}
+
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+    asm volatile(
+        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+            smem_u32(dst)),
+        "l"(src), "r"(bytes), "r"(smem_u32(bar))
+        : "memory");
+}
+
+template <int NC>
+struct TmaGeom {
+    static constexpr int kStripWords = NC * 32 * 4;            // words per CTA strip
+    static constexpr int kStageBytes = kStripWords * 4 + 32;   // + 16 B margin each side
+};
+
+struct LifeTmaParams {
+    const uint32_t* in;
+    uint32_t* out;
+    int64_t pitch_w, rows, nw, nstrips;
+    int64_t begin[2], end[2], nchunks[2];
+    int top_map, bot_map;
+};
+
+template <int NC, int NS, int CM>
+__global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_constant__ LifeTmaParams p) {
+    using G = TmaGeom<NC>;
+    extern __shared__ __align__(128) uint8_t smem[];
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
+    uint64_t* empty = full + NS;
+
+    const int band = blockIdx.y;
+    const int64_t nchunks = p.nchunks[band];
+    const int64_t strip = blockIdx.x % p.nstrips;
+    const int64_t chunk = blockIdx.x / p.nstrips;
+    if (chunk >= nchunks) return;  // whole CTA
+    const int64_t rb = p.begin[band], nr = p.end[band] - rb;
+    const int64_t ys = rb + chunk * nr / nchunks;
+    const int64_t ye = rb + (chunk + 1) * nr / nchunks;
+    if (ys >= ye) return;
+    const int64_t w0 = strip * G::kStripWords;                        // first word of the strip
+    const int64_t seg = min((int64_t)G::kStripWords, p.nw - w0);      // words in the strip (multiple of 4)
+    const bool first_strip = strip == 0, last_strip = w0 + seg == p.nw;
+    const int64_t nrows_in = ye - ys + 2;                              // input rows ys-1 .. ye
+
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < NS; ++s) {
+            mbar_init(&full[s], 1);
+            mbar_init(&empty[s], NC);
+        }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+
+    if (warp == NC) {
+        // ------------------------------------------------------ producer
+        if (lane == 0) {
+            const uint32_t* row_top = p.in + map_row(p, ys - 1) * p.pitch_w;
+            const uint32_t* row_bot = p.in + map_row(p, ye) * p.pitch_w;
+            const uint32_t main_bytes = (uint32_t)(seg * 4) + (first_strip ? 0u : 16u) + (last_strip ? 0u : 16u);
+            uint32_t tx = main_bytes;
+            if (CM == COL_WRAP) tx += (first_strip ? 16u : 0u) + (last_strip ? 16u : 0u);
+            for (int64_t i = 0; i < nrows_in; ++i) {
+                const int s = (int)(i % NS);
+                if (i >= NS) mbar_wait(&empty[s], (uint32_t)(((i / NS) + 1) & 1));
+                const int64_t row = ys - 1 + i;
+                const uint32_t* rp = row < ys ? row_top : (row >= ye ? row_bot : p.in + row * p.pitch_w);
+                uint8_t* st = smem + s * G::kStageBytes;
+                mbar_arrive_expect_tx(&full[s], tx);
+                if (first_strip)
+                    bulk_g2s(st + 16, rp + w0, main_bytes, &full[s]);
+                else
+                    bulk_g2s(st, rp + w0 - 4, main_bytes, &full[s]);
+                if (CM == COL_WRAP) {
+                    if (first_strip) bulk_g2s(st, rp + p.nw - 4, 16, &full[s]);         // words nw-4..nw-1
+                    if (last_strip) bulk_g2s(st + 16 + seg * 4, rp, 16, &full[s]);       // words 0..3
                 }
             }
         }
+        return;
     }
+
+    // ------------------------------------------------------ consumers
+    // Input row i (global row ys-1+i) sits in stage i % NS; the loop is
+    // unrolled by NS (a multiple of 3) so stage indices and the 3-row
+    // rotation of the row sums are compile-time register renames.
+    static_assert(NS % 3 == 0, "NS must be a multiple of 3");
+    const int t = warp * 32 + lane;               // vector index within the strip
+    const bool active = t * 4 < (int)seg;
+    const bool row_first = first_strip && t == 0;
+    const bool row_last = last_strip && (t + 1) * 4 == (int)seg;
+    const int n_in = (int)nrows_in;
+    uint32_t r0[3][4], r1[3][4], xs[3][4];        // row sums and raw words of 3 rows
+    uint32_t* out_row = p.out + ys * p.pitch_w + w0 + t * 4;
+
+    auto consume = [&](int i, int k, int slot) {
+        // k = i % NS (static), slot = i % 3 (static)
+        mbar_wait(&full[k], (uint32_t)((i / NS) & 1));
+        const uint32_t* st = reinterpret_cast<const uint32_t*>(smem + k * G::kStageBytes);
+        const uint4 v = *reinterpret_cast<const uint4*>(st + 4 + t * 4);
+        uint32_t lw = st[4 + t * 4 - 1];
+        uint32_t rw = st[4 + t * 4 + 4];
+        __syncwarp();
+        if (lane == 0) mbar_arrive(&empty[k]);
+        if (CM != COL_WRAP) {
+            if (row_first) lw = (CM == COL_CLAMP) ? (v.x << 31) : 0u;
+            if (row_last) rw = (CM == COL_CLAMP) ? (v.w >> 31) : 0u;
+        }
+        xs[slot][0] = v.x; xs[slot][1] = v.y; xs[slot][2] = v.z; xs[slot][3] = v.w;
+#pragma unroll
+        for (int q = 0; q < 4; ++q) {
+            const uint32_t ls = (q == 0) ? lw : xs[slot][q - 1];
+            const uint32_t rs = (q == 3) ? rw : xs[slot][q + 1];
+            const uint32_t L = __funnelshift_l(ls, xs[slot][q], 1);
+            const uint32_t R = __funnelshift_r(xs[slot][q], rs, 1);
+            r0[slot][q] = L ^ xs[slot][q] ^ R;
+            r1[slot][q] = maj3(L, xs[slot][q], R);
+        }
+    };
+    auto emit = [&](int slot) {
+        // output row for centre row in slot (slot+2)%3, above = (slot+1)%3, below = slot
+        const int A = (slot + 1) % 3, B = (slot + 2) % 3, C = slot;
+        uint32_t o[4];
+#pragma unroll
+        for (int q = 0; q < 4; ++q)
+            o[q] = life_word(r0[A][q], r1[A][q], r0[B][q], r1[B][q], r0[C][q], r1[C][q], xs[B][q]);
+        if (active) *reinterpret_cast<uint4*>(out_row) = make_uint4(o[0], o[1], o[2], o[3]);
+        out_row += p.pitch_w;
+    };
+
+    // first trip: rows 0,1 only fill the window
+    int i = 0;
+    if (n_in >= NS) {
+#pragma unroll
+        for (int k = 0; k < NS; ++k) {
+            consume(k, k, k % 3);
+            if (k >= 2) emit(k % 3);
+        }
+        i = NS;
+        for (; i + NS <= n_in; i += NS) {
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                consume(i + k, k, k % 3);
+                emit(k % 3);
+            }
+        }
+    }
+    // last (partial) trip
+#pragma unroll
+    for (int k = 0; k < NS; ++k) {
+        if (i + k < n_in) {
+            consume(i + k, k, k % 3);  // i is a multiple of NS, so (i+k)%3 == k%3 only if NS%3==0
+            if (i + k >= 2) emit(k % 3);
+        }
+    }
+}
+
+template <int NC, int NS, int CM>
+cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+    using G = TmaGeom<NC>;
+    LifeTmaParams p;
+    p.in = static_cast<const uint32_t*>(g.in);
+    p.out = static_cast<uint32_t*>(g.out);
+    p.pitch_w = g.pitch / 4;
+    p.rows = g.rows;
+    p.nw = g.w / 32;
+    p.nstrips = (p.nw + G::kStripWords - 1) / G::kStripWords;
+    p.top_map = g.top_map;
+    p.bot_map = g.bot_map;
+    const int smem = NS * G::kStageBytes + 2 * NS * 8;
+    static int ctas_per_sm = 0;
+    if (ctas_per_sm == 0) {
+        cudaError_t e = cudaFuncSetAttribute(life_tma_kernel<NC, NS, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, life_tma_kernel<NC, NS, CM>, (NC + 1) * 32, smem);
+        if (e != cudaSuccess) return e;
+        if (ctas_per_sm < 1) ctas_per_sm = 1;
+        const int want = kTmaCtasPerSm > 0 ? kTmaCtasPerSm : (16 / NC > 0 ? 16 / NC : 1);
+        if (want < ctas_per_sm) ctas_per_sm = want;
+    }
+    const int64_t resident = (int64_t)num_sms * ctas_per_sm;
+    int64_t max_ctas = 0;
+    for (int i = 0; i < 2; ++i) {
+        p.begin[i] = p.end[i] = 0;
+        p.nchunks[i] = 0;
+    }
+    for (int i = 0; i < b.nbands; ++i) {
+        p.begin[i] = b.begin[i];
+        p.end[i] = b.end[i];
+        const int64_t nr = b.end[i] - b.begin[i];
+        int64_t nch = resident / (p.nstrips * b.nbands);
+        if (nch < 1) nch = 1;
+        if (nch > nr) nch = nr;
+        if (nr <= 0) nch = 0;
+        p.nchunks[i] = nch;
+        if (nch * p.nstrips > max_ctas) max_ctas = nch * p.nstrips;
+    }
+    if (max_ctas == 0) return cudaSuccess;
+    dim3 grid((unsigned)max_ctas, (unsigned)b.nbands);
+    life_tma_kernel<NC, NS, CM><<<grid, (NC + 1) * 32, smem, s>>>(p);
+    return cudaGetLastError();
+}
+
+template <int NC, int NS>
+cudaError_t launch_life_tma_nc(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+    switch (g.col_mode) {
+        case COL_WRAP: return launch_life_tma_t<NC, NS, COL_WRAP>(g, b, num_sms, s);
+        case COL_CLAMP: return launch_life_tma_t<NC, NS, COL_CLAMP>(g, b, num_sms, s);
+        default: return launch_life_tma_t<NC, NS, COL_ZERO>(g, b, num_sms, s);
+    }
+}
+
+// Strip width: the whole row when it fits in 16 warps x 512 B (every config:
+// 65536 cells = 8 KB = 16 warps), so each CTA is ONE sequential DRAM stream;
+// ~16 consumer warps per SM in total (measured best: fewer, longer streams
+// keep HBM pages open — tools/membench.cu, profiles/).
+template <int NS>
+cudaError_t launch_life_tma(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+    const int64_t nvec = g.w / 128;  // 16-byte vectors per row
+    if (nvec > 8 * 32) return launch_life_tma_nc<16, NS>(g, b, num_sms, s);
+    if (nvec > 4 * 32) return launch_life_tma_nc<8, NS>(g, b, num_sms, s);
+    if (nvec > 2 * 32) return launch_life_tma_nc<4, NS>(g, b, num_sms, s);
+    return launch_life_tma_nc<2, NS>(g, b, num_sms, s);
 }
 
 // ------------------------------------------------------------ pack / unpack
@@ -263,7 +577,7 @@ __global__ void unpack_life_kernel(const uint32_t* __restrict__ src, int64_t src
     }
 }
 
-template <int V, int P>
+template <int V, int P, int CM>
 cudaError_t launch_life_t(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
     LifeParams p;
     p.in = static_cast<const uint32_t*>(g.in);
@@ -280,7 +594,7 @@ cudaError_t launch_life_t(const StencilGeom& g, const RowBands& b, int num_sms, 
     static int blocks_per_sm = 0;  // per (V,P) instantiation; device-independent enough
     if (blocks_per_sm == 0) {
         cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm,
-                                                                      life_step_kernel<V, P>, kThreads, 0);
+                                                                      life_step_kernel<V, P, CM>, kThreads, 0);
         if (e != cudaSuccess) return e;
         if (blocks_per_sm < 1) blocks_per_sm = 1;
     }
@@ -303,16 +617,29 @@ cudaError_t launch_life_t(const StencilGeom& g, const RowBands& b, int num_sms, 
     }
     if (max_warps == 0) return cudaSuccess;
     dim3 grid((unsigned)((max_warps + kThreads / 32 - 1) / (kThreads / 32)), (unsigned)b.nbands);
-    life_step_kernel<V, P><<<grid, kThreads, 0, s>>>(p);
+    life_step_kernel<V, P, CM><<<grid, kThreads, 0, s>>>(p);
     return cudaGetLastError();
+}
+
+template <int V, int P>
+cudaError_t launch_life_cm(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+    switch (g.col_mode) {
+        case COL_WRAP: return launch_life_t<V, P, COL_WRAP>(g, b, num_sms, s);
+        case COL_CLAMP: return launch_life_t<V, P, COL_CLAMP>(g, b, num_sms, s);
+        default: return launch_life_t<V, P, COL_ZERO>(g, b, num_sms, s);
+    }
 }
 
 }  // namespace
 
 cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
     const int64_t nw = g.w / 32;
-    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_t<4, 3>(g, b, num_sms, s);
-    return launch_life_t<2, 3>(g, b, num_sms, s);
+#ifdef MAPSM_LIFE_REGS
+    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_cm<4, kLifeP>(g, b, num_sms, s);
+#else
+    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_tma<kTmaNS>(g, b, num_sms, s);
+#endif
+    return launch_life_cm<2, kLifeP>(g, b, num_sms, s);
 }
 
 cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, int64_t dst_pitch,

@@ -14,7 +14,7 @@
 //     to two neighbours, so it is computed in O(1).
 #include <cstdint>
 
-#include "../../include/mapsm.h"
+#include "mapsm.h"
 
 namespace mapsm {
 

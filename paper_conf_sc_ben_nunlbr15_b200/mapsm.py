@@ -13,7 +13,9 @@ import os
 
 import numpy as np
 
-_LIB_PATH = os.path.join(os.path.dirname(os.path.abspath(__file__)), "libmapsm.so")
+# MAPSM_LIB may point at an alternative build of the same library (kernel
+# tuning experiments); the default is the in-tree build.
+_LIB_PATH = os.environ.get("MAPSM_LIB") or os.path.join(os.path.dirname(os.path.abspath(__file__)), "libmapsm.so")
 
 # enums (include/mapsm.h)
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
