@@ -42,7 +42,8 @@ def _sources():
 
 
 def _deps():
-    return _sources() + glob.glob(os.path.join(CSRC, "*.h")) + [os.path.join(INCLUDE, "mapsm.h"), __file__]
+    return (_sources() + glob.glob(os.path.join(CSRC, "*.h")) + glob.glob(os.path.join(CSRC, "*.cuh"))
+            + [os.path.join(INCLUDE, "mapsm.h"), __file__])
 
 
 def needs_build() -> bool:
@@ -64,15 +65,28 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, cs
     os.makedirs(obj_dir, exist_ok=True)
     nvcc = os.environ.get("NVCC", "nvcc")
     incs = ["-I", INCLUDE, "-I", src_dir, "-I", _nccl_include()]
-    objs = []
     srcs = sorted(glob.glob(os.path.join(src_dir, "*.cu")) + glob.glob(os.path.join(src_dir, "*.cpp")))
+    objs, cmds = [], []
     for src in srcs:
         obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
-        cmd = [nvcc, *ARCH, *NVFLAGS, *(extra or []), *incs, "-c", src, "-o", obj]
+        cmds.append([nvcc, *ARCH, *NVFLAGS, *(extra or []), *incs, "-c", src, "-o", obj])
+        objs.append(obj)
+    # translation units compile in parallel (the conv radii are the slow ones)
+    from concurrent.futures import ThreadPoolExecutor
+
+    def run(cmd):
         if verbose:
             print(" ".join(cmd), file=sys.stderr)
-        subprocess.check_call(cmd)
-        objs.append(obj)
+        return subprocess.run(cmd, capture_output=not verbose, text=True)
+
+    with ThreadPoolExecutor(max_workers=min(8, os.cpu_count() or 4)) as ex:
+        results = list(ex.map(run, cmds))
+    for cmd, res in zip(cmds, results):
+        if res.returncode != 0:
+            if not verbose:
+                sys.stderr.write(res.stdout or "")
+                sys.stderr.write(res.stderr or "")
+            raise subprocess.CalledProcessError(res.returncode, cmd)
     tmp = lib_path + ".tmp"
     cmd = [nvcc, *ARCH, "-shared", "-o", tmp, *objs, "-ldl", "-lpthread"]
     if verbose:

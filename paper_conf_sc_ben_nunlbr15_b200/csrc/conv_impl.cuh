@@ -1,0 +1,490 @@
+#pragma once
+// conv.cu — fp32 window convolution (cross-correlation), radius 1..4, sm_100a.
+//
+// Path rows a4/a5 of SURVEY §8(a), float case: Window(2D) input (Table 1
+// P:L87-88, "N-dimensional convolution") -> Structured Injective output
+// (P:L102).  Per output cell, exactly (reading c11):
+//     acc = +0.0f; for dy=-r..r: for dx=-r..r: acc = fmaf(W[dy][dx], in[y+dy][x+dx], acc)
+// so the result is bit-identical to any implementation of that definition.
+//
+// Design.  Each lane owns 4 consecutive output columns (one
+// 128-bit load/store per row) and a warp streams down a chunk of rows.  Input
+// row Y is loaded once and feeds, in the fixed tap order, the 2r+1 output rows
+// y = Y-r..Y+r whose accumulators are live in registers: because rows stream
+// in increasing Y, output y receives its dy = -r..r tap rows in exactly the
+// required order (this is the paper's ILP over rows, taken to the
+// whole chunk).  The 2r horizontal neighbours come from the adjacent lanes via
+// shuffles (edge lanes load one extra float4).  Weights are a kernel parameter
+// (constant bank) indexed by compile-time tap numbers, so every FFMA takes its
+// weight straight from the constant bank.  No tensor cores: a 2D stencil is
+// not a dense contraction and reshaping it into one would not be exact.
+#include <cuda_runtime.h>
+#include <stdint.h>
+
+#include <type_traits>
+
+#include "kernels.h"
+#include "tma_rows.cuh"
+
+namespace mapsm {
+namespace conv_detail {
+
+constexpr int kThreads = 256;
+constexpr unsigned kFull = 0xffffffffu;
+
+template <int R>
+struct ConvParams {
+    const float* in;
+    float* out;
+    int64_t pitch_f;  // row pitch in floats
+    int64_t rows;
+    int64_t w;
+    int64_t nvec;     // w / 4
+    int64_t warps_per_row;
+    int64_t begin[2], end[2], nchunks[2];
+    int top_map, bot_map, col_mode;
+    float wt[(2 * R + 1) * (2 * R + 1)];
+};
+
+template <class Prm>
+__device__ __forceinline__ int64_t map_row(const Prm& p, int64_t y) {
+    if (y < 0) {
+        if (p.top_map == ROWMAP_WRAP) {
+            y %= p.rows;
+            if (y < 0) y += p.rows;
+        } else if (p.top_map == ROWMAP_CLAMP) {
+            y = 0;
+        }
+    } else if (y >= p.rows) {
+        if (p.bot_map == ROWMAP_WRAP) y %= p.rows;
+        else if (p.bot_map == ROWMAP_CLAMP) y = p.rows - 1;
+    }
+    return y;
+}
+
+struct F4Fetch {
+    float4 v, l, r;  // own vector, left/right edge vectors (edge lanes only)
+};
+
+struct ConvLane {
+    int64_t vi;
+    bool active, need_l, need_r;
+    int64_t l_idx, r_idx;  // float index of the edge float4, -1 = synthesise (CLAMP/ZERO)
+};
+
+template <class Prm>
+__device__ __forceinline__ void conv_fetch(const Prm& p, const ConvLane& c, int64_t Y, F4Fetch& f) {
+    const float* row = p.in + map_row(p, Y) * p.pitch_f;
+    const float4 z = make_float4(0.f, 0.f, 0.f, 0.f);
+    f.v = c.active ? __ldg(reinterpret_cast<const float4*>(row + c.vi * 4)) : z;
+    f.l = (c.need_l && c.l_idx >= 0) ? __ldg(reinterpret_cast<const float4*>(row + c.l_idx)) : z;
+    f.r = (c.need_r && c.r_idx >= 0) ? __ldg(reinterpret_cast<const float4*>(row + c.r_idx)) : z;
+}
+
+// v[i] = in[Y][x0 - R + i], i in [0, 4 + 2R)
+template <int R, class Prm>
+__device__ __forceinline__ void conv_window(const Prm& p, const ConvLane& c, const F4Fetch& f,
+                                            float (&v)[4 + 2 * R]) {
+    const float own[4] = {f.v.x, f.v.y, f.v.z, f.v.w};
+    float lft[4], rgt[4];
+    lft[0] = __shfl_up_sync(kFull, f.v.x, 1);
+    lft[1] = __shfl_up_sync(kFull, f.v.y, 1);
+    lft[2] = __shfl_up_sync(kFull, f.v.z, 1);
+    lft[3] = __shfl_up_sync(kFull, f.v.w, 1);
+    rgt[0] = __shfl_down_sync(kFull, f.v.x, 1);
+    rgt[1] = __shfl_down_sync(kFull, f.v.y, 1);
+    rgt[2] = __shfl_down_sync(kFull, f.v.z, 1);
+    rgt[3] = __shfl_down_sync(kFull, f.v.w, 1);
+    if (c.need_l) {
+        if (c.l_idx >= 0) {
+            lft[0] = f.l.x; lft[1] = f.l.y; lft[2] = f.l.z; lft[3] = f.l.w;
+        } else {
+            const float e = (p.col_mode == COL_CLAMP) ? own[0] : 0.f;
+            lft[0] = lft[1] = lft[2] = lft[3] = e;
+        }
+    }
+    if (c.need_r) {
+        if (c.r_idx >= 0) {
+            rgt[0] = f.r.x; rgt[1] = f.r.y; rgt[2] = f.r.z; rgt[3] = f.r.w;
+        } else {
+            const float e = (p.col_mode == COL_CLAMP) ? own[3] : 0.f;
+            rgt[0] = rgt[1] = rgt[2] = rgt[3] = e;
+        }
+    }
+#pragma unroll
+    for (int i = 0; i < R; ++i) v[i] = lft[4 - R + i];
+#pragma unroll
+    for (int i = 0; i < 4; ++i) v[R + i] = own[i];
+#pragma unroll
+    for (int i = 0; i < R; ++i) v[R + 4 + i] = rgt[i];
+}
+
+// PF = rows of loads in flight per lane; U = unroll, a multiple of both the
+// accumulator ring (2R+1) and PF so every ring index is a compile-time constant.
+template <int R, int PF>
+__global__ void __launch_bounds__(kThreads) conv_step_kernel(const __grid_constant__ ConvParams<R> p) {
+    constexpr int K = 2 * R + 1;
+    constexpr int U = K * PF;
+    const int lane = threadIdx.x & 31;
+    const int64_t warp_gid = (int64_t)blockIdx.x * (kThreads / 32) + (threadIdx.x >> 5);
+    const int band = blockIdx.y;
+    const int64_t nchunks = p.nchunks[band];
+    const int64_t strip = warp_gid % p.warps_per_row;
+    const int64_t chunk = warp_gid / p.warps_per_row;
+    if (chunk >= nchunks) return;
+    const int64_t rb = p.begin[band], nr = p.end[band] - rb;
+    const int64_t ys = rb + chunk * nr / nchunks;
+    const int64_t ye = rb + (chunk + 1) * nr / nchunks;
+    if (ys >= ye) return;
+
+    ConvLane c;
+    c.vi = strip * 32 + lane;
+    c.active = c.vi < p.nvec;
+    c.need_l = c.active && (lane == 0 || c.vi == 0);
+    c.need_r = c.active && (lane == 31 || c.vi == p.nvec - 1);
+    c.l_idx = (c.vi == 0) ? (p.col_mode == COL_WRAP ? p.w - 4 : -1) : c.vi * 4 - 4;
+    c.r_idx = (c.vi == p.nvec - 1) ? (p.col_mode == COL_WRAP ? 0 : -1) : c.vi * 4 + 4;
+
+    const int64_t y_first = ys - R;      // first input row
+    const int64_t y_last = ye + R - 1;   // last input row
+
+    F4Fetch ring[PF];
+#pragma unroll
+    for (int k = 0; k < PF; ++k)
+        if (y_first + k <= y_last) conv_fetch(p, c, y_first + k, ring[k]);
+
+    float acc[K][4];
+#pragma unroll
+    for (int j = 0; j < K; ++j)
+#pragma unroll
+        for (int q = 0; q < 4; ++q) acc[j][q] = 0.f;
+
+    for (int64_t Yb = y_first; Yb <= y_last; Yb += U) {
+#pragma unroll
+        for (int s = 0; s < U; ++s) {
+            const int64_t Y = Yb + s;
+            if (Y <= y_last) {
+                const F4Fetch f = ring[s % PF];
+                if (Y + PF <= y_last) conv_fetch(p, c, Y + PF, ring[s % PF]);
+                float v[4 + 2 * R];
+                conv_window<R>(p, c, f, v);
+                // Tap row d (dy = d - R) of output y = Y + R - d; slot (s - d) mod K.
+#pragma unroll
+                for (int d = 0; d < K; ++d) {
+                    const int64_t y = Y + R - d;
+                    const int slot = ((s - d) % K + K) % K;
+                    if (y >= ys && y < ye) {
+                        if (d == 0) {
+#pragma unroll
+                            for (int q = 0; q < 4; ++q) acc[slot][q] = 0.f;
+                        }
+#pragma unroll
+                        for (int q = 0; q < 4; ++q) {
+                            float a = acc[slot][q];
+#pragma unroll
+                            for (int e = 0; e < K; ++e) a = __fmaf_rn(p.wt[d * K + e], v[q + e], a);
+                            acc[slot][q] = a;
+                        }
+                        if (d == K - 1 && c.active) {
+                            float* o = p.out + y * p.pitch_f + c.vi * 4;
+                            *reinterpret_cast<float4*>(o) =
+                                make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                        }
+                    }
+                }
+            }
+        }
+    }
+}
+
+// Generic path for widths that are not a multiple of 4 (or < 4): one thread
+// per output cell, per-tap boundary resolution.  Same tap order.
+template <int R>
+__global__ void conv_generic_kernel(const __grid_constant__ ConvParams<R> p) {
+    constexpr int K = 2 * R + 1;
+    const int64_t x = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int band = blockIdx.z;
+    if (x >= p.w) return;
+    for (int64_t y = p.begin[band] + blockIdx.y; y < p.end[band]; y += gridDim.y) {
+    float acc = 0.f;
+#pragma unroll
+    for (int d = 0; d < K; ++d) {
+        const float* row = p.in + map_row(p, y + d - R) * p.pitch_f;
+#pragma unroll
+        for (int e = 0; e < K; ++e) {
+            int64_t xx = x + e - R;
+            float v;
+            if (xx >= 0 && xx < p.w) {
+                v = __ldg(row + xx);
+            } else if (p.col_mode == COL_WRAP) {
+                xx %= p.w;
+                if (xx < 0) xx += p.w;
+                v = __ldg(row + xx);
+            } else if (p.col_mode == COL_CLAMP) {
+                v = __ldg(row + (xx < 0 ? 0 : p.w - 1));
+            } else {
+                v = 0.f;
+            }
+            acc = __fmaf_rn(p.wt[d * K + e], v, acc);
+        }
+    }
+    p.out[y * p.pitch_f + x] = acc;
+    }
+}
+
+// ------------------------------------------------ TMA-bulk pipelined kernel
+// Rows stream through the shared-memory ring of tma_rows.cuh (producer warp +
+// NC consumer warps, one CTA strip = NC x 128 floats).  Consumer lane t owns 4
+// output columns; for input row Y it reads 12 floats (its 4 plus 4 on each
+// side, from the stage: no shuffles) and advances the 2R+1 live accumulator
+// rows in the fixed tap order.  The loop is unrolled by NS, a multiple of
+// 2R+1, so the accumulator ring and the stage index are compile-time.
+template <int R>
+struct ConvTmaParams {
+    tma::RowStream s;
+    float wt[(2 * R + 1) * (2 * R + 1)];
+};
+
+template <int R, int NC, int NS, int CM>
+__global__ void __launch_bounds__((NC + 1) * 32, 1) conv_tma_kernel(const __grid_constant__ ConvTmaParams<R> pp) {
+    constexpr int K = 2 * R + 1;
+    static_assert(NS % K == 0, "NS must be a multiple of 2R+1");
+    using G = tma::Geom<NC>;
+    const tma::RowStream& p = pp.s;
+    extern __shared__ __align__(128) uint8_t smem[];
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
+    uint64_t* empty = full + NS;
+    tma::init_barriers<NS>(full, empty, NC);
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    tma::SegIter it = tma::seg_iter(p);
+    tma::Seg sg;
+    tma::RingPos ring;
+
+    if (warp == NC) {
+        if (lane == 0) {
+            while (tma::seg_next<NC>(p, it, sg)) {
+                tma::produce_align<NS>(full, empty, ring);
+                tma::produce<NC, NS, CM == COL_WRAP>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R, ring);
+            }
+        }
+        return;
+    }
+
+    const int t = warp * 32 + lane;
+    float acc[K][4];
+    while (tma::seg_next<NC>(p, it, sg)) {
+        tma::consume_align<NS>(full, empty, ring, lane);
+        uint32_t ph = ring.phase;  // segment starts at stage 0
+        const int n_out = (int)(sg.ye - sg.ys);
+        const int n_in = n_out + 2 * R;  // input rows ys-R .. ye+R-1
+        const bool active = t * 4 < (int)sg.seg;
+        const bool row_first = sg.first_strip && t == 0;
+        const bool row_last = sg.last_strip && (t + 1) * 4 == (int)sg.seg;
+        float* out0 = static_cast<float*>(p.out) + sg.ys * p.pitch + sg.e0 + t * 4;
+
+        // Input row j: output rows o = j - d (d = 0..2R, tap row dy = d - R)
+        // take their d-th tap row from it; o starts at d == 0 and completes
+        // at d == 2R.
+        auto step = [&](int j, int k, bool check) {
+            tma::mbar_wait(&full[k], ph);
+            const float* st = reinterpret_cast<const float*>(smem + k * G::kStageBytes);
+            const float4 L = *reinterpret_cast<const float4*>(st + t * 4);
+            const float4 O = *reinterpret_cast<const float4*>(st + t * 4 + 4);
+            const float4 Rv = *reinterpret_cast<const float4*>(st + t * 4 + 8);
+            __syncwarp();
+            if (lane == 0) tma::mbar_arrive(&empty[k]);
+            float lf[4] = {L.x, L.y, L.z, L.w};
+            float rf[4] = {Rv.x, Rv.y, Rv.z, Rv.w};
+            if (CM != COL_WRAP) {
+                if (row_first) {
+                    const float e = (CM == COL_CLAMP) ? O.x : 0.f;
+                    lf[0] = lf[1] = lf[2] = lf[3] = e;
+                }
+                if (row_last) {
+                    const float e = (CM == COL_CLAMP) ? O.w : 0.f;
+                    rf[0] = rf[1] = rf[2] = rf[3] = e;
+                }
+            }
+            float v[4 + 2 * R];
+#pragma unroll
+            for (int q = 0; q < R; ++q) v[q] = lf[4 - R + q];
+            v[R] = O.x; v[R + 1] = O.y; v[R + 2] = O.z; v[R + 3] = O.w;
+#pragma unroll
+            for (int q = 0; q < R; ++q) v[R + 4 + q] = rf[q];
+#pragma unroll
+            for (int d = 0; d < K; ++d) {
+                const int o = j - d;
+                const int slot = ((k - d) % K + K) % K;  // == o mod K since NS % K == 0
+                if (!check || (o >= 0 && o < n_out)) {
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) {
+                        float a = (d == 0) ? 0.f : acc[slot][q];
+#pragma unroll
+                        for (int e = 0; e < K; ++e) a = __fmaf_rn(pp.wt[d * K + e], v[q + e], a);
+                        acc[slot][q] = a;
+                    }
+                    if (d == K - 1 && active)
+                        *reinterpret_cast<float4*>(out0 + (int64_t)o * p.pitch) =
+                            make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                }
+            }
+        };
+
+        const uint32_t ph0 = ph;
+        int j = 0;
+        if (n_in >= NS) {
+#pragma unroll
+            for (int k = 0; k < NS; ++k) step(k, k, true);  // first trip: o < 0 for d > k (static)
+            ph ^= 1u;
+            // steady trips: every output touched lies in [0, n_out)
+            for (j = NS; j + NS <= n_in && j + NS - 1 < n_out; j += NS) {
+#pragma unroll
+                for (int k = 0; k < NS; ++k) step(j + k, k, false);
+                ph ^= 1u;
+            }
+        }
+        for (; j < n_in; j += NS) {  // remaining rows: full checks
+#pragma unroll
+            for (int k = 0; k < NS; ++k)
+                if (j + k < n_in) step(j + k, k, true);
+            ph ^= 1u;
+        }
+        ring.stage = n_in % NS;
+        ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
+        ring.count += n_in;
+    }
+}
+
+template <int R, int NC, int NS, int CM>
+cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
+                              cudaStream_t s) {
+    using G = tma::Geom<NC>;
+    constexpr int K = 2 * R + 1;
+    ConvTmaParams<R> pp;
+    tma::RowStream& p = pp.s;
+    p.in = static_cast<const uint32_t*>(g.in);
+    p.out = g.out;
+    p.pitch = g.pitch / 4;
+    p.rows = g.rows;
+    p.n = g.w;
+    p.top_map = g.top_map;
+    p.bot_map = g.bot_map;
+    for (int j = 0; j < K * K; ++j) pp.wt[j] = weights[j];
+    const int smem = NS * G::kStageBytes + 2 * NS * 8;
+    static int ctas_per_sm = 0;
+    if (ctas_per_sm == 0) {
+        cudaError_t e = cudaFuncSetAttribute(conv_tma_kernel<R, NC, NS, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        if (e != cudaSuccess) return e;
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, conv_tma_kernel<R, NC, NS, CM>, (NC + 1) * 32, smem);
+        if (e != cudaSuccess) return e;
+        if (ctas_per_sm < 1) ctas_per_sm = 1;
+        // HBM-bound radii: ~16 consumer warps per SM; FMA-bound radii (r >= 3,
+        // 49-81 taps): one CTA per SM, registers hold the accumulator ring.
+        const int want = R <= 2 ? (16 / NC > 0 ? 16 / NC : 1) : 1;
+        if (want < ctas_per_sm) ctas_per_sm = want;
+    }
+    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems);
+    if (ctas == 0) return cudaSuccess;
+    dim3 grid((unsigned)ctas, (unsigned)b.nbands);
+    conv_tma_kernel<R, NC, NS, CM><<<grid, (NC + 1) * 32, smem, s>>>(pp);
+    return cudaGetLastError();
+}
+
+template <int R, int NS>
+cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
+                            cudaStream_t s) {
+    // whole-row strips up to 16 warps x 128 floats; otherwise 16-warp strips
+    const int64_t nvec = g.w / 4;
+    auto go = [&](auto nc_tag) -> cudaError_t {
+        constexpr int NC = decltype(nc_tag)::value;
+        switch (g.col_mode) {
+            case COL_WRAP: return launch_conv_tma_t<R, NC, NS, COL_WRAP>(g, b, weights, num_sms, s);
+            case COL_CLAMP: return launch_conv_tma_t<R, NC, NS, COL_CLAMP>(g, b, weights, num_sms, s);
+            default: return launch_conv_tma_t<R, NC, NS, COL_ZERO>(g, b, weights, num_sms, s);
+        }
+    };
+    if constexpr (R <= 2) {
+        if (nvec > 8 * 32) return go(std::integral_constant<int, 16>());
+    }
+    if (nvec > 4 * 32) return go(std::integral_constant<int, 8>());
+    if (nvec > 2 * 32) return go(std::integral_constant<int, 4>());
+    return go(std::integral_constant<int, 2>());
+}
+
+template <int R, int PF>
+cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
+                          cudaStream_t s) {
+    constexpr int K = 2 * R + 1;
+    ConvParams<R> p;
+    p.in = static_cast<const float*>(g.in);
+    p.out = static_cast<float*>(g.out);
+    p.pitch_f = g.pitch / 4;
+    p.rows = g.rows;
+    p.w = g.w;
+    p.nvec = g.w / 4;
+    p.warps_per_row = (p.nvec + 31) / 32;
+    p.top_map = g.top_map;
+    p.bot_map = g.bot_map;
+    p.col_mode = g.col_mode;
+    for (int i = 0; i < K * K; ++i) p.wt[i] = weights[i];
+    for (int i = 0; i < 2; ++i) {
+        p.begin[i] = p.end[i] = 0;
+        p.nchunks[i] = 0;
+    }
+    const bool fast = (g.w % 4 == 0) && (g.pitch % 16 == 0) && g.w >= 4;
+    if (!fast) {
+        int64_t maxr = 0;
+        for (int i = 0; i < b.nbands; ++i) {
+            p.begin[i] = b.begin[i];
+            p.end[i] = b.end[i];
+            if (b.end[i] - b.begin[i] > maxr) maxr = b.end[i] - b.begin[i];
+        }
+        if (maxr <= 0) return cudaSuccess;
+        dim3 grid((unsigned)((g.w + 127) / 128), (unsigned)(maxr < 4096 ? maxr : 4096), (unsigned)b.nbands);
+        conv_generic_kernel<R><<<grid, 128, 0, s>>>(p);
+        return cudaGetLastError();
+    }
+    static int blocks_per_sm = 0;
+    if (blocks_per_sm == 0) {
+        cudaError_t e =
+            cudaOccupancyMaxActiveBlocksPerMultiprocessor(&blocks_per_sm, conv_step_kernel<R, PF>, kThreads, 0);
+        if (e != cudaSuccess) return e;
+        if (blocks_per_sm < 1) blocks_per_sm = 1;
+    }
+    const int64_t resident_warps = (int64_t)num_sms * blocks_per_sm * (kThreads / 32);
+    int64_t max_warps = 0;
+    for (int i = 0; i < b.nbands; ++i) {
+        p.begin[i] = b.begin[i];
+        p.end[i] = b.end[i];
+        const int64_t nr = b.end[i] - b.begin[i];
+        int64_t nch = resident_warps / (p.warps_per_row * b.nbands);
+        if (nch < 1) nch = 1;
+        if (nch > nr) nch = nr;
+        if (nr <= 0) nch = 0;
+        p.nchunks[i] = nch;
+        if (nch * p.warps_per_row > max_warps) max_warps = nch * p.warps_per_row;
+    }
+    if (max_warps == 0) return cudaSuccess;
+    dim3 grid((unsigned)((max_warps + kThreads / 32 - 1) / (kThreads / 32)), (unsigned)b.nbands);
+    conv_step_kernel<R, PF><<<grid, kThreads, 0, s>>>(p);
+    return cudaGetLastError();
+}
+
+}  // namespace conv_detail
+
+// Per-radius entry point (explicitly instantiated in conv_r<R>.cu so the four
+// radii compile in parallel).  Rows of a multiple of 4 floats take the TMA
+// pipeline; other widths the simple register kernel.
+template <int R>
+cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
+                               cudaStream_t s) {
+    constexpr int kNS = R == 1 ? 12 : R == 2 ? 10 : R == 3 ? 14 : 9;  // multiples of 2R+1
+    constexpr int kPF = R <= 2 ? 2 : 1;
+#ifndef MAPSM_CONV_REGS
+    if (g.w % 4 == 0 && g.w >= 4 && g.pitch % 16 == 0)
+        return conv_detail::launch_conv_tma<R, kNS>(g, b, weights, num_sms, s);
+#endif
+    return conv_detail::launch_conv_t<R, kPF>(g, b, weights, num_sms, s);
+}
+
+}  // namespace mapsm

@@ -1,0 +1,6 @@
+// conv_r3.cu — radius-3 instantiation of the fp32 window convolution (see conv_impl.cuh).
+#include "conv_impl.cuh"
+
+namespace mapsm {
+template cudaError_t launch_conv_radius<3>(const StencilGeom&, const RowBands&, const float*, int, cudaStream_t);
+}  // namespace mapsm

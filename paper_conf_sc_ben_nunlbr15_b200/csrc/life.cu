@@ -25,6 +25,7 @@
 #include <stdint.h>
 
 #include "kernels.h"
+#include "tma_rows.cuh"
 
 namespace mapsm {
 namespace {
@@ -265,213 +266,130 @@ __global__ void __launch_bounds__(kThreads) life_step_kernel(const __grid_consta
 
 // ------------------------------------------------ TMA-bulk pipelined kernel
 // For rows that are a multiple of 128 bits (w % 128 == 0, every BASELINE
-// config): warp-specialised producer/consumer.  One producer warp streams the
-// CTA's strip (NC consumer warps x 512 B) of successive rows into an NS-stage
-// shared-memory ring with cp.async.bulk (TMA bulk copies, completion counted
-// on an mbarrier per stage); the NC consumer warps read their 16 B plus the
-// neighbouring words from shared memory, compute, and store straight to HBM.
-// The data in flight lives in shared memory, not registers, so the pipeline
-// depth (NS rows) is independent of occupancy.  Each stage row carries a
-// 16-byte margin on each side: the neighbouring strip's edge words, or at the
-// row ends the WRAP source (a separate 16-byte bulk copy) — so no shuffles and
-// no per-lane edge loads are needed.
-
-__device__ __forceinline__ uint32_t smem_u32(const void* p) {
-    return static_cast<uint32_t>(__cvta_generic_to_shared(p));
-}
-
-__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
-    asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(bar)), "r"(count) : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
-    asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(bar)), "r"(bytes)
-                 : "memory");
-}
-
-__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
-    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(bar)) : "memory");
-}
-
-__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
-    uint32_t done = 0;
-    do {
-        asm volatile(
-            "{\n\t.reg .pred p;\n\t"
-            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
-            "selp.u32 %0, 1, 0, p;\n\t}"
-            : "=r"(done)
-            : "r"(smem_u32(bar)), "r"(parity)
-            : "memory");
-    } while (!done);
-}
-
-__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
-    asm volatile(
-        "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
-            smem_u32(dst)),
-        "l"(src), "r"(bytes), "r"(smem_u32(bar))
-        : "memory");
-}
-
-template <int NC>
-struct TmaGeom {
-    static constexpr int kStripWords = NC * 32 * 4;            // words per CTA strip
-    static constexpr int kStageBytes = kStripWords * 4 + 32;   // + 16 B margin each side
-};
-
-struct LifeTmaParams {
-    const uint32_t* in;
-    uint32_t* out;
-    int64_t pitch_w, rows, nw, nstrips;
-    int64_t begin[2], end[2], nchunks[2];
-    int top_map, bot_map;
-};
+// config): warp-specialised producer/consumer over the row-streaming pipeline
+// of tma_rows.cuh.  One producer warp streams the CTA's strip (NC consumer
+// warps x 512 B; the whole row when w <= 65536) of successive rows into an
+// NS-stage shared-memory ring with TMA bulk copies; the NC consumer warps read
+// their 16 B plus the neighbouring words (the stage's 16-byte margins hold the
+// neighbouring strips' edge words, or the WRAP source at the row ends), do the
+// bit-sliced update, and store straight to HBM.
 
 template <int NC, int NS, int CM>
-__global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_constant__ LifeTmaParams p) {
-    using G = TmaGeom<NC>;
+__global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_constant__ tma::RowStream p) {
+    using G = tma::Geom<NC>;
     extern __shared__ __align__(128) uint8_t smem[];
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
     uint64_t* empty = full + NS;
-
-    const int band = blockIdx.y;
-    const int64_t nchunks = p.nchunks[band];
-    const int64_t strip = blockIdx.x % p.nstrips;
-    const int64_t chunk = blockIdx.x / p.nstrips;
-    if (chunk >= nchunks) return;  // whole CTA
-    const int64_t rb = p.begin[band], nr = p.end[band] - rb;
-    const int64_t ys = rb + chunk * nr / nchunks;
-    const int64_t ye = rb + (chunk + 1) * nr / nchunks;
-    if (ys >= ye) return;
-    const int64_t w0 = strip * G::kStripWords;                        // first word of the strip
-    const int64_t seg = min((int64_t)G::kStripWords, p.nw - w0);      // words in the strip (multiple of 4)
-    const bool first_strip = strip == 0, last_strip = w0 + seg == p.nw;
-    const int64_t nrows_in = ye - ys + 2;                              // input rows ys-1 .. ye
-
+    tma::init_barriers<NS>(full, empty, NC);
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-    if (threadIdx.x == 0) {
-        for (int s = 0; s < NS; ++s) {
-            mbar_init(&full[s], 1);
-            mbar_init(&empty[s], NC);
-        }
-        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
-    }
-    __syncthreads();
+    tma::SegIter it = tma::seg_iter(p);
+    tma::Seg sg;
+    tma::RingPos ring;  // CTA-wide ring position (same sequence in producer and consumers)
 
     if (warp == NC) {
-        // ------------------------------------------------------ producer
         if (lane == 0) {
-            const uint32_t* row_top = p.in + map_row(p, ys - 1) * p.pitch_w;
-            const uint32_t* row_bot = p.in + map_row(p, ye) * p.pitch_w;
-            const uint32_t main_bytes = (uint32_t)(seg * 4) + (first_strip ? 0u : 16u) + (last_strip ? 0u : 16u);
-            uint32_t tx = main_bytes;
-            if (CM == COL_WRAP) tx += (first_strip ? 16u : 0u) + (last_strip ? 16u : 0u);
-            for (int64_t i = 0; i < nrows_in; ++i) {
-                const int s = (int)(i % NS);
-                if (i >= NS) mbar_wait(&empty[s], (uint32_t)(((i / NS) + 1) & 1));
-                const int64_t row = ys - 1 + i;
-                const uint32_t* rp = row < ys ? row_top : (row >= ye ? row_bot : p.in + row * p.pitch_w);
-                uint8_t* st = smem + s * G::kStageBytes;
-                mbar_arrive_expect_tx(&full[s], tx);
-                if (first_strip)
-                    bulk_g2s(st + 16, rp + w0, main_bytes, &full[s]);
-                else
-                    bulk_g2s(st, rp + w0 - 4, main_bytes, &full[s]);
-                if (CM == COL_WRAP) {
-                    if (first_strip) bulk_g2s(st, rp + p.nw - 4, 16, &full[s]);         // words nw-4..nw-1
-                    if (last_strip) bulk_g2s(st + 16 + seg * 4, rp, 16, &full[s]);       // words 0..3
-                }
+            while (tma::seg_next<NC>(p, it, sg)) {
+                tma::produce_align<NS>(full, empty, ring);
+                tma::produce<NC, NS, CM == COL_WRAP>(p, sg, smem, full, empty, sg.ys - 1, sg.ye - sg.ys + 2, ring);
             }
         }
         return;
     }
 
     // ------------------------------------------------------ consumers
-    // Input row i (global row ys-1+i) sits in stage i % NS; the loop is
-    // unrolled by NS (a multiple of 3) so stage indices and the 3-row
-    // rotation of the row sums are compile-time register renames.
+    // Input row j of a segment (global row ys-1+j) sits in stage (base+j) % NS
+    // with base a multiple of NS; the loop is unrolled by NS (a multiple of 3)
+    // so stage indices and the 3-row rotation of the row sums are
+    // compile-time register renames.
     static_assert(NS % 3 == 0, "NS must be a multiple of 3");
-    const int t = warp * 32 + lane;               // vector index within the strip
-    const bool active = t * 4 < (int)seg;
-    const bool row_first = first_strip && t == 0;
-    const bool row_last = last_strip && (t + 1) * 4 == (int)seg;
-    const int n_in = (int)nrows_in;
-    uint32_t r0[3][4], r1[3][4], xs[3][4];        // row sums and raw words of 3 rows
-    uint32_t* out_row = p.out + ys * p.pitch_w + w0 + t * 4;
+    const int t = warp * 32 + lane;  // vector index within the strip
+    uint32_t r0[3][4], r1[3][4], xs[3][4];  // row sums and raw words of 3 rows
+    while (tma::seg_next<NC>(p, it, sg)) {
+        tma::consume_align<NS>(full, empty, ring, lane);
+        uint32_t ph = ring.phase;  // segment starts at stage 0
+        const int n_in = (int)(sg.ye - sg.ys + 2);  // input rows ys-1 .. ye
+        const bool active = t * 4 < (int)sg.seg;
+        const bool row_first = sg.first_strip && t == 0;
+        const bool row_last = sg.last_strip && (t + 1) * 4 == (int)sg.seg;
+        uint32_t* out_row = static_cast<uint32_t*>(p.out) + sg.ys * p.pitch + sg.e0 + t * 4;
 
-    auto consume = [&](int i, int k, int slot) {
-        // k = i % NS (static), slot = i % 3 (static)
-        mbar_wait(&full[k], (uint32_t)((i / NS) & 1));
-        const uint32_t* st = reinterpret_cast<const uint32_t*>(smem + k * G::kStageBytes);
-        const uint4 v = *reinterpret_cast<const uint4*>(st + 4 + t * 4);
-        uint32_t lw = st[4 + t * 4 - 1];
-        uint32_t rw = st[4 + t * 4 + 4];
-        __syncwarp();
-        if (lane == 0) mbar_arrive(&empty[k]);
-        if (CM != COL_WRAP) {
-            if (row_first) lw = (CM == COL_CLAMP) ? (v.x << 31) : 0u;
-            if (row_last) rw = (CM == COL_CLAMP) ? (v.w >> 31) : 0u;
-        }
-        xs[slot][0] = v.x; xs[slot][1] = v.y; xs[slot][2] = v.z; xs[slot][3] = v.w;
+        auto consume = [&](int j, int k, int slot) {
+            // k = j % NS (static), slot = j % 3 (static)
+            tma::mbar_wait(&full[k], ph);
+            const uint32_t* st = reinterpret_cast<const uint32_t*>(smem + k * G::kStageBytes);
+            const uint4 v = *reinterpret_cast<const uint4*>(st + 4 + t * 4);
+            uint32_t lw = st[4 + t * 4 - 1];
+            uint32_t rw = st[4 + t * 4 + 4];
+            __syncwarp();
+            if (lane == 0) tma::mbar_arrive(&empty[k]);
+            if (CM != COL_WRAP) {
+                if (row_first) lw = (CM == COL_CLAMP) ? (v.x << 31) : 0u;  // column -1 := column 0 / 0
+                if (row_last) rw = (CM == COL_CLAMP) ? (v.w >> 31) : 0u;   // column w := column w-1 / 0
+            }
+            xs[slot][0] = v.x; xs[slot][1] = v.y; xs[slot][2] = v.z; xs[slot][3] = v.w;
 #pragma unroll
-        for (int q = 0; q < 4; ++q) {
-            const uint32_t ls = (q == 0) ? lw : xs[slot][q - 1];
-            const uint32_t rs = (q == 3) ? rw : xs[slot][q + 1];
-            const uint32_t L = __funnelshift_l(ls, xs[slot][q], 1);
-            const uint32_t R = __funnelshift_r(xs[slot][q], rs, 1);
-            r0[slot][q] = L ^ xs[slot][q] ^ R;
-            r1[slot][q] = maj3(L, xs[slot][q], R);
-        }
-    };
-    auto emit = [&](int slot) {
-        // output row for centre row in slot (slot+2)%3, above = (slot+1)%3, below = slot
-        const int A = (slot + 1) % 3, B = (slot + 2) % 3, C = slot;
-        uint32_t o[4];
+            for (int q = 0; q < 4; ++q) {
+                const uint32_t ls = (q == 0) ? lw : xs[slot][q - 1];
+                const uint32_t rs = (q == 3) ? rw : xs[slot][q + 1];
+                const uint32_t L = __funnelshift_l(ls, xs[slot][q], 1);
+                const uint32_t R = __funnelshift_r(xs[slot][q], rs, 1);
+                r0[slot][q] = L ^ xs[slot][q] ^ R;
+                r1[slot][q] = maj3(L, xs[slot][q], R);
+            }
+        };
+        auto emit = [&](int slot) {
+            // centre row in slot (slot+2)%3, row above in (slot+1)%3, row below in slot
+            const int A = (slot + 1) % 3, B = (slot + 2) % 3, C = slot;
+            uint32_t o[4];
 #pragma unroll
-        for (int q = 0; q < 4; ++q)
-            o[q] = life_word(r0[A][q], r1[A][q], r0[B][q], r1[B][q], r0[C][q], r1[C][q], xs[B][q]);
-        if (active) *reinterpret_cast<uint4*>(out_row) = make_uint4(o[0], o[1], o[2], o[3]);
-        out_row += p.pitch_w;
-    };
+            for (int q = 0; q < 4; ++q)
+                o[q] = life_word(r0[A][q], r1[A][q], r0[B][q], r1[B][q], r0[C][q], r1[C][q], xs[B][q]);
+            if (active) *reinterpret_cast<uint4*>(out_row) = make_uint4(o[0], o[1], o[2], o[3]);
+            out_row += p.pitch;
+        };
 
-    // first trip: rows 0,1 only fill the window
-    int i = 0;
-    if (n_in >= NS) {
-#pragma unroll
-        for (int k = 0; k < NS; ++k) {
-            consume(k, k, k % 3);
-            if (k >= 2) emit(k % 3);
-        }
-        i = NS;
-        for (; i + NS <= n_in; i += NS) {
+        const uint32_t ph0 = ph;
+        int j = 0;
+        if (n_in >= NS) {
+            // first trip: input rows 0,1 only fill the window
 #pragma unroll
             for (int k = 0; k < NS; ++k) {
-                consume(i + k, k, k % 3);
-                emit(k % 3);
+                consume(k, k, k % 3);
+                if (k >= 2) emit(k % 3);
+            }
+            ph ^= 1u;
+            for (j = NS; j + NS <= n_in; j += NS) {
+#pragma unroll
+                for (int k = 0; k < NS; ++k) {
+                    consume(j + k, k, k % 3);
+                    emit(k % 3);
+                }
+                ph ^= 1u;
             }
         }
-    }
-    // last (partial) trip
+        // last (partial) trip; j is a multiple of NS (and of 3)
 #pragma unroll
-    for (int k = 0; k < NS; ++k) {
-        if (i + k < n_in) {
-            consume(i + k, k, k % 3);  // i is a multiple of NS, so (i+k)%3 == k%3 only if NS%3==0
-            if (i + k >= 2) emit(k % 3);
+        for (int k = 0; k < NS; ++k) {
+            if (j + k < n_in) {
+                consume(j + k, k, k % 3);
+                if (j + k >= 2) emit(k % 3);
+            }
         }
+        ring.stage = n_in % NS;
+        ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
+        ring.count += n_in;
     }
 }
 
 template <int NC, int NS, int CM>
 cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
-    using G = TmaGeom<NC>;
-    LifeTmaParams p;
+    using G = tma::Geom<NC>;
+    tma::RowStream p;
     p.in = static_cast<const uint32_t*>(g.in);
-    p.out = static_cast<uint32_t*>(g.out);
-    p.pitch_w = g.pitch / 4;
+    p.out = g.out;
+    p.pitch = g.pitch / 4;
     p.rows = g.rows;
-    p.nw = g.w / 32;
-    p.nstrips = (p.nw + G::kStripWords - 1) / G::kStripWords;
+    p.n = g.w / 32;
     p.top_map = g.top_map;
     p.bot_map = g.bot_map;
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
@@ -485,25 +403,9 @@ cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_s
         const int want = kTmaCtasPerSm > 0 ? kTmaCtasPerSm : (16 / NC > 0 ? 16 / NC : 1);
         if (want < ctas_per_sm) ctas_per_sm = want;
     }
-    const int64_t resident = (int64_t)num_sms * ctas_per_sm;
-    int64_t max_ctas = 0;
-    for (int i = 0; i < 2; ++i) {
-        p.begin[i] = p.end[i] = 0;
-        p.nchunks[i] = 0;
-    }
-    for (int i = 0; i < b.nbands; ++i) {
-        p.begin[i] = b.begin[i];
-        p.end[i] = b.end[i];
-        const int64_t nr = b.end[i] - b.begin[i];
-        int64_t nch = resident / (p.nstrips * b.nbands);
-        if (nch < 1) nch = 1;
-        if (nch > nr) nch = nr;
-        if (nr <= 0) nch = 0;
-        p.nchunks[i] = nch;
-        if (nch * p.nstrips > max_ctas) max_ctas = nch * p.nstrips;
-    }
-    if (max_ctas == 0) return cudaSuccess;
-    dim3 grid((unsigned)max_ctas, (unsigned)b.nbands);
+    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems);
+    if (ctas == 0) return cudaSuccess;
+    dim3 grid((unsigned)ctas, (unsigned)b.nbands);
     life_tma_kernel<NC, NS, CM><<<grid, (NC + 1) * 32, smem, s>>>(p);
     return cudaGetLastError();
 }
