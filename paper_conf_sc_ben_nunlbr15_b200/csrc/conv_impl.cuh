@@ -29,6 +29,19 @@
 namespace mapsm {
 namespace conv_detail {
 
+#ifndef MAPSM_CONV_BIG_CTAS
+#define MAPSM_CONV_BIG_CTAS 1
+#endif
+#ifndef MAPSM_CONV_BIG_NC
+#define MAPSM_CONV_BIG_NC 8
+#endif
+constexpr int kConvBigCtas = MAPSM_CONV_BIG_CTAS;  // CTAs per SM for r >= 3
+constexpr int kConvBigNC = MAPSM_CONV_BIG_NC;      // consumer warps per CTA for r >= 3 (8 or 16)
+#ifndef MAPSM_CONV_BIG_EPL
+#define MAPSM_CONV_BIG_EPL 4
+#endif
+constexpr int kConvBigEPL = MAPSM_CONV_BIG_EPL;    // floats per lane for r >= 3
+
 constexpr int kThreads = 256;
 constexpr unsigned kFull = 0xffffffffu;
 
@@ -234,22 +247,39 @@ __global__ void conv_generic_kernel(const __grid_constant__ ConvParams<R> p) {
 
 // ------------------------------------------------ TMA-bulk pipelined kernel
 // Rows stream through the shared-memory ring of tma_rows.cuh (producer warp +
-// NC consumer warps, one CTA strip = NC x 128 floats).  Consumer lane t owns 4
-// output columns; for input row Y it reads 12 floats (its 4 plus 4 on each
-// side, from the stage: no shuffles) and advances the 2R+1 live accumulator
-// rows in the fixed tap order.  The loop is unrolled by NS, a multiple of
-// 2R+1, so the accumulator ring and the stage index are compile-time.
+// NC consumer warps, one CTA strip = NC x 32 x EPL floats).  Consumer lane t
+// owns EPL output columns; for input row Y it reads EPL + 8 floats (its own
+// plus 4 on each side, from the stage: no shuffles) and advances the 2R+1
+// live accumulator rows in the fixed tap order.  The loop is unrolled by NS,
+// a multiple of 2R+1, so the accumulator ring and the stage index are
+// compile-time.  EPL = 4 (one 16-byte vector per lane) for every radius:
+// EPL = 2 halves the unrolled code for r >= 3 but measured 12% slower on 9x9
+// (profiles/r01_conv9_variants.txt), the per-row overhead doubling relative
+// to the FMAs.
 template <int R>
 struct ConvTmaParams {
     tma::RowStream s;
     float wt[(2 * R + 1) * (2 * R + 1)];
 };
 
-template <int R, int NC, int NS, int CM>
-__global__ void __launch_bounds__((NC + 1) * 32, 1) conv_tma_kernel(const __grid_constant__ ConvTmaParams<R> pp) {
+template <int EPL>
+struct VecF;
+template <>
+struct VecF<4> {
+    using T = float4;
+};
+template <>
+struct VecF<2> {
+    using T = float2;
+};
+
+template <int R, int NC, int NS, int CM, int EPL>
+__global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) conv_tma_kernel(const __grid_constant__ ConvTmaParams<R> pp) {
     constexpr int K = 2 * R + 1;
     static_assert(NS % K == 0, "NS must be a multiple of 2R+1");
-    using G = tma::Geom<NC>;
+    static_assert(R <= 4, "16-byte stage margins cover r <= 4");
+    using G = tma::Geom<NC, EPL>;
+    using VT = typename VecF<EPL>::T;
     const tma::RowStream& p = pp.s;
     extern __shared__ __align__(128) uint8_t smem[];
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
@@ -262,25 +292,26 @@ __global__ void __launch_bounds__((NC + 1) * 32, 1) conv_tma_kernel(const __grid
 
     if (warp == NC) {
         if (lane == 0) {
-            while (tma::seg_next<NC>(p, it, sg)) {
+            while (tma::seg_next<NC, EPL>(p, it, sg)) {
                 tma::produce_align<NS>(full, empty, ring);
-                tma::produce<NC, NS, CM == COL_WRAP>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R, ring);
+                tma::produce<NC, NS, CM == COL_WRAP, EPL>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R,
+                                                         ring);
             }
         }
         return;
     }
 
     const int t = warp * 32 + lane;
-    float acc[K][4];
-    while (tma::seg_next<NC>(p, it, sg)) {
+    float acc[K][EPL];
+    while (tma::seg_next<NC, EPL>(p, it, sg)) {
         tma::consume_align<NS>(full, empty, ring, lane);
         uint32_t ph = ring.phase;  // segment starts at stage 0
         const int n_out = (int)(sg.ye - sg.ys);
         const int n_in = n_out + 2 * R;  // input rows ys-R .. ye+R-1
-        const bool active = t * 4 < (int)sg.seg;
+        const bool active = t * EPL < (int)sg.seg;
         const bool row_first = sg.first_strip && t == 0;
-        const bool row_last = sg.last_strip && (t + 1) * 4 == (int)sg.seg;
-        float* out0 = static_cast<float*>(p.out) + sg.ys * p.pitch + sg.e0 + t * 4;
+        const bool row_last = sg.last_strip && (t + 1) * EPL == (int)sg.seg;
+        float* out0 = static_cast<float*>(p.out) + sg.ys * p.pitch + sg.e0 + t * EPL;
 
         // Input row j: output rows o = j - d (d = 0..2R, tap row dy = d - R)
         // take their d-th tap row from it; o starts at d == 0 and completes
@@ -288,44 +319,52 @@ __global__ void __launch_bounds__((NC + 1) * 32, 1) conv_tma_kernel(const __grid
         auto step = [&](int j, int k, bool check) {
             tma::mbar_wait(&full[k], ph);
             const float* st = reinterpret_cast<const float*>(smem + k * G::kStageBytes);
-            const float4 L = *reinterpret_cast<const float4*>(st + t * 4);
-            const float4 O = *reinterpret_cast<const float4*>(st + t * 4 + 4);
-            const float4 Rv = *reinterpret_cast<const float4*>(st + t * 4 + 8);
-            __syncwarp();
-            if (lane == 0) tma::mbar_arrive(&empty[k]);
-            float lf[4] = {L.x, L.y, L.z, L.w};
-            float rf[4] = {Rv.x, Rv.y, Rv.z, Rv.w};
-            if (CM != COL_WRAP) {
-                if (row_first) {
-                    const float e = (CM == COL_CLAMP) ? O.x : 0.f;
-                    lf[0] = lf[1] = lf[2] = lf[3] = e;
-                }
-                if (row_last) {
-                    const float e = (CM == COL_CLAMP) ? O.w : 0.f;
-                    rf[0] = rf[1] = rf[2] = rf[3] = e;
+            // buf[m] = stage float t*EPL + m = strip element t*EPL - 4 + m
+            float buf[EPL + 8];
+#pragma unroll
+            for (int m = 0; m < EPL + 8; m += EPL) {
+                const VT q = *reinterpret_cast<const VT*>(st + t * EPL + m);
+                if constexpr (EPL == 4) {
+                    buf[m] = q.x; buf[m + 1] = q.y; buf[m + 2] = q.z; buf[m + 3] = q.w;
+                } else {
+                    buf[m] = q.x; buf[m + 1] = q.y;
                 }
             }
-            float v[4 + 2 * R];
+            __syncwarp();
+            if (lane == 0) tma::mbar_arrive(&empty[k]);
+            if (CM != COL_WRAP) {
+                if (row_first) {
+                    const float e = (CM == COL_CLAMP) ? buf[4] : 0.f;
 #pragma unroll
-            for (int q = 0; q < R; ++q) v[q] = lf[4 - R + q];
-            v[R] = O.x; v[R + 1] = O.y; v[R + 2] = O.z; v[R + 3] = O.w;
+                    for (int m = 0; m < 4; ++m) buf[m] = e;
+                }
+                if (row_last) {
+                    const float e = (CM == COL_CLAMP) ? buf[3 + EPL] : 0.f;
 #pragma unroll
-            for (int q = 0; q < R; ++q) v[R + 4 + q] = rf[q];
+                    for (int m = 4 + EPL; m < 8 + EPL; ++m) buf[m] = e;
+                }
+            }
+            // v[q + e] = element t*EPL + q + e - R  ->  buf[4 - R + q + e]
 #pragma unroll
             for (int d = 0; d < K; ++d) {
                 const int o = j - d;
                 const int slot = ((k - d) % K + K) % K;  // == o mod K since NS % K == 0
                 if (!check || (o >= 0 && o < n_out)) {
 #pragma unroll
-                    for (int q = 0; q < 4; ++q) {
+                    for (int q = 0; q < EPL; ++q) {
                         float a = (d == 0) ? 0.f : acc[slot][q];
 #pragma unroll
-                        for (int e = 0; e < K; ++e) a = __fmaf_rn(pp.wt[d * K + e], v[q + e], a);
+                        for (int e = 0; e < K; ++e) a = __fmaf_rn(pp.wt[d * K + e], buf[4 - R + q + e], a);
                         acc[slot][q] = a;
                     }
-                    if (d == K - 1 && active)
-                        *reinterpret_cast<float4*>(out0 + (int64_t)o * p.pitch) =
-                            make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                    if (d == K - 1 && active) {
+                        if constexpr (EPL == 4)
+                            *reinterpret_cast<float4*>(out0 + (int64_t)o * p.pitch) =
+                                make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                        else
+                            *reinterpret_cast<float2*>(out0 + (int64_t)o * p.pitch) =
+                                make_float2(acc[slot][0], acc[slot][1]);
+                    }
                 }
             }
         };
@@ -355,10 +394,10 @@ __global__ void __launch_bounds__((NC + 1) * 32, 1) conv_tma_kernel(const __grid
     }
 }
 
-template <int R, int NC, int NS, int CM>
+template <int R, int NC, int NS, int CM, int EPL>
 cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                               cudaStream_t s) {
-    using G = tma::Geom<NC>;
+    using G = tma::Geom<NC, EPL>;
     constexpr int K = 2 * R + 1;
     ConvTmaParams<R> pp;
     tma::RowStream& p = pp.s;
@@ -373,37 +412,38 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
     static int ctas_per_sm = 0;
     if (ctas_per_sm == 0) {
-        cudaError_t e = cudaFuncSetAttribute(conv_tma_kernel<R, NC, NS, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+        auto kfn = conv_tma_kernel<R, NC, NS, CM, EPL>;
+        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
         if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, conv_tma_kernel<R, NC, NS, CM>, (NC + 1) * 32, smem);
+        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, kfn, (NC + 1) * 32, smem);
         if (e != cudaSuccess) return e;
         if (ctas_per_sm < 1) ctas_per_sm = 1;
         // HBM-bound radii: ~16 consumer warps per SM; FMA-bound radii (r >= 3,
-        // 49-81 taps): one CTA per SM, registers hold the accumulator ring.
-        const int want = R <= 2 ? (16 / NC > 0 ? 16 / NC : 1) : 1;
+        // 49-81 taps): kConvBigCtas CTAs per SM.
+        const int want = R <= 2 ? (16 / NC > 0 ? 16 / NC : 1) : kConvBigCtas;
         if (want < ctas_per_sm) ctas_per_sm = want;
     }
     const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems);
     if (ctas == 0) return cudaSuccess;
     dim3 grid((unsigned)ctas, (unsigned)b.nbands);
-    conv_tma_kernel<R, NC, NS, CM><<<grid, (NC + 1) * 32, smem, s>>>(pp);
+    conv_tma_kernel<R, NC, NS, CM, EPL><<<grid, (NC + 1) * 32, smem, s>>>(pp);
     return cudaGetLastError();
 }
 
 template <int R, int NS>
 cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                             cudaStream_t s) {
-    // whole-row strips up to 16 warps x 128 floats; otherwise 16-warp strips
-    const int64_t nvec = g.w / 4;
+    constexpr int EPL = R <= 2 ? 4 : kConvBigEPL;
+    const int64_t nvec = g.w / EPL;
     auto go = [&](auto nc_tag) -> cudaError_t {
         constexpr int NC = decltype(nc_tag)::value;
         switch (g.col_mode) {
-            case COL_WRAP: return launch_conv_tma_t<R, NC, NS, COL_WRAP>(g, b, weights, num_sms, s);
-            case COL_CLAMP: return launch_conv_tma_t<R, NC, NS, COL_CLAMP>(g, b, weights, num_sms, s);
-            default: return launch_conv_tma_t<R, NC, NS, COL_ZERO>(g, b, weights, num_sms, s);
+            case COL_WRAP: return launch_conv_tma_t<R, NC, NS, COL_WRAP, EPL>(g, b, weights, num_sms, s);
+            case COL_CLAMP: return launch_conv_tma_t<R, NC, NS, COL_CLAMP, EPL>(g, b, weights, num_sms, s);
+            default: return launch_conv_tma_t<R, NC, NS, COL_ZERO, EPL>(g, b, weights, num_sms, s);
         }
     };
-    if constexpr (R <= 2) {
+    if constexpr (R <= 2 || kConvBigNC == 16) {
         if (nvec > 8 * 32) return go(std::integral_constant<int, 16>());
     }
     if (nvec > 4 * 32) return go(std::integral_constant<int, 8>());
@@ -472,9 +512,6 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
 
 }  // namespace conv_detail
 
-// Per-radius entry point (explicitly instantiated in conv_r<R>.cu so the four
-// radii compile in parallel).  Rows of a multiple of 4 floats take the TMA
-// pipeline; other widths the simple register kernel.
 template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                                cudaStream_t s) {

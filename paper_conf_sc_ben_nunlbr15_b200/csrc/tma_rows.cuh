@@ -67,9 +67,10 @@ __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t by
         : "memory");
 }
 
-template <int NC>
+// NC consumer warps, EPL 4-byte elements per lane (4 = one 16-byte vector).
+template <int NC, int EPL = 4>
 struct Geom {
-    static constexpr int kStripElems = NC * 32 * 4;           // 4-byte elements per strip
+    static constexpr int kStripElems = NC * 32 * EPL;         // 4-byte elements per strip
     static constexpr int kStageBytes = kStripElems * 4 + 32;  // + 16 B margin each side
 };
 
@@ -125,7 +126,7 @@ __device__ __forceinline__ SegIter seg_iter(const RowStream& p) {
     return it;
 }
 
-template <int NC>
+template <int NC, int EPL = 4>
 __device__ __forceinline__ bool seg_next(const RowStream& p, SegIter& it, Seg& s) {
     if (it.pos >= it.hi) return false;
     const int64_t strip = it.pos / it.nr, r0 = it.pos % it.nr;
@@ -133,8 +134,9 @@ __device__ __forceinline__ bool seg_next(const RowStream& p, SegIter& it, Seg& s
     s.ys = it.rb + r0;
     s.ye = it.rb + r1;
     it.pos += r1 - r0;
-    s.e0 = strip * Geom<NC>::kStripElems;
-    s.seg = p.n - s.e0 < Geom<NC>::kStripElems ? p.n - s.e0 : Geom<NC>::kStripElems;
+    using G = Geom<NC, EPL>;
+    s.e0 = strip * G::kStripElems;
+    s.seg = p.n - s.e0 < G::kStripElems ? p.n - s.e0 : G::kStripElems;
     s.first_strip = strip == 0;
     s.last_strip = s.e0 + s.seg == p.n;
     return true;
@@ -195,10 +197,10 @@ __device__ __forceinline__ void consume_align(uint64_t* full, uint64_t* empty, R
 // segment's strip into the ring, continuing the CTA-wide row counter i.  Row
 // i goes to stage i % NS; before reusing a stage it waits until all consumer
 // warps released the row that occupied it.
-template <int NC, int NS, bool WRAP_COLS>
+template <int NC, int NS, bool WRAP_COLS, int EPL = 4>
 __device__ __forceinline__ void produce(const RowStream& p, const Seg& t, uint8_t* smem, uint64_t* full,
                                         uint64_t* empty, int64_t y_first, int64_t n_in, RingPos& r) {
-    using G = Geom<NC>;
+    using G = Geom<NC, EPL>;
     const uint32_t main_bytes = (uint32_t)(t.seg * 4) + (t.first_strip ? 0u : 16u) + (t.last_strip ? 0u : 16u);
     uint32_t tx = main_bytes;
     if (WRAP_COLS) tx += (t.first_strip ? 16u : 0u) + (t.last_strip ? 16u : 0u);
