@@ -25,6 +25,8 @@ SEED_CONV5_FIELD = 0x5EED0004
 SEED_CONV5_W = 0x5EED0044
 SEED_CONV9_FIELD = 0x5EED0005
 SEED_CONV9_W = 0x5EED0055
+SEED_HIST_UNIFORM = 0x5EED0006
+SEED_HIST_SKEWED = 0x5EED0066
 
 
 def build(force: bool = False) -> str:
@@ -49,6 +51,8 @@ def _L():
         _lib.mapsm_gen_field_f32.restype = None
         _lib.mapsm_gen_weights_f32.argtypes = [u64, ctypes.c_int, p]
         _lib.mapsm_gen_weights_f32.restype = None
+        _lib.mapsm_gen_image_u8.argtypes = [u64, i64, i64, i64, p, i64, ctypes.c_int]
+        _lib.mapsm_gen_image_u8.restype = None
     return _lib
 
 
@@ -80,6 +84,16 @@ def weights_f32(seed: int, r: int) -> np.ndarray:
     out = np.empty(k * k, dtype=np.float32)
     _L().mapsm_gen_weights_f32(seed, r, out.ctypes.data)
     return out.reshape(k, k)
+
+
+def image_u8(seed: int, w: int, h: int, y0: int = 0, kind: str = "uniform",
+             out: np.ndarray | None = None) -> np.ndarray:
+    """Rows [y0, y0+h) of a synthetic u8 image (histogram path)."""
+    if out is None:
+        out = np.empty((h, w), dtype=np.uint8)
+    assert out.dtype == np.uint8 and out.strides[1] == 1
+    _L().mapsm_gen_image_u8(seed, w, y0, h, out.ctypes.data, out.strides[0], {"uniform": 0, "skewed": 1}[kind])
+    return out
 
 
 # Hand-placed patterns (SURVEY §8(c) "BJ.configs[1]" pin).

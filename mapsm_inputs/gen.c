@@ -56,3 +56,26 @@ void mapsm_gen_weights_f32(uint64_t seed, int r, float* out) {
     }
     for (int t = 0; t < taps; ++t) out[t] = (float)(raw[t] / sum);
 }
+
+/* u8 images for the histogram (Reductive-Static) path, rows [y0, y0+rows),
+ * row stride `pitch` bytes.  kind 0: uniform, pixel = v >> 56.
+ * kind 1: skewed ("natural-image-like" concentration around 128 that makes
+ * bins collide): the mean of the 4 high bytes of v, rounded down. */
+void mapsm_gen_image_u8(uint64_t seed, int64_t w, int64_t y0, int64_t rows, uint8_t* out, int64_t pitch,
+                        int kind) {
+#pragma omp parallel for schedule(static)
+    for (int64_t y = 0; y < rows; ++y) {
+        uint64_t base = seed + (uint64_t)(y0 + y) * (uint64_t)w;
+        uint8_t* o = out + y * pitch;
+        for (int64_t x = 0; x < w; ++x) {
+            uint64_t v = splitmix64(base + (uint64_t)x);
+            if (kind == 0) {
+                o[x] = (uint8_t)(v >> 56);
+            } else {
+                unsigned s = (unsigned)((v >> 56) & 255) + (unsigned)((v >> 48) & 255) + (unsigned)((v >> 40) & 255) +
+                             (unsigned)((v >> 32) & 255);
+                o[x] = (uint8_t)(s / 4);
+            }
+        }
+    }
+}

@@ -11,7 +11,8 @@ imports it.
 Parity status: Life pinned (closed forms, scipy neighbour count,
 known methuselah, exhaustive tiny tori); fp32 conv pinned (exact-rational fma
 chain, scipy correlate in fp64, roll/identity closed forms, mass invariant);
-fp64 conv pinned (scipy correlate).  No function is "parity unpinned".
+fp64 conv pinned (scipy correlate); histogram pinned (numpy.bincount, closed
+forms, invariants).  No function is "parity unpinned".
 """
 from __future__ import annotations
 
@@ -51,6 +52,8 @@ def _L():
         for f in (_lib.oracle_life_ex, _lib.oracle_conv_ex, _lib.oracle_conv_f64_ex):
             f.restype = ci
         _lib.oracle_num_threads.restype = ci
+        _lib.oracle_histogram.argtypes = [p, i64, i64, i64, ci, p]
+        _lib.oracle_histogram.restype = ci
     return _lib
 
 
@@ -104,6 +107,18 @@ def conv_f64(field: np.ndarray, weights: np.ndarray, n: int, boundary="wrap", si
                                  *_sides(boundary, sides))
     if rc != 0:
         raise ValueError("oracle_conv_f64_ex rejected its arguments")
+    return out
+
+
+def histogram(img: np.ndarray, nbins: int = 256) -> np.ndarray:
+    """256-bin histogram of a u8 image (Reductive-Static pattern, Fig 4)."""
+    a = np.asarray(img)
+    assert a.dtype == np.uint8 and a.ndim == 2 and a.strides[1] == 1
+    h, w = a.shape
+    out = np.zeros(nbins, dtype=np.uint64)
+    rc = _L().oracle_histogram(a.ctypes.data, w, h, a.strides[0] if h > 0 else w, nbins, out.ctypes.data)
+    if rc != 0:
+        raise ValueError("oracle_histogram rejected its arguments")
     return out
 
 

@@ -222,6 +222,21 @@ int oracle_conv_f64(const float* in, double* out, int64_t w, int64_t h, int64_t 
     return oracle_conv_f64_ex(in, out, w, h, n, r, weights, boundary, boundary, boundary, boundary);
 }
 
+/* ------------------------------------------------------------ Histogram */
+
+/* Reductive (Static) output pattern (§3.2; Fig 4 P:L359-403 §4.5.3,
+ * "auto bin = *image_iter; hist_iter[bin] += 1"): the BINS-bin histogram of a
+ * w x h image of u8 pixels, bin = pixel value (reading h1).  Counts are
+ * 64-bit (reading h2).  Plain sequential loop over rows and columns; `pitch`
+ * is the row stride in bytes (padding bytes are not pixels). */
+int oracle_histogram(const uint8_t* img, int64_t w, int64_t h, int64_t pitch, int nbins, uint64_t* bins) {
+    if (w < 0 || h < 0 || pitch < w || nbins != 256 || !bins) return -1;
+    for (int b = 0; b < nbins; ++b) bins[b] = 0;
+    for (int64_t y = 0; y < h; ++y)
+        for (int64_t x = 0; x < w; ++x) bins[img[y * pitch + x]] += 1;
+    return 0;
+}
+
 /* Number of OpenMP threads the oracle will use (for the cpu_baseline record). */
 int oracle_num_threads(void) {
     int n = 1;
