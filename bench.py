@@ -1,23 +1,26 @@
 """bench.py — Game of Life cell-updates/s and % HBM roofline on 1..8 B200.
 
 Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` (torchrun
-for N > 1) prints ONE JSON line on rank 0.
+for N > 1) prints ONE JSON line on rank 0.  Default workload = BASELINE.json
+configs[2] at N=1 (``life64k``); ``--workload`` selects the other configs
+(``life8k``, ``conv5``, ``conv9``) and the §8(f) NEXT-1 histogram (``hist8k``).
 
-* step      = one ``mapsm_iterate(grid, n)`` call: n generations (BASELINE.json
-              configs[2]: 200) of the whole hot path over the row-slab-
-              partitioned grid — boundary rows, halo exchange (N > 1),
-              interior, buffer swap — with the grid resident in HBM.
-* value     = w*h*n*K / max-over-ranks device time of the K timed steps
-              (CUDA events on the library's compute stream; L2 is flushed
-              between steps, outside the events).
-* e2e       = the same metric through the public C ABI with HOST buffers:
-              per step mapsm_bind (pinned u8 host rows -> device, packed),
-              mapsm_iterate(n), mapsm_read (device -> pinned host u8).
-* roofline  = the dominant kernel (life_step_kernel): 0.25 B/cell-update
-              algorithmic (1 bit in + 1 bit out), per launch, vs the measured
-              HBM copy bandwidth (MEASURED_PEAKS.json hbm_gbs).
-* cpu_baseline = the CPU oracle (oracle/oracle.c, OpenMP) timed on a bounded
-              sample of the same workload on rank 0 only.
+* step      = one pass of the hot path over the resident grid: for the stencils
+              one ``mapsm_iterate(grid, n)`` call (n generations: boundary rows,
+              halo exchange when N > 1, interior, buffer swap); for the histogram
+              one ``mapsm_histogram`` (per-slab bins, cross-GPU aggregation).
+* value     = work units (cell-updates or pixels) of all ranks in K steps / the
+              max-over-ranks device time of the K steps (CUDA events on the
+              library's compute stream; L2 flushed between steps outside the
+              events).
+* e2e       = the same metric through the public C ABI with pinned HOST buffers
+              and the host<->device copies inside the timed region (mapsm_bind
+              of the host rows, the step, mapsm_read / histogram to host).
+* roofline  = the dominant kernel vs the measured HBM copy bandwidth
+              (MEASURED_PEAKS.json hbm_gbs); algorithmic bytes: 0.25 B per Life
+              cell-update, 8 B per conv cell-update, 1 B per histogram pixel.
+* cpu_baseline = the CPU oracle (oracle/, OpenMP) timed on a bounded sample of
+              the same workload on rank 0 only.
 ``--impl reference`` times only the oracle (this tier's reference arm).
 """
 from __future__ import annotations
@@ -34,10 +37,7 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
-import numpy as np  # noqa: E402
-
 WORKLOADS = {
-    # name: (op, w, h_total_at_1gpu, radius, boundary, n per step, seed field, seed weights, scaling)
     "life64k": dict(op="life", w=65536, h=65536, r=1, b="wrap", n=200, seed=0x5EED0003, wseed=None,
                     scaling="strong", bcell=0.25,
                     label="Game of Life 65536x65536 WRAP, random p=0.5 (splitmix64 seed 0x5EED0003), "
@@ -53,7 +53,20 @@ WORKLOADS = {
                   scaling="weak", bcell=8.0,
                   label="fp32 9x9 (r=4) window stencil, 32768 wide x 4096 rows per GPU, ZERO, 100 iterations per "
                         "step (BASELINE configs[4], weak scaling)"),
+    "hist8k": dict(op="histogram", w=8192, h=8192, r=0, b="no_checks", n=1, seed=0x5EED0006, wseed=None,
+                   scaling="strong", bcell=1.0,
+                   label="256-bin histogram of an 8192x8192 u8 image, uniform pixels (seed 0x5EED0006), one "
+                         "Reductive-Static task per step (SURVEY §8(f) NEXT-1; the paper's 8K image, P:L477-479)"),
 }
+
+
+def metric_of(wl):
+    if wl["op"] == "life":
+        return "Game of Life cell-updates/s", "cell-updates/s"
+    if wl["op"] == "conv":
+        k = 2 * wl["r"] + 1
+        return f"fp32 {k}x{k} window-conv cell-updates/s", "cell-updates/s"
+    return "256-bin histogram pixels/s", "pixels/s"
 
 
 def load_peaks():
@@ -116,73 +129,87 @@ class ClockSampler:
                 "reasons": sorted(reasons), "samples": len(sm)}
 
 
-def cpu_baseline(wl, budget_s=12.0):
-    """Time the oracle (as it stands) on a bounded sample of the workload."""
+# ------------------------------------------------------------------ oracle leg
+
+def _oracle_sample(wl):
+    """(run(k), work units per iteration, description) for a bounded sample."""
     import mapsm_inputs as mi
     import oracle
 
     w = wl["w"]
-    rows = 512 if wl["op"] == "life" else 256
     if wl["op"] == "life":
+        rows = 512
         g0 = mi.life_u8(wl["seed"], w, rows)
-        run = lambda n: oracle.life(g0, n, wl["b"])
-    else:
+        return (lambda k: oracle.life(g0, k, wl["b"])), w * rows, f"{w} x {rows} rows"
+    if wl["op"] == "conv":
+        rows = 256
         g0 = mi.field_f32(wl["seed"], w, rows)
         W = mi.weights_f32(wl["wseed"], wl["r"])
-        run = lambda n: oracle.conv(g0, W, n, wl["b"])
+        return (lambda k: oracle.conv(g0, W, k, wl["b"])), w * rows, f"{w} x {rows} rows"
+    img = mi.image_u8(wl["seed"], w, wl["h"])
+
+    def run(k):
+        for _ in range(k):
+            oracle.histogram(img)
+    return run, w * wl["h"], f"the full {w} x {wl['h']} image"
+
+
+def _oracle_threads(wl):
+    import oracle
+
+    return 1 if wl["op"] == "histogram" else oracle.num_threads()  # the histogram oracle is sequential
+
+
+def cpu_baseline(wl, budget_s=12.0):
+    """Time the oracle (as it stands) on a bounded sample of the workload."""
+    run, units, what = _oracle_sample(wl)
     t0 = time.perf_counter()
     run(1)
     t1 = time.perf_counter() - t0
-    n = max(1, min(wl["n"], int(budget_s / max(t1, 1e-6))))
+    cap = wl["n"] if wl["op"] != "histogram" else 50
+    n = max(1, min(cap, int(budget_s / max(t1, 1e-6))))
     t0 = time.perf_counter()
     run(n)
     dt = time.perf_counter() - t0
-    return {"value": w * rows * n / dt, "unit": "cell-updates/s", "cores": oracle.num_threads(), "kind": "oracle",
-            "sample": f"{w} x {rows} rows of the same {wl['op']} workload ({wl['b']} boundary on the sample), "
-                      f"{n} iterations, {dt:.1f} s wall (oracle.c, OpenMP, byte/cell Life or fmaf-chain conv)"}
+    _, unit = metric_of(wl)
+    return {"value": units * n / dt, "unit": unit, "cores": _oracle_threads(wl), "kind": "oracle",
+            "sample": f"{what} of the same {wl['op']} workload ({wl['b']} boundary on the sample), {n} iterations, "
+                      f"{dt:.1f} s wall (oracle/oracle.c)"}
 
 
 def run_reference(args, wl, rank, world):
     """Reference arm of this tier: the oracle as it stands, on the host cores,
-    rank 0 only; each step is a bounded sample (full width, 512 or 256 rows,
-    k iterations) of the same workload, sized so W+K steps take ~1 minute."""
+    rank 0 only; each step is a bounded sample of the same workload, sized so
+    W+K steps take ~1 minute."""
     if rank != 0:
         return
-    import mapsm_inputs as mi
-    import oracle
-
-    w = wl["w"]
-    rows = 512 if wl["op"] == "life" else 256
-    if wl["op"] == "life":
-        g0 = mi.life_u8(wl["seed"], w, rows)
-        run = lambda k: oracle.life(g0, k, wl["b"])
-    else:
-        g0 = mi.field_f32(wl["seed"], w, rows)
-        W = mi.weights_f32(wl["wseed"], wl["r"])
-        run = lambda k: oracle.conv(g0, W, k, wl["b"])
+    run, units, what = _oracle_sample(wl)
     t0 = time.perf_counter()
     run(1)
     t1 = time.perf_counter() - t0
-    per_step = max(1, min(wl["n"], int(60.0 / max(1, args.steps + args.warmup) / max(t1, 1e-6))))
+    cap = wl["n"] if wl["op"] != "histogram" else 50
+    per_step = max(1, min(cap, int(60.0 / max(1, args.steps + args.warmup) / max(t1, 1e-6))))
     for _ in range(args.warmup):
         run(per_step)
     t0 = time.perf_counter()
     for _ in range(args.steps):
         run(per_step)
     dt = time.perf_counter() - t0
-    value = w * rows * per_step * args.steps / dt
-    cb = {"value": value, "unit": "cell-updates/s", "cores": oracle.num_threads(), "kind": "oracle",
-          "sample": f"per step: {w} x {rows} rows, {per_step} iterations of the same workload "
-                    f"({wl['b']} boundary on the sample); {args.steps} timed steps, {dt:.1f} s"}
-    metric = "Game of Life cell-updates/s" if wl["op"] == "life" else f"fp32 {2*wl['r']+1}x{2*wl['r']+1} window-conv cell-updates/s"
-    line = {"impl": "reference", "metric": metric, "value": value, "unit": "cell-updates/s",
+    value = units * per_step * args.steps / dt
+    metric, unit = metric_of(wl)
+    cb = {"value": value, "unit": unit, "cores": _oracle_threads(wl), "kind": "oracle",
+          "sample": f"per step: {what}, {per_step} iterations of the same workload; {args.steps} timed steps, "
+                    f"{dt:.1f} s"}
+    line = {"impl": "reference", "metric": metric, "value": value, "unit": unit,
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
             "higher_is_better": True, "scaling": wl["scaling"], "vs_baseline": None,
-            "dtype": "u8" if wl["op"] == "life" else "f32", "data": "synthetic",
+            "dtype": "f32" if wl["op"] == "conv" else "u8", "data": "synthetic",
             "config": {"workload": wl["label"]}, "cpu_baseline": cb,
-            "e2e": {"value": value, "unit": "cell-updates/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
+            "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
 
+
+# ------------------------------------------------------------------ GPU leg
 
 def main():
     ap = argparse.ArgumentParser()
@@ -225,25 +252,36 @@ def main():
         uid = obj[0]
     ctx = M.mapsm_ctx_create(rank, world, local_rank, uid, stream.cuda_stream)
 
+    op = wl["op"]
     w = wl["w"]
     h = wl["h"] * (world if wl["scaling"] == "weak" else 1)
     n = wl["n"]
-    W = mi.weights_f32(wl["wseed"], wl["r"]) if wl["op"] == "conv" else None
-    grid = M.Grid(ctx, w, h, wl["op"], wl["r"], wl["b"], W)
+    W = mi.weights_f32(wl["wseed"], wl["r"]) if op == "conv" else None
+    grid = M.Grid(ctx, w, h, op, wl["r"], wl["b"], W)
     if args.graph_iters:
         grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
     y0, rows = grid.local_rows()
-    host_dtype = torch.uint8 if wl["op"] == "life" else torch.float32
+    host_dtype = torch.float32 if op == "conv" else torch.uint8
     # pinned host rows of this rank (input and result buffers for e2e)
     h_in = torch.empty((rows, w), dtype=host_dtype, pin_memory=True)
-    if wl["op"] == "life":
+    if op == "life":
         mi.life_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
-    else:
+    elif op == "conv":
         mi.field_f32(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
-    h_out = torch.empty_like(h_in, pin_memory=True)
+    else:
+        mi.image_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
+    h_out = torch.empty_like(h_in, pin_memory=True) if op != "histogram" else None
+    d_bins = torch.zeros(256, dtype=torch.int64, device=dev)
+    h_bins = torch.zeros(256, dtype=torch.int64, pin_memory=True)
     grid.bind(h_in)
     info0 = grid.info()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
+
+    def step():
+        if op == "histogram":
+            M.mapsm_histogram(grid.handle, d_bins)
+        else:
+            grid.iterate(n)
 
     def barrier():
         if world > 1:
@@ -252,7 +290,7 @@ def main():
 
     # warm-up (graph capture, NCCL connections, clocks)
     for _ in range(args.warmup):
-        grid.iterate(n)
+        step()
     barrier()
 
     # timed region: K steps, L2 flushed between steps outside the events
@@ -266,7 +304,7 @@ def main():
         e0 = torch.cuda.Event(enable_timing=True)
         e1 = torch.cuda.Event(enable_timing=True)
         e0.record(stream)
-        grid.iterate(n)
+        step()
         e1.record(stream)
         e1.synchronize()
         total_ms += e0.elapsed_time(e1)
@@ -281,53 +319,60 @@ def main():
         dist.all_reduce(tl, op=dist.ReduceOp.SUM)
     total_ms = float(t.item())
     total_launches = int(tl.item())
-    cells_per_step = w * h * n
-    value = cells_per_step * args.steps / (total_ms / 1e3)
+    units_per_step = w * h * n
+    value = units_per_step * args.steps / (total_ms / 1e3)
     ms_per_step = total_ms / args.steps
 
-    # Dominant-kernel timing: CUDA events around every bulk launch on the
-    # launching stream (direct launches, same kernels/config) for one step.
-    grid.set_option(M.OPT_TIMING, 1)
-    grid.iterate(n)
-    bulk_ms, bulk_n, bnd_ms, bnd_n = M.mapsm_get_timing(grid.handle)
-    grid.set_option(M.OPT_TIMING, 0)
     peak_gbs, peak_src = load_peaks()
     bcell = wl["bcell"]
     slab_cells = rows * w
-    if world == 1:
-        # whole step = back-to-back bulk launches: region time / launches, measured over the timed region
-        per_launch_s = (total_ms / 1e3) / max(1, launches)
-        achieved_region = bcell * slab_cells / per_launch_s / 1e9
+    # achieved over the timed region: each stencil step is n back-to-back bulk
+    # launches (N == 1), the histogram step one launch (plus its aggregation)
+    bulk_launches_per_step = n if op != "histogram" else 1
+    per_launch_s = (total_ms / 1e3) / (args.steps * bulk_launches_per_step)
+    achieved_region = bcell * slab_cells / per_launch_s / 1e9
+    kernel = {"life": "life_tma_kernel", "conv": "conv_tma_kernel", "histogram": "histogram_kernel"}[op]
+    roofline = {"bound": "hbm", "peak": peak_gbs, "unit": "GB/s", "kernel": kernel,
+                "bytes_per_unit": bcell, "algorithmic_bytes_per_launch": bcell * slab_cells, "peak_source": peak_src}
+    per_kernel_s = None
+    if op != "histogram":
+        # CUDA events around every bulk launch on the launching stream
+        # (direct launches, same kernels and configuration) for one step
+        grid.set_option(M.OPT_TIMING, 1)
+        grid.iterate(n)
+        bulk_ms, bulk_n, bnd_ms, bnd_n = M.mapsm_get_timing(grid.handle)
+        grid.set_option(M.OPT_TIMING, 0)
+        bulk_rows = rows if bnd_n == 0 else rows - 2 * wl["r"]
+        per_kernel_s = (bulk_ms / 1e3) / max(1, bulk_n)
+        achieved_kernel = bcell * bulk_rows * w / per_kernel_s / 1e9
+        roofline["achieved_events_per_launch_GBps"] = achieved_kernel
+        roofline["kernel_ms_per_launch"] = per_kernel_s * 1e3
+        achieved = achieved_region if world == 1 else achieved_kernel
     else:
-        achieved_region = None
-    bulk_rows = rows if bnd_n == 0 else rows - 2 * wl["r"]
-    per_kernel_s = (bulk_ms / 1e3) / max(1, bulk_n)
-    achieved_kernel = bcell * bulk_rows * w / per_kernel_s / 1e9
-    achieved = achieved_region if achieved_region is not None else achieved_kernel
-    traffic = None
+        achieved = achieved_region
+        roofline["note"] = ("whole step timed (memset + kernel + aggregation + bins copy); the 64 MiB image "
+                            "is re-read from HBM after each L2 flush")
+    roofline["achieved"] = achieved
+    roofline["frac"] = achieved / peak_gbs
+    roofline["frac_vs_8TBps_spec"] = achieved / 8000.0
+    roofline["traffic"] = None
     tfile = os.path.join(ROOT, "profiles", "traffic.json")
     if os.path.exists(tfile):
         try:
-            traffic = json.load(open(tfile)).get(args.workload)
+            roofline["traffic"] = json.load(open(tfile)).get(args.workload)
         except Exception:
-            traffic = None
-    roofline = {"bound": "hbm", "achieved": achieved, "peak": peak_gbs, "unit": "GB/s",
-                "frac": achieved / peak_gbs, "traffic": traffic,
-                "kernel": "life_step_kernel" if wl["op"] == "life" else "conv_step_kernel",
-                "bytes_per_cell_update": bcell, "algorithmic_bytes_per_launch": bcell * slab_cells,
-                "peak_source": peak_src, "achieved_events_per_launch_GBps": achieved_kernel,
-                "kernel_ms_per_launch": per_kernel_s * 1e3,
-                "frac_vs_8TBps_spec": achieved / 8000.0}
-    if wl["op"] == "conv":
-        # 9x9 is FP32-FMA bound; report the FMA-pipe fraction alongside
+            pass
+    if op == "conv":
         fma_per_cell = (2 * wl["r"] + 1) ** 2
         sm_mhz = clocks.get("sm_mhz") or 1965.0
         fma_peak = 148 * 128 * sm_mhz * 1e6
         roofline["fma_frac_at_sampled_clock"] = (bulk_rows * w * fma_per_cell / per_kernel_s) / fma_peak
+        if wl["r"] >= 3:
+            roofline["note"] = "9x9 is FP32-FMA bound (20.25 FMA/B): fma_frac is the binding fraction"
 
     # halo-exchange exposure (N > 1): same steps without the exchange
     exposure = None
-    if world > 1:
+    if world > 1 and op != "histogram":
         grid.set_option(M.OPT_NO_EXCHANGE, 1)
         grid.iterate(n)
         barrier()
@@ -352,39 +397,46 @@ def main():
         barrier()
         e0.record(stream)
         grid.bind(h_in)
-        grid.iterate(n)
-        M.mapsm_read(grid.handle, h_out)
+        if op == "histogram":
+            M.mapsm_histogram(grid.handle, h_bins)
+        else:
+            grid.iterate(n)
+            M.mapsm_read(grid.handle, h_out)
         e1.record(stream)
         e1.synchronize()
         e2e_ms += e0.elapsed_time(e1)
     te = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_value = cells_per_step * args.e2e_steps / (float(te.item()) / 1e3)
-    elem = 1 if wl["op"] == "life" else 4
+    e2e_value = units_per_step * args.e2e_steps / (float(te.item()) / 1e3)
+    elem = 4 if op == "conv" else 1
+    h2d = h * w * elem
+    d2h = 256 * 8 * world if op == "histogram" else h * w * elem
 
     grid.close()
     M.mapsm_ctx_destroy(ctx)
 
     if rank == 0:
         cb = None if args.no_cpu_baseline else cpu_baseline(wl)
-        ws_mib = 2 * (rows + 2 * wl["r"]) * info0.pitch_bytes / 2**20
-        metric = ("Game of Life cell-updates/s" if wl["op"] == "life"
-                  else f"fp32 {2*wl['r']+1}x{2*wl['r']+1} window-conv cell-updates/s")
+        nbuf = 1 if op == "histogram" else 2
+        ws_mib = nbuf * (rows + 2 * wl["r"]) * info0.pitch_bytes / 2**20
+        metric, unit = metric_of(wl)
+        dtype = {"life": "u32 bit-sliced (1 bit/cell)", "conv": "f32", "histogram": "u8 in, u32/u64 counts"}[op]
+        para = f"row-slab x{world}"
+        if world > 1:
+            para += " + NCCL allreduce of bins" if op == "histogram" else " + NCCL halo exchange"
         line = {
-            "metric": metric, "value": value, "unit": "cell-updates/s", "n_gpus": world, "steps": args.steps,
+            "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": wl["scaling"], "vs_baseline": None,
-            "dtype": "u32 bit-sliced (1 bit/cell)" if wl["op"] == "life" else "f32",
-            "data": "synthetic",
+            "scaling": wl["scaling"], "vs_baseline": None, "dtype": dtype, "data": "synthetic",
             "config": {"workload": wl["label"], "w": w, "h": h, "iterations_per_step": n, "radius": wl["r"],
-                       "boundary": wl["b"], "parallelism": f"row-slab x{world}" + (" + NCCL halo exchange" if world > 1 else ""),
-                       "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU double-buffer "
-                             f"working set {ws_mib:.0f} MiB vs 126 MB L2",
+                       "boundary": wl["b"], "parallelism": para,
+                       "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU working set "
+                             f"{ws_mib:.0f} MiB vs 126 MB L2",
                        "cuda_graphs": used_graphs},
-            "e2e": {"value": e2e_value, "unit": "cell-updates/s", "h2d_bytes_per_step": h * w * elem,
-                    "d2h_bytes_per_step": h * w * elem,
-                    "how": "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step"},
+            "e2e": {"value": e2e_value, "unit": unit, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                    "how": ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step" if op == "histogram"
+                            else "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")},
             "gpu_launches": total_launches,
             "roofline": roofline,
             "clocks": clocks,

@@ -11,14 +11,18 @@
  * partitioning ... evenly distributing the thread-blocks among the devices",
  * P:L59), with the r halo rows the Window pattern implies exchanged between
  * neighbouring slabs every iteration ("two-line boundary exchanges per
- * iteration").  Two operators:
+ * iteration").  Three operators:
  *   - MAPSM_OP_LIFE: Conway's Game of Life, B3/S23 on the 3x3 window (P:L133,
  *     Gardner [14] P:L619), radius 1, u8 cells on the host (nonzero = alive),
  *     bit-packed 32 cells per 32-bit word on the device;
  *   - MAPSM_OP_CONV: fp32 window convolution (Table 1, "N-dimensional
  *     convolution"), cross-correlation with (2r+1)^2 row-major weights,
  *     1 <= r <= 4, one fmaf per tap in row-major (dy, dx) order starting from
- *     +0.0f (reading c11) so results are reproducible bit for bit.
+ *     +0.0f (reading c11) so results are reproducible bit for bit;
+ *   - MAPSM_OP_HISTOGRAM: the Reductive (Static) output pattern (P:L104,
+ *     Fig 4): 256-bin histogram of a u8 image (bin = pixel value,
+ *     64-bit counts) over a radius-0 NO_CHECKS window; per-slab partial
+ *     histograms are aggregated across slabs.
  * Boundaries (the Window container's "boundary condition management",
  * P:L115; WRAP is the paper's GoL mode): WRAP = torus on both axes,
  * CLAMP = replicate the nearest edge cell, ZERO = constant 0 outside.
@@ -72,8 +76,10 @@ typedef enum {
 } mapsm_status;
 
 typedef enum { MAPSM_U8 = 1, MAPSM_F32 = 2 } mapsm_dtype;
-typedef enum { MAPSM_WRAP = 0, MAPSM_CLAMP = 1, MAPSM_ZERO = 2 } mapsm_boundary;
-typedef enum { MAPSM_OP_LIFE = 0, MAPSM_OP_CONV = 1 } mapsm_op;
+/* MAPSM_NO_CHECKS: the paper's boundary mode for a radius-0 window (Fig 4,
+ * P:L369), used by the histogram's 1x1 Window input. */
+typedef enum { MAPSM_WRAP = 0, MAPSM_CLAMP = 1, MAPSM_ZERO = 2, MAPSM_NO_CHECKS = 3 } mapsm_boundary;
+typedef enum { MAPSM_OP_LIFE = 0, MAPSM_OP_CONV = 1, MAPSM_OP_HISTOGRAM = 2 } mapsm_op;
 
 /* How a slab obtains the r rows just above (top) / below (bottom) its owned
  * rows — the Segment Location Monitor's answer (Alg 2) for this path. */
@@ -142,13 +148,16 @@ mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, mapsm_dtype 
 /* Window(2D) pattern: radius and boundary.  Partitions the rows over
  * the slabs and allocates both buffers of every local slab with 2r halo rows
  * (the Memory Analyzer's bounding box after both AnalyzeCalls, P:L167-169,
- * P:L281).  EUNSUPPORTED: Life with r != 1, conv with r outside 1..4.
- * EINVAL: a slab would have fewer than r rows (g > 1), or Life with w % 64
- * != 0.  ENOMEM on allocation failure.                                       */
+ * P:L281).  U8 grids: radius 1 = Life (bit-packed storage), radius 0 with
+ * NO_CHECKS = histogram input (byte storage, one buffer).  F32: radius 1..4.
+ * EUNSUPPORTED: any other radius/boundary combination.  EINVAL: a slab would
+ * have fewer than r rows (g > 1), or Life with w % 64 != 0.  ENOMEM on
+ * allocation failure.                                                        */
 mapsm_status mapsm_window_set(mapsm_grid grid, int radius, mapsm_boundary boundary);
 
-/* Operator: LIFE (weights must be NULL, dtype U8) or CONV (weights = (2r+1)^2
- * fp32 values, row-major over (dy, dx), copied; dtype F32).                  */
+/* Operator: LIFE (weights must be NULL, dtype U8, r = 1), CONV (weights =
+ * (2r+1)^2 fp32 values, row-major over (dy, dx), copied; dtype F32) or
+ * HISTOGRAM (weights NULL, dtype U8, r = 0).                                 */
 mapsm_status mapsm_op_set(mapsm_grid grid, mapsm_op op, const float* weights);
 
 /* Owned rows of local slab `local_index` (0 in multi-process mode).          */
@@ -171,6 +180,14 @@ mapsm_status mapsm_sync(mapsm_grid grid);
  * to `ptr` on rank `root` (other ranks pass NULL).  Life output bytes are
  * exactly 0/1.  Collective; synchronises.                                    */
 mapsm_status mapsm_gather(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, int root);
+
+/* Reductive (Static) aggregate (Fig 4; duplicate-and-aggregate
+ * P:L103-105): the 256-bin histogram of the bound image (all slabs of all
+ * processes: per-slab shared-memory bins, device-side sum across local slabs,
+ * ncclAllReduce across processes) written to bins[0..255] (host or device
+ * memory, 64-bit counts) on every process.  nbins must be 256; the grid's op
+ * must be HISTOGRAM (else ESTATE).  Collective; synchronises.              */
+mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
 
 /* Copy only this process's own rows (same row range as mapsm_bind) to `ptr`;
  * not collective; synchronises.                                              */

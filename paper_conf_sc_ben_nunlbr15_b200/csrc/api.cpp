@@ -85,6 +85,7 @@ struct NcclApi {
     decltype(&ncclRecv) recv = nullptr;
     decltype(&ncclGroupStart) groupStart = nullptr;
     decltype(&ncclGroupEnd) groupEnd = nullptr;
+    decltype(&ncclAllReduce) allReduce = nullptr;
     decltype(&ncclGetErrorString) errStr = nullptr;
 };
 static NcclApi g_nccl;
@@ -105,6 +106,7 @@ static mapsm_status nccl_load() {
     SYM(recv, "ncclRecv");
     SYM(groupStart, "ncclGroupStart");
     SYM(groupEnd, "ncclGroupEnd");
+    SYM(allReduce, "ncclAllReduce");
     SYM(errStr, "ncclGetErrorString");
 #undef SYM
     g_nccl.h = h;
@@ -146,6 +148,7 @@ struct Slab {
     cudaEvent_t ev_b = nullptr, ev_h = nullptr;
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int64_t graph_iters = 0;
+    unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
     void* staging = nullptr;   // device staging for host bind/gather (Life)
     int64_t staging_bytes = 0;
     std::vector<TimingPair> t_bulk, t_bnd;
@@ -171,6 +174,7 @@ struct mapsm_grid_s {
     bool opt_graphs = true, opt_no_exchange = false, opt_timing = false;
     int64_t opt_graph_iters = 16;
     bool used_graphs = false;
+    bool packed() const { return dtype == MAPSM_U8 && r == 1; }   // Life: bit-packed rows
 };
 
 static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
@@ -302,6 +306,7 @@ static void free_slab(Slab& s) {
     for (int b = 0; b < 2; ++b)
         if (s.base[b]) cudaFree(s.base[b]);
     if (s.staging) cudaFree(s.staging);
+    if (s.hist) cudaFree(s.hist);
     for (int b = 0; b < 2; ++b)
         if (s.graph[b]) cudaGraphExecDestroy(s.graph[b]);
     for (auto& t : s.t_bulk) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
@@ -316,11 +321,15 @@ static void free_slab(Slab& s) {
 extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundary boundary) {
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
     if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "window_set after bind (allocation depends on r)");
-    if (boundary != MAPSM_WRAP && boundary != MAPSM_CLAMP && boundary != MAPSM_ZERO)
+    if (boundary != MAPSM_WRAP && boundary != MAPSM_CLAMP && boundary != MAPSM_ZERO && boundary != MAPSM_NO_CHECKS)
         return fail(MAPSM_EINVAL, "boundary %d", (int)boundary);
+    if ((radius == 0) != (boundary == MAPSM_NO_CHECKS))
+        return fail(MAPSM_EUNSUPPORTED, "NO_CHECKS goes with radius 0 (histogram input), got r=%d b=%d", radius,
+                    (int)boundary);
     if (g->dtype == MAPSM_U8) {
-        if (radius != 1) return fail(MAPSM_EUNSUPPORTED, "Life (u8) needs radius 1, got %d", radius);
-        if (g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
+        if (radius != 1 && radius != 0)
+            return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
+        if (radius == 1 && g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
     } else {
         if (radius < 1 || radius > 4) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..4, got %d", radius);
     }
@@ -338,7 +347,7 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     g->device_bytes = 0;
     g->r = radius;
     g->boundary = boundary;
-    const int64_t row_bytes = g->dtype == MAPSM_U8 ? g->w / 8 : g->w * 4;
+    const int64_t row_bytes = g->packed() ? g->w / 8 : g->w * g->elem;
     const int64_t align = row_bytes >= 128 ? 128 : 16;
     g->pitch = (row_bytes + align - 1) / align * align;
     const int nloc = c->local ? c->g : 1;
@@ -351,7 +360,12 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         CK(cudaSetDevice(s.device));
         CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
         const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
-        for (int b = 0; b < 2; ++b) {
+        const int nbuf = radius == 0 ? 1 : 2;  // a reductive (non-iterated) task needs no double buffer
+        if (radius == 0) {
+            CK(cudaMalloc(&s.hist, 256 * sizeof(unsigned long long)));
+            g->device_bytes += 256 * sizeof(unsigned long long);
+        }
+        for (int b = 0; b < nbuf; ++b) {
             cudaError_t e = cudaMalloc(&s.base[b], bytes);
             if (e != cudaSuccess) {
                 cudaGetLastError();
@@ -376,7 +390,10 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     }
     CK(cudaDeviceSynchronize());
     g->state = ST_WINDOW;
-    if (g->dtype == MAPSM_U8) g->state = ST_OP;  // Life is the only u8 operator; op_set optional
+    if (g->dtype == MAPSM_U8) {  // one operator per u8 radius: op_set is optional
+        g->op = radius == 1 ? MAPSM_OP_LIFE : MAPSM_OP_HISTOGRAM;
+        g->state = ST_OP;
+    }
     return MAPSM_OK;
 }
 
@@ -384,8 +401,12 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
     if (g->state < ST_WINDOW) return fail(MAPSM_ESTATE, "op_set before window_set");
     if (op == MAPSM_OP_LIFE) {
-        if (g->dtype != MAPSM_U8) return fail(MAPSM_EUNSUPPORTED, "Life needs dtype U8");
+        if (g->dtype != MAPSM_U8 || g->r != 1) return fail(MAPSM_EUNSUPPORTED, "Life needs dtype U8 and radius 1");
         if (weights) return fail(MAPSM_EINVAL, "Life takes no weights");
+    } else if (op == MAPSM_OP_HISTOGRAM) {
+        if (g->dtype != MAPSM_U8 || g->r != 0)
+            return fail(MAPSM_EUNSUPPORTED, "histogram needs dtype U8 and radius 0 (NO_CHECKS)");
+        if (weights) return fail(MAPSM_EINVAL, "histogram takes no weights");
     } else if (op == MAPSM_OP_CONV) {
         if (g->dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "conv needs dtype F32");
         if (!weights) return fail(MAPSM_EINVAL, "conv needs (2r+1)^2 weights");
@@ -590,6 +611,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "iterate before bind");
     if (n < 0) return fail(MAPSM_EINVAL, "n < 0");
     if (n == 0) return MAPSM_OK;
+    if (g->op == MAPSM_OP_HISTOGRAM) return fail(MAPSM_EUNSUPPORTED, "a Reductive (histogram) grid is not iterated");
     DeviceGuard dg;
     // CUDA graphs for the single-stream-per-process modes (g == 1 and NCCL);
     // local multi-slab mode issues directly (it is the single-GPU test vehicle).
@@ -693,8 +715,8 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
             if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
         const char* src = static_cast<const char*>(ptr) + (s.plan.y0 - y_first) * pitch;
         const int64_t rows = s.plan.rows;
-        if (g->dtype == MAPSM_F32) {
-            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->pitch, src, pitch, g->w * 4, rows, cudaMemcpyDefault,
+        if (!g->packed()) {
+            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->pitch, src, pitch, g->w * g->elem, rows, cudaMemcpyDefault,
                                  s.main));
         } else if (on_dev && pdev == s.device) {
             CK(launch_pack_life(reinterpret_cast<const uint8_t*>(src), pitch, row_ptr(g, s, 0, 0), g->pitch, rows,
@@ -739,8 +761,8 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
 // Copy owned rows of the current buffer of slab s to dst (pitch dpitch).
 static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitch, bool dst_on_dev) {
     const int64_t rows = s.plan.rows;
-    if (g->dtype == MAPSM_F32) {
-        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->pitch, g->w * 4, rows, cudaMemcpyDefault,
+    if (!g->packed()) {
+        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->pitch, g->w * g->elem, rows, cudaMemcpyDefault,
                              s.main));
         return MAPSM_OK;
     }
@@ -837,6 +859,49 @@ extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int
     cudaStreamSynchronize(s.main);
     cudaFree(tmp);
     if (st != MAPSM_OK) return st;
+    return check_async(g);
+}
+
+// ---------------------------------------------------------------- histogram
+
+extern "C" mapsm_status mapsm_histogram(mapsm_grid g, uint64_t* bins, int nbins) {
+    if (!g || !bins) return fail(MAPSM_EINVAL, "NULL argument");
+    if (nbins != 256) return fail(MAPSM_EINVAL, "nbins must be 256");
+    if (g->state < ST_BOUND || g->op != MAPSM_OP_HISTOGRAM) return fail(MAPSM_ESTATE, "histogram needs a bound HISTOGRAM grid");
+    DeviceGuard dg;
+    mapsm_ctx c = g->ctx;
+    // 1. per-slab partial histograms (shared-memory bins + one commit per CTA)
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(launch_histogram(reinterpret_cast<const uint8_t*>(row_ptr(g, s, 0, 0)), g->pitch, g->w, s.plan.rows, s.hist,
+                            s.num_sms, s.main));
+        g->launches++;
+        CK(cudaEventRecord(s.ev_b, s.main));
+    }
+    // 2. aggregate the duplicated outputs: local slabs summed on
+    //    slab 0's device, then across processes with ncclAllReduce.
+    Slab& s0 = g->slabs[0];
+    CK(cudaSetDevice(s0.device));
+    if (g->slabs.size() > 1) {
+        const int n = (int)g->slabs.size();
+        std::vector<const unsigned long long*> parts(n);
+        for (int k = 0; k < n; ++k) {
+            parts[k] = g->slabs[k].hist;
+            if (k) CK(cudaStreamWaitEvent(s0.main, g->slabs[k].ev_b, 0));
+        }
+        TRY(ensure_staging(s0, (int64_t)(n * sizeof(void*) + 256 * sizeof(unsigned long long))));
+        auto* dparts = static_cast<const unsigned long long**>(s0.staging);
+        auto* sum = reinterpret_cast<unsigned long long*>(static_cast<char*>(s0.staging) + n * sizeof(void*) +
+                                                          (8 - (n * sizeof(void*)) % 8) % 8);
+        CK(cudaMemcpyAsync(dparts, parts.data(), n * sizeof(void*), cudaMemcpyHostToDevice, s0.main));
+        CK(launch_histogram_sum(dparts, n, sum, s0.main));
+        g->launches++;
+        CK(cudaMemcpyAsync(s0.hist, sum, 256 * sizeof(unsigned long long), cudaMemcpyDeviceToDevice, s0.main));
+        CK(cudaStreamSynchronize(s0.main));  // `parts` is host memory read by the async copy
+    }
+    if (c->world > 1)
+        NK(g_nccl.allReduce(s0.hist, s0.hist, 256, ncclUint64, ncclSum, c->comm, s0.main));
+    CK(cudaMemcpyAsync(bins, s0.hist, 256 * sizeof(unsigned long long), cudaMemcpyDefault, s0.main));
     return check_async(g);
 }
 

@@ -48,4 +48,11 @@ cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst,
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
                              int num_sms, cudaStream_t s);
 
+// Reductive (Static) output: 256-bin histogram of a u8 slab into out[256]
+// (zeroed here; 64-bit counts); and the sum of g partial histograms.
+cudaError_t launch_histogram(const uint8_t* img, int64_t pitch, int64_t w, int64_t rows, unsigned long long* out,
+                             int num_sms, cudaStream_t s);
+cudaError_t launch_histogram_sum(const unsigned long long* const* parts_dev, int g, unsigned long long* out,
+                                 cudaStream_t s);
+
 }  // namespace mapsm

@@ -20,7 +20,8 @@ namespace mapsm {
 
 mapsm_status compute_plan(int64_t h, int g, int r, mapsm_boundary b, int rank, mapsm_slab_plan* out) {
     if (!out || g < 1 || h < 1 || r < 0 || rank < 0 || rank >= g) return MAPSM_EINVAL;
-    if (b != MAPSM_WRAP && b != MAPSM_CLAMP && b != MAPSM_ZERO) return MAPSM_EINVAL;
+    if (b != MAPSM_WRAP && b != MAPSM_CLAMP && b != MAPSM_ZERO && b != MAPSM_NO_CHECKS) return MAPSM_EINVAL;
+    if (b == MAPSM_NO_CHECKS && r != 0) return MAPSM_EINVAL;  // NO_CHECKS = no neighbours (radius 0)
     const int64_t base = h / g, extra = h % g;
     if (g > 1 && base < r) return MAPSM_EINVAL;  // a halo row would not belong to a neighbour
     mapsm_slab_plan p;

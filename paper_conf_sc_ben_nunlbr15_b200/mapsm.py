@@ -20,17 +20,17 @@ _LIB_PATH = os.environ.get("MAPSM_LIB") or os.path.join(os.path.dirname(os.path.
 # enums (include/mapsm.h)
 OK, EINVAL, ENOMEM, ECUDA, ENCCL, ESTATE, EUNSUPPORTED = 0, -1, -2, -3, -4, -5, -6
 U8, F32 = 1, 2
-WRAP, CLAMP, ZERO = 0, 1, 2
-OP_LIFE, OP_CONV = 0, 1
+WRAP, CLAMP, ZERO, NO_CHECKS = 0, 1, 2, 3
+OP_LIFE, OP_CONV, OP_HISTOGRAM = 0, 1, 2
 HALO_EXCHANGE, HALO_WRAP_LOCAL, HALO_CLAMP, HALO_ZERO = 0, 1, 2, 3
 OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING = 1, 2, 3, 4
 
-BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO}
+BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO, "no_checks": NO_CHECKS}
 
 EXPORTED = [
     "mapsm_plan_query", "mapsm_ctx_create", "mapsm_ctx_create_local", "mapsm_ctx_destroy",
     "mapsm_nccl_unique_id", "mapsm_grid_create", "mapsm_window_set", "mapsm_op_set", "mapsm_grid_slab",
-    "mapsm_bind", "mapsm_iterate", "mapsm_sync", "mapsm_gather", "mapsm_read", "mapsm_grid_destroy",
+    "mapsm_bind", "mapsm_iterate", "mapsm_sync", "mapsm_gather", "mapsm_read", "mapsm_histogram", "mapsm_grid_destroy",
     "mapsm_get_info", "mapsm_set_option", "mapsm_get_timing", "mapsm_grid_stream", "mapsm_status_string",
     "mapsm_last_error", "mapsm_version",
 ]
@@ -85,6 +85,7 @@ def lib() -> ctypes.CDLL:
         "mapsm_sync": [vp],
         "mapsm_gather": [vp, vp, i64, ci],
         "mapsm_read": [vp, vp, i64],
+        "mapsm_histogram": [vp, vp, ci],
         "mapsm_grid_destroy": [vp],
         "mapsm_get_info": [vp, P(mapsm_grid_info)],
         "mapsm_set_option": [vp, ci, i64],
@@ -211,6 +212,14 @@ def mapsm_read(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
     _check(lib().mapsm_read(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read")
 
 
+def mapsm_histogram(grid: int, bins=None) -> np.ndarray:
+    """Reductive-Static aggregate: 256 uint64 counts (into `bins` if given:
+    a numpy array or a torch tensor, host or device)."""
+    out = np.zeros(256, dtype=np.uint64) if bins is None else bins
+    _check(lib().mapsm_histogram(grid, _ptr(out), 256), "mapsm_histogram")
+    return out
+
+
 def mapsm_grid_destroy(grid: int) -> None:
     _check(lib().mapsm_grid_destroy(grid), "mapsm_grid_destroy")
 
@@ -253,12 +262,16 @@ class Grid:
                  weights=None):
         self.ctx, self.w, self.h = ctx, w, h
         self.op = op
-        self.dtype = U8 if op == "life" else F32
+        self.dtype = F32 if op == "conv" else U8
+        if op == "histogram":
+            radius, boundary = 0, "no_checks"
         self.handle = mapsm_grid_create(ctx, w, h, self.dtype)
         try:
             mapsm_window_set(self.handle, radius, BOUNDARY[boundary] if isinstance(boundary, str) else boundary)
             if op == "life":
                 mapsm_op_set(self.handle, OP_LIFE, None)
+            elif op == "histogram":
+                mapsm_op_set(self.handle, OP_HISTOGRAM, None)
             else:
                 mapsm_op_set(self.handle, OP_CONV, weights)
         except Exception:
@@ -293,6 +306,9 @@ class Grid:
             out = np.empty((self.h, self.w), dtype=np.uint8 if self.dtype == U8 else np.float32)
         mapsm_gather(self.handle, out, None, root)
         return out
+
+    def histogram(self, bins=None):
+        return mapsm_histogram(self.handle, bins)
 
     def info(self) -> mapsm_grid_info:
         return mapsm_get_info(self.handle)

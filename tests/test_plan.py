@@ -87,3 +87,10 @@ def test_min_slab_height_equals_r():
 def test_bench_configs_partition(g, h):
     for p in plans(h, g, 4 if h == 32768 else 1, M.WRAP):
         assert p.rows == h // g
+
+
+def test_no_checks_is_radius_zero_only():
+    p = M.mapsm_plan_query(100, 4, 0, M.NO_CHECKS, 2)
+    assert p.rows == 25 and p.n_recv == 0 and p.alloc_rows == 25
+    with pytest.raises(M.MapsmError):
+        M.mapsm_plan_query(100, 4, 1, M.NO_CHECKS, 0)
