@@ -218,12 +218,17 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *   MAPSM_OPT_NO_EXCHANGE 1 = skip the halo exchange (bench only: measures
  *                         exchange exposure; results are then WRONG for g > 1)
  *   MAPSM_OPT_TIMING      1 = record CUDA events around every compute kernel
- *                         (forces direct launches); read with mapsm_get_timing */
+ *                         (forces direct launches); read with mapsm_get_timing
+ *   MAPSM_OPT_PERSISTENT  1 (default) Life slabs without exchanged halos whose
+ *                         double buffer fits in L2 (<= 64 MiB) run up to 1024
+ *                         generations per cooperative launch (grid barrier
+ *                         between generations); 0 = one launch per generation */
 typedef enum {
     MAPSM_OPT_GRAPHS = 1,
     MAPSM_OPT_GRAPH_ITERS = 2,
     MAPSM_OPT_NO_EXCHANGE = 3,
-    MAPSM_OPT_TIMING = 4
+    MAPSM_OPT_TIMING = 4,
+    MAPSM_OPT_PERSISTENT = 5
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

@@ -149,6 +149,7 @@ struct Slab {
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int64_t graph_iters = 0;
     unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
+    unsigned int* gbar = nullptr;        // grid-barrier word of the persistent Life kernel
     void* staging = nullptr;   // device staging for host bind/gather (Life)
     int64_t staging_bytes = 0;
     std::vector<TimingPair> t_bulk, t_bnd;
@@ -171,7 +172,7 @@ struct mapsm_grid_s {
     std::vector<Slab> slabs;
     int cur = 0;                    // buffer holding the current generation
     int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
-    bool opt_graphs = true, opt_no_exchange = false, opt_timing = false;
+    bool opt_graphs = true, opt_no_exchange = false, opt_timing = false, opt_persistent = true;
     int64_t opt_graph_iters = 16;
     bool used_graphs = false;
     bool packed() const { return dtype == MAPSM_U8 && r == 1; }   // Life: bit-packed rows
@@ -307,6 +308,7 @@ static void free_slab(Slab& s) {
         if (s.base[b]) cudaFree(s.base[b]);
     if (s.staging) cudaFree(s.staging);
     if (s.hist) cudaFree(s.hist);
+    if (s.gbar) cudaFree(s.gbar);
     for (int b = 0; b < 2; ++b)
         if (s.graph[b]) cudaGraphExecDestroy(s.graph[b]);
     for (auto& t : s.t_bulk) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
@@ -613,6 +615,34 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     if (n == 0) return MAPSM_OK;
     if (g->op == MAPSM_OP_HISTOGRAM) return fail(MAPSM_EUNSUPPORTED, "a Reductive (histogram) grid is not iterated");
     DeviceGuard dg;
+    // L2-resident Life slabs with no exchanged halos: persistent kernel, up to
+    // kPersistChunk generations per cooperative launch.
+    if (g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 &&
+        !has_exchange(g->slabs[0]) && 2 * g->slabs[0].plan.alloc_rows * g->pitch <= (64ll << 20)) {
+        Slab& s = g->slabs[0];
+        CK(cudaSetDevice(s.device));
+        if (!s.gbar) CK(cudaMalloc(&s.gbar, sizeof(unsigned int)));
+        const int64_t kPersistChunk = 1024;
+        for (int64_t done = 0; done < n;) {
+            const int64_t k = (n - done < kPersistChunk) ? n - done : kPersistChunk;
+            StencilGeom geom;
+            geom.in = row_ptr(g, s, g->cur, 0);
+            geom.out = row_ptr(g, s, g->cur ^ 1, 0);
+            geom.pitch = g->pitch;
+            geom.rows = s.plan.rows;
+            geom.w = g->w;
+            geom.top_map = rowmap_of(s.plan.top_kind);
+            geom.bot_map = rowmap_of(s.plan.bottom_kind);
+            geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+            cudaError_t e = launch_life_persistent(geom, k, s.gbar, s.num_sms, s.main);
+            if (e != cudaSuccess) return fail(MAPSM_ECUDA, "persistent Life launch: %s", cudaGetErrorString(e));
+            g->launches++;
+            if (k & 1) g->cur ^= 1;
+            g->gen += k;
+            done += k;
+        }
+        return MAPSM_OK;
+    }
     // CUDA graphs for the single-stream-per-process modes (g == 1 and NCCL);
     // local multi-slab mode issues directly (it is the single-GPU test vehicle).
     const bool graphs = g->opt_graphs && !g->opt_timing && !g->ctx->local;
@@ -949,6 +979,7 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             g->opt_graph_iters = v;
             break;
         case MAPSM_OPT_NO_EXCHANGE: g->opt_no_exchange = v != 0; break;
+        case MAPSM_OPT_PERSISTENT: g->opt_persistent = v != 0; break;
         case MAPSM_OPT_TIMING:
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;

@@ -39,6 +39,11 @@ struct RowBands {
 // `resident_warps` = warps the device keeps resident for this kernel
 // (persistent-style row chunking); 0 = compute from the occupancy API.
 cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s);
+// n generations of a whole slab (no exchanged halos) in ONE cooperative
+// launch with a grid barrier between generations; g.in/g.out are the buffers
+// of generation 0 / 1 (generation n ends in g.in if n is even, else g.out).
+// `bar` = one device word of barrier state.
+cudaError_t launch_life_persistent(const StencilGeom& g, int64_t n, unsigned int* bar, int num_sms, cudaStream_t s);
 cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, int64_t dst_pitch,
                              int64_t rows, int64_t w, cudaStream_t s);
 cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst, int64_t dst_pitch,

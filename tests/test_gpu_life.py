@@ -14,11 +14,13 @@ pytestmark = pytest.mark.gpu
 GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
 
 
-def run(ctx, g0, n, b, steps=None, graphs=True, graph_iters=None):
+def run(ctx, g0, n, b, steps=None, graphs=True, graph_iters=None, persistent=True):
     h, w = g0.shape
     with M.Grid(ctx, w, h, "life", 1, b) as g:
         if not graphs:
             g.set_option(M.OPT_GRAPHS, 0)
+        if not persistent:
+            g.set_option(M.OPT_PERSISTENT, 0)
         if graph_iters:
             g.set_option(M.OPT_GRAPH_ITERS, graph_iters)
         g.bind(g0)
@@ -37,6 +39,9 @@ def test_config0_closed_form(ctx):
             exp[y, x] = 1
     out, info = run(ctx, mi.config0_grid(), 100, "wrap")
     assert np.array_equal(out, exp)
+    assert info.generation == 100 and info.launches == 1  # persistent kernel: one launch
+    out, info = run(ctx, mi.config0_grid(), 100, "wrap", persistent=False)
+    assert np.array_equal(out, exp)
     assert info.generation == 100 and info.launches == 100
 
 
@@ -44,10 +49,11 @@ def test_config0_closed_form(ctx):
 @pytest.mark.parametrize("shape", [(64, 1), (64, 2), (64, 3), (128, 130), (192, 77), (320, 64), (1024, 333),
                                    (4096, 257), (8192 + 64, 100)])
 @pytest.mark.parametrize("n", [0, 1, 2, 7])
-def test_random_vs_oracle(ctx, b, shape, n):
+@pytest.mark.parametrize("persistent", [True, False])
+def test_random_vs_oracle(ctx, b, shape, n, persistent):
     w, h = shape
     g0 = mi.life_u8(1000 + w + h, w, h)
-    out, _ = run(ctx, g0, n, b)
+    out, _ = run(ctx, g0, n, b, persistent=persistent)
     assert np.array_equal(out, oracle.life(g0, n, b))
 
 
@@ -79,12 +85,14 @@ def test_all_512_neighbourhoods_at_word_edges(ctx, center, b):
 def test_graphs_direct_and_split_calls_agree(ctx):
     g0 = mi.life_u8(5, 512, 300)
     exp = oracle.life(g0, 37, "wrap")
-    a, ia = run(ctx, g0, 37, "wrap")
-    b, ib = run(ctx, g0, 37, "wrap", graphs=False)
-    c, _ = run(ctx, g0, 37, "wrap", steps=[5, 6, 1, 20, 5], graph_iters=4)
-    assert np.array_equal(a, exp) and np.array_equal(b, exp) and np.array_equal(c, exp)
+    a, ia = run(ctx, g0, 37, "wrap", persistent=False)
+    b, ib = run(ctx, g0, 37, "wrap", graphs=False, persistent=False)
+    c, _ = run(ctx, g0, 37, "wrap", steps=[5, 6, 1, 20, 5], graph_iters=4, persistent=False)
+    d, idd = run(ctx, g0, 37, "wrap", steps=[5, 6, 1, 20, 5])
+    assert np.array_equal(a, exp) and np.array_equal(b, exp) and np.array_equal(c, exp) and np.array_equal(d, exp)
     assert ia.used_graphs == 1 and ib.used_graphs == 0
     assert ia.launches == ib.launches == 37
+    assert idd.launches == 5 and idd.used_graphs == 0  # persistent: one launch per iterate call
 
 
 @pytest.mark.parametrize("g", [2, 3, 4, 8])
@@ -97,6 +105,14 @@ def test_local_multislab_partition_invariance(local_ctx, g, b):
     assert info.world == g and info.local_slabs == g
     exp_recv = sum(M.mapsm_plan_query(h, g, 1, M.BOUNDARY[b], k).n_recv for k in range(g))
     assert info.exchanges == exp_recv * n
+
+
+def test_persistent_long_run_many_chunks(ctx):
+    """> 1024 generations: several persistent launches, odd total."""
+    g0 = mi.life_u8(77, 256, 96)
+    out, info = run(ctx, g0, 2051, "wrap")
+    assert np.array_equal(out, oracle.life(g0, 2051, "wrap"))
+    assert info.launches == 3
 
 
 def test_local_multislab_min_height(local_ctx):
@@ -151,7 +167,7 @@ def test_config2_8192_full_run_sampled(ctx):
     n = 1000
     g0 = mi.life_u8(mi.SEED_LIFE_8K, w, h)
     out, info = run(ctx, g0, n, "wrap")
-    assert info.used_graphs == 1
+    assert info.launches == 1  # the bench's path for this L2-resident grid: one persistent launch
     gen = lambda y0, k: mi.life_u8(mi.SEED_LIFE_8K, w, k, y0=y0)
     for (ys, xs) in [(0, 0), (4000, 6000), (8190, 8160)]:
         exp = cone_eval("life", gen, h, w, 1, n, "wrap", ys, ys + 2, xs, xs + 32)
