@@ -222,13 +222,27 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *   MAPSM_OPT_PERSISTENT  1 (default) Life slabs without exchanged halos whose
  *                         double buffer fits in L2 (<= 64 MiB) run up to 1024
  *                         generations per cooperative launch (grid barrier
- *                         between generations); 0 = one launch per generation */
+ *                         between generations); 0 = one launch per generation
+ *   MAPSM_OPT_EXCHANGE    MAPSM_EXCHANGE_COPY (default): boundary-row kernel,
+ *                         then NCCL send/recv (multi-process) or peer
+ *                         cudaMemcpyAsync (single process) on a side stream,
+ *                         overlapped with the interior kernel.
+ *                         MAPSM_EXCHANGE_P2P: ONE fused kernel per iteration
+ *                         whose boundary CTAs store their rows straight into
+ *                         the neighbours' halo rows (NVLink peer stores via
+ *                         CUDA IPC, or same-process pointers) and signal them
+ *                         through a device mailbox; the neighbour's CTAs that
+ *                         need those rows wait on it.  Needs rows per slab >
+ *                         2r and the TMA kernels (Life w % 128 == 0, conv
+ *                         w % 4 == 0); set before bind.                       */
+typedef enum { MAPSM_EXCHANGE_COPY = 0, MAPSM_EXCHANGE_P2P = 1 } mapsm_exchange;
 typedef enum {
     MAPSM_OPT_GRAPHS = 1,
     MAPSM_OPT_GRAPH_ITERS = 2,
     MAPSM_OPT_NO_EXCHANGE = 3,
     MAPSM_OPT_TIMING = 4,
-    MAPSM_OPT_PERSISTENT = 5
+    MAPSM_OPT_PERSISTENT = 5,
+    MAPSM_OPT_EXCHANGE = 6
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

@@ -86,6 +86,7 @@ struct NcclApi {
     decltype(&ncclGroupStart) groupStart = nullptr;
     decltype(&ncclGroupEnd) groupEnd = nullptr;
     decltype(&ncclAllReduce) allReduce = nullptr;
+    decltype(&ncclAllGather) allGather = nullptr;
     decltype(&ncclGetErrorString) errStr = nullptr;
 };
 static NcclApi g_nccl;
@@ -107,6 +108,7 @@ static mapsm_status nccl_load() {
     SYM(groupStart, "ncclGroupStart");
     SYM(groupEnd, "ncclGroupEnd");
     SYM(allReduce, "ncclAllReduce");
+    SYM(allGather, "ncclAllGather");
     SYM(errStr, "ncclGetErrorString");
 #undef SYM
     g_nccl.h = h;
@@ -150,6 +152,15 @@ struct Slab {
     int64_t graph_iters = 0;
     unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
     unsigned int* gbar = nullptr;        // grid-barrier word of the persistent Life kernel
+    // fused peer-memory exchange (MAPSM_OPT_EXCHANGE = P2P): my mailbox and
+    // the neighbours' buffers / mailboxes (same process, or CUDA IPC)
+    void* mailbox = nullptr;
+    char* up_base[2] = {nullptr, nullptr};
+    char* down_base[2] = {nullptr, nullptr};
+    char* up_mail = nullptr;
+    char* down_mail = nullptr;
+    int64_t up_rows = 0;                 // owned rows of the up neighbour (its bottom halo follows them)
+    std::vector<void*> ipc_opened;       // peer mappings to close at destroy
     void* staging = nullptr;   // device staging for host bind/gather (Life)
     int64_t staging_bytes = 0;
     std::vector<TimingPair> t_bulk, t_bnd;
@@ -173,10 +184,14 @@ struct mapsm_grid_s {
     int cur = 0;                    // buffer holding the current generation
     int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
     bool opt_graphs = true, opt_no_exchange = false, opt_timing = false, opt_persistent = true;
+    bool opt_p2p = false;       // fused compute + peer-memory halo exchange
+    bool p2p_linked = false;    // peer pointers resolved
     int64_t opt_graph_iters = 16;
     bool used_graphs = false;
     bool packed() const { return dtype == MAPSM_U8 && r == 1; }   // Life: bit-packed rows
 };
+
+static const size_t kMailboxBytes = 64;  // >= sizeof(tma::Mailbox)
 
 static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
     return s.base[b] + (y + g->r) * g->pitch;
@@ -309,6 +324,8 @@ static void free_slab(Slab& s) {
     if (s.staging) cudaFree(s.staging);
     if (s.hist) cudaFree(s.hist);
     if (s.gbar) cudaFree(s.gbar);
+    if (s.mailbox) cudaFree(s.mailbox);
+    for (void* q : s.ipc_opened) cudaIpcCloseMemHandle(q);
     for (int b = 0; b < 2; ++b)
         if (s.graph[b]) cudaGraphExecDestroy(s.graph[b]);
     for (auto& t : s.t_bulk) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
@@ -363,6 +380,8 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
         const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
         const int nbuf = radius == 0 ? 1 : 2;  // a reductive (non-iterated) task needs no double buffer
+        CK(cudaMalloc(&s.mailbox, kMailboxBytes));
+        CK(cudaMemset(s.mailbox, 0, kMailboxBytes));
         if (radius == 0) {
             CK(cudaMalloc(&s.hist, 256 * sizeof(unsigned long long)));
             g->device_bytes += 256 * sizeof(unsigned long long);
@@ -389,6 +408,12 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         CK(cudaStreamCreateWithFlags(&s.side, cudaStreamNonBlocking));
         CK(cudaEventCreateWithFlags(&s.ev_b, cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&s.ev_h, cudaEventDisableTiming));
+    }
+    // slabs sharing a device split its SMs (their kernels run concurrently)
+    for (auto& s : g->slabs) {
+        int same = 0;
+        for (auto& t : g->slabs) same += t.device == s.device;
+        if (same > 1) s.num_sms = s.num_sms / same > 0 ? s.num_sms / same : 1;
     }
     CK(cudaDeviceSynchronize());
     g->state = ST_WINDOW;
@@ -484,7 +509,8 @@ static mapsm_status exchange_nccl(mapsm_grid_s* g, int b) {
 
 // ------------------------------------------------------------- compute step
 
-static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk) {
+static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk,
+                                const FusedLink* link = nullptr) {
     StencilGeom geom;
     geom.in = row_ptr(g, s, b_in, 0);
     geom.out = row_ptr(g, s, b_in ^ 1, 0);
@@ -509,9 +535,9 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
     }
     cudaError_t e;
     if (g->op == MAPSM_OP_LIFE)
-        e = launch_life_step(geom, bands, s.num_sms, s.main);
+        e = launch_life_step(geom, bands, s.num_sms, s.main, link);
     else
-        e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main);
+        e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main, link);
     if (e != cudaSuccess) return fail(MAPSM_ECUDA, "stencil launch: %s", cudaGetErrorString(e));
     if (tp) CK(cudaEventRecord(tp->b, s.main));
     g->launches++;
@@ -582,6 +608,132 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
     return MAPSM_OK;
 }
 
+// ------------------------------------------------ fused peer-memory exchange
+
+// Can this grid run the fused exchange?  (TMA kernels, every slab > 2r rows.)
+static bool p2p_eligible(const mapsm_grid_s* g) {
+    if (g->op != MAPSM_OP_LIFE && g->op != MAPSM_OP_CONV) return false;
+    if (g->op == MAPSM_OP_LIFE && ((g->w / 32) % 4 != 0 || g->pitch % 16 != 0)) return false;
+    if (g->op == MAPSM_OP_CONV && (g->w % 4 != 0 || g->pitch % 16 != 0)) return false;
+    return g->h / g->ctx->g > 2 * (int64_t)g->r;
+}
+
+static bool fused_now(const mapsm_grid_s* g) {
+    if (!g->opt_p2p || g->opt_no_exchange) return false;
+    for (auto& s : g->slabs)
+        if (has_exchange(s)) return true;
+    return false;
+}
+
+// Resolve the neighbours' buffers and mailboxes: plain pointers between slabs
+// of one process; CUDA IPC handles (all-gathered with NCCL) across processes.
+static mapsm_status p2p_link(mapsm_grid_s* g) {
+    if (g->p2p_linked) return MAPSM_OK;
+    mapsm_ctx c = g->ctx;
+    if (c->local) {
+        for (auto& s : g->slabs) {
+            if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
+                Slab& u = g->slabs[s.plan.up];
+                s.up_base[0] = u.base[0];
+                s.up_base[1] = u.base[1];
+                s.up_mail = static_cast<char*>(u.mailbox);
+                s.up_rows = u.plan.rows;
+            }
+            if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
+                Slab& d = g->slabs[s.plan.down];
+                s.down_base[0] = d.base[0];
+                s.down_base[1] = d.base[1];
+                s.down_mail = static_cast<char*>(d.mailbox);
+            }
+        }
+        g->p2p_linked = true;
+        return MAPSM_OK;
+    }
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    const int W = c->world;
+    const size_t hb = 3 * sizeof(cudaIpcMemHandle_t);
+    std::vector<char> mine(hb), all(hb * W);
+    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()), s.base[0]));
+    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()) + 1, s.base[1]));
+    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()) + 2, s.mailbox));
+    char* dev = nullptr;
+    CK(cudaMalloc(&dev, hb * (W + 1)));
+    CK(cudaMemcpyAsync(dev, mine.data(), hb, cudaMemcpyHostToDevice, s.main));
+    ncclResult_t nr = g_nccl.allGather(dev, dev + hb, hb, ncclUint8, c->comm, s.main);
+    cudaError_t ce = cudaMemcpyAsync(all.data(), dev + hb, hb * W, cudaMemcpyDeviceToHost, s.main);
+    cudaError_t se = cudaStreamSynchronize(s.main);
+    cudaFree(dev);
+    if (nr != ncclSuccess) return fail(MAPSM_ENCCL, "IPC handle all-gather: %s", g_nccl.errStr(nr));
+    if (ce != cudaSuccess || se != cudaSuccess) return fail(MAPSM_ECUDA, "IPC handle all-gather copy failed");
+    auto open = [&](int rank, int k, void** out) -> mapsm_status {
+        cudaIpcMemHandle_t h;
+        memcpy(&h, all.data() + (size_t)rank * hb + k * sizeof(h), sizeof(h));
+        CK(cudaIpcOpenMemHandle(out, h, cudaIpcMemLazyEnablePeerAccess));
+        s.ipc_opened.push_back(*out);
+        return MAPSM_OK;
+    };
+    void* p[3];
+    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
+        for (int k = 0; k < 3; ++k) TRY(open(s.plan.up, k, &p[k]));
+        s.up_base[0] = static_cast<char*>(p[0]);
+        s.up_base[1] = static_cast<char*>(p[1]);
+        s.up_mail = static_cast<char*>(p[2]);
+        mapsm_slab_plan up;
+        compute_plan(g->h, c->g, g->r, g->boundary, s.plan.up, &up);
+        s.up_rows = up.rows;
+    }
+    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
+        if (s.plan.down == s.plan.up && s.up_mail) {  // g == 2 under WRAP: one peer, mapped once
+            s.down_base[0] = s.up_base[0];
+            s.down_base[1] = s.up_base[1];
+            s.down_mail = s.up_mail;
+        } else {
+            for (int k = 0; k < 3; ++k) TRY(open(s.plan.down, k, &p[k]));
+            s.down_base[0] = static_cast<char*>(p[0]);
+            s.down_base[1] = static_cast<char*>(p[1]);
+            s.down_mail = static_cast<char*>(p[2]);
+        }
+    }
+    g->p2p_linked = true;
+    return MAPSM_OK;
+}
+
+// One fused iteration: per slab ONE launch with bands [top boundary rows,
+// bottom boundary rows, interior]; the boundary CTAs deliver their rows into
+// the neighbours' halos of the output buffer and signal their mailboxes.
+static mapsm_status iterate_fused(mapsm_grid_s* g, int b_in) {
+    const int r = g->r;
+    const int bo = b_in ^ 1;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+        const int64_t rows = s.plan.rows;
+        RowBands bands;
+        bands.nbands = 0;
+        if (top) { bands.begin[bands.nbands] = 0; bands.end[bands.nbands] = r; bands.nbands++; }
+        if (bot) { bands.begin[bands.nbands] = rows - r; bands.end[bands.nbands] = rows; bands.nbands++; }
+        bands.begin[bands.nbands] = top ? r : 0;
+        bands.end[bands.nbands] = bot ? rows - r : rows;
+        bands.nbands++;
+        FusedLink L;
+        L.mailbox = s.mailbox;
+        L.dst_up = top ? s.up_base[bo] + (s.up_rows + r) * g->pitch : nullptr;  // up's row up_rows (bottom halo)
+        L.dst_down = bot ? s.down_base[bo] : nullptr;                           // down's row -r (top halo)
+        L.sig_up = top ? reinterpret_cast<unsigned int*>(s.up_mail + 16) : nullptr;      // recv_bot
+        L.sig_down = bot ? reinterpret_cast<unsigned int*>(s.down_mail + 12) : nullptr;  // recv_top
+        L.wait_top = top;
+        L.wait_bot = bot;
+        TRY(launch_step(g, s, b_in, bands, true, &L));
+        g->exchanges += s.plan.n_recv;
+    }
+    return MAPSM_OK;
+}
+
+static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
+    return fused_now(g) ? iterate_fused(g, b_in) : iterate_once(g, b_in);
+}
+
 static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters) {
     CK(cudaSetDevice(s.device));
     const int64_t l0 = g->launches, x0 = g->exchanges;
@@ -589,7 +741,7 @@ static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64
     mapsm_status st = MAPSM_OK;
     int cur = start_cur;
     for (int64_t k = 0; k < iters && st == MAPSM_OK; ++k) {
-        st = iterate_once(g, cur);
+        st = step_all(g, cur);
         cur ^= 1;
     }
     cudaGraph_t graph = nullptr;
@@ -661,7 +813,9 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
             // launches per iteration (for the counters; graphs replay them)
             RowBands bnd, inner;
             split_bands(g, s, bnd, inner);
-            per_graph_launches = has_exchange(s) ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0)) : 1;
+            per_graph_launches = (has_exchange(s) && !fused_now(g))
+                                     ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0))
+                                     : 1;
             per_graph_exch = (has_exchange(s) && !g->opt_no_exchange) ? s.plan.n_recv : 0;
         }
         while (n - done >= gi) {
@@ -677,7 +831,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
         }
     }
     for (; done < n; ++done) {
-        TRY(iterate_once(g, g->cur));
+        TRY(step_all(g, g->cur));
         g->cur ^= 1;
         g->gen++;
     }
@@ -774,6 +928,18 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     g->launches = 0;
     g->exchanges = 0;
     g->state = ST_BOUND;
+    if (g->opt_p2p) {
+        if (!p2p_eligible(g))
+            return fail(MAPSM_EUNSUPPORTED, "P2P exchange needs the TMA kernels (Life w %% 128, conv w %% 4) and slabs > 2r rows");
+        TRY(p2p_link(g));
+        // reset the mailboxes BEFORE the initial exchange: a neighbour cannot
+        // deliver generation 1 until that exchange (which needs us) completed
+        for (auto& s : g->slabs) {
+            CK(cudaSetDevice(s.device));
+            CK(cudaMemsetAsync(s.mailbox, 0, kMailboxBytes, s.main));
+            CK(cudaStreamSynchronize(s.main));
+        }
+    }
     // Fill the halos of the current buffer once (the first exchange).
     bool any = false;
     for (auto& s : g->slabs) any |= has_exchange(s);
@@ -980,6 +1146,12 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             break;
         case MAPSM_OPT_NO_EXCHANGE: g->opt_no_exchange = v != 0; break;
         case MAPSM_OPT_PERSISTENT: g->opt_persistent = v != 0; break;
+        case MAPSM_OPT_EXCHANGE:
+            if (v != MAPSM_EXCHANGE_COPY && v != MAPSM_EXCHANGE_P2P) return fail(MAPSM_EINVAL, "exchange mode %lld", (long long)v);
+            if (g->state >= ST_BOUND && (v == MAPSM_EXCHANGE_P2P) != g->opt_p2p)
+                return fail(MAPSM_ESTATE, "set MAPSM_OPT_EXCHANGE before bind");
+            g->opt_p2p = v == MAPSM_EXCHANGE_P2P;
+            break;
         case MAPSM_OPT_TIMING:
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;

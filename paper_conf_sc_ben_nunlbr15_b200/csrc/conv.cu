@@ -8,15 +8,15 @@ namespace mapsm {
 
 template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
-                               cudaStream_t s);
+                               cudaStream_t s, const FusedLink* link);
 
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights, int num_sms,
-                             cudaStream_t s) {
+                             cudaStream_t s, const FusedLink* link) {
     switch (r) {
-        case 1: return launch_conv_radius<1>(g, b, weights, num_sms, s);
-        case 2: return launch_conv_radius<2>(g, b, weights, num_sms, s);
-        case 3: return launch_conv_radius<3>(g, b, weights, num_sms, s);
-        case 4: return launch_conv_radius<4>(g, b, weights, num_sms, s);
+        case 1: return launch_conv_radius<1>(g, b, weights, num_sms, s, link);
+        case 2: return launch_conv_radius<2>(g, b, weights, num_sms, s, link);
+        case 3: return launch_conv_radius<3>(g, b, weights, num_sms, s, link);
+        case 4: return launch_conv_radius<4>(g, b, weights, num_sms, s, link);
         default: return cudaErrorInvalidValue;
     }
 }

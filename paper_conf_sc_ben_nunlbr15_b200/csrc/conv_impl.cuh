@@ -273,7 +273,7 @@ struct VecF<2> {
     using T = float2;
 };
 
-template <int R, int NC, int NS, int CM, int EPL>
+template <int R, int NC, int NS, int CM, int EPL, bool FUSED>
 __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) conv_tma_kernel(const __grid_constant__ ConvTmaParams<R> pp) {
     constexpr int K = 2 * R + 1;
     static_assert(NS % K == 0, "NS must be a multiple of 2R+1");
@@ -290,17 +290,22 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
     tma::Seg sg;
     tma::RingPos ring;
 
+    const tma::HaloLink& Lk = p.link;
     if (warp == NC) {
-        if (lane == 0) {
+        constexpr int PL = R <= 2 ? 2 : 1;  // producer lanes (see tma_rows.cuh)
+        if (lane < PL) {
+            const unsigned int halo_target =
+                FUSED ? (unsigned int)(Lk.mine->gen * (unsigned long long)(Lk.r * p.nstrips)) : 0u;
             while (tma::seg_next<NC, EPL>(p, it, sg)) {
-                tma::produce_align<NS>(full, empty, ring);
-                tma::produce<NC, NS, CM == COL_WRAP, EPL>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R,
-                                                         ring);
+                tma::produce_align<NS, PL>(full, empty, ring, lane);
+                tma::produce<NC, NS, CM == COL_WRAP, EPL, PL>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R,
+                                                         ring, halo_target, lane);
             }
         }
+        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32);
         return;
     }
-
+    {
     const int t = warp * 32 + lane;
     float acc[K][EPL];
     while (tma::seg_next<NC, EPL>(p, it, sg)) {
@@ -311,6 +316,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         const bool active = t * EPL < (int)sg.seg;
         const bool row_first = sg.first_strip && t == 0;
         const bool row_last = sg.last_strip && (t + 1) * EPL == (int)sg.seg;
+        const bool whole = sg.first_strip && sg.last_strip;
         float* out0 = static_cast<float*>(p.out) + sg.ys * p.pitch + sg.e0 + t * EPL;
 
         // Input row j: output rows o = j - d (d = 0..2R, tap row dy = d - R)
@@ -323,7 +329,14 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
             float buf[EPL + 8];
 #pragma unroll
             for (int m = 0; m < EPL + 8; m += EPL) {
-                const VT q = *reinterpret_cast<const VT*>(st + t * EPL + m);
+                // WRAP at the ends of a whole-row strip: the other end of the row
+                // is in the stage itself (no margin copy was made)
+                int off = t * EPL + m;
+                if (CM == COL_WRAP && whole) {
+                    if (m < 4 && row_first) off = (int)sg.seg + m;           // elements seg-4+m
+                    if (m >= 4 + EPL && row_last) off = m - EPL;             // elements m-4-EPL..
+                }
+                const VT q = *reinterpret_cast<const VT*>(st + off);
                 if constexpr (EPL == 4) {
                     buf[m] = q.x; buf[m + 1] = q.y; buf[m + 2] = q.z; buf[m + 3] = q.w;
                 } else {
@@ -358,12 +371,22 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                         acc[slot][q] = a;
                     }
                     if (d == K - 1 && active) {
+                        using OT = typename VecF<EPL>::T;
+                        OT ov;
                         if constexpr (EPL == 4)
-                            *reinterpret_cast<float4*>(out0 + (int64_t)o * p.pitch) =
-                                make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                            ov = make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
                         else
-                            *reinterpret_cast<float2*>(out0 + (int64_t)o * p.pitch) =
-                                make_float2(acc[slot][0], acc[slot][1]);
+                            ov = make_float2(acc[slot][0], acc[slot][1]);
+                        *reinterpret_cast<OT*>(out0 + (int64_t)o * p.pitch) = ov;
+                        if constexpr (FUSED) {  // boundary rows also go to the neighbours' halos
+                            const int64_t yo = sg.ys + o;
+                            if (Lk.dst_up && yo < R)
+                                *reinterpret_cast<OT*>(reinterpret_cast<float*>(Lk.dst_up) + yo * p.pitch + sg.e0 +
+                                                       t * EPL) = ov;
+                            if (Lk.dst_down && yo >= p.rows - R)
+                                *reinterpret_cast<OT*>(reinterpret_cast<float*>(Lk.dst_down) +
+                                                       (yo - (p.rows - R)) * p.pitch + sg.e0 + t * EPL) = ov;
+                        }
                     }
                 }
             }
@@ -391,12 +414,24 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         ring.stage = n_in % NS;
         ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
         ring.count += n_in;
+        if constexpr (FUSED) {
+            if (Lk.dst_up && sg.ys < R) {
+                const int64_t e = sg.ye < R ? sg.ye : R;
+                tma::publish_delivery(Lk.sig_up, (unsigned int)(e - sg.ys), NC);
+            }
+            if (Lk.dst_down && sg.ye > p.rows - R) {
+                const int64_t b0 = sg.ys > p.rows - R ? sg.ys : p.rows - R;
+                tma::publish_delivery(Lk.sig_down, (unsigned int)(sg.ye - b0), NC);
+            }
+        }
     }
+    }
+    if constexpr (FUSED) tma::finish_launch_consumers(Lk.mine, (NC + 1) * 32);
 }
 
 template <int R, int NC, int NS, int CM, int EPL>
 cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
-                              cudaStream_t s) {
+                              cudaStream_t s, const FusedLink* link) {
     using G = tma::Geom<NC, EPL>;
     constexpr int K = 2 * R + 1;
     ConvTmaParams<R> pp;
@@ -412,9 +447,12 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
     static int ctas_per_sm = 0;
     if (ctas_per_sm == 0) {
-        auto kfn = conv_tma_kernel<R, NC, NS, CM, EPL>;
-        cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-        if (e != cudaSuccess) return e;
+        auto kfn = conv_tma_kernel<R, NC, NS, CM, EPL, false>;
+        for (auto kf : {conv_tma_kernel<R, NC, NS, CM, EPL, false>, conv_tma_kernel<R, NC, NS, CM, EPL, true>}) {
+            cudaError_t e = cudaFuncSetAttribute(kf, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+            if (e != cudaSuccess) return e;
+        }
+        cudaError_t e;
         e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, kfn, (NC + 1) * 32, smem);
         if (e != cudaSuccess) return e;
         if (ctas_per_sm < 1) ctas_per_sm = 1;
@@ -423,24 +461,27 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
         const int want = R <= 2 ? (16 / NC > 0 ? 16 / NC : 1) : kConvBigCtas;
         if (want < ctas_per_sm) ctas_per_sm = want;
     }
-    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems);
+    tma_set_link(p, link, R);
+    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems, link != nullptr);
     if (ctas == 0) return cudaSuccess;
-    dim3 grid((unsigned)ctas, (unsigned)b.nbands);
-    conv_tma_kernel<R, NC, NS, CM, EPL><<<grid, (NC + 1) * 32, smem, s>>>(pp);
+    if (link)
+        conv_tma_kernel<R, NC, NS, CM, EPL, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(pp);
+    else
+        conv_tma_kernel<R, NC, NS, CM, EPL, false><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(pp);
     return cudaGetLastError();
 }
 
 template <int R, int NS>
 cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
-                            cudaStream_t s) {
+                            cudaStream_t s, const FusedLink* link) {
     constexpr int EPL = R <= 2 ? 4 : kConvBigEPL;
     const int64_t nvec = g.w / EPL;
     auto go = [&](auto nc_tag) -> cudaError_t {
         constexpr int NC = decltype(nc_tag)::value;
         switch (g.col_mode) {
-            case COL_WRAP: return launch_conv_tma_t<R, NC, NS, COL_WRAP, EPL>(g, b, weights, num_sms, s);
-            case COL_CLAMP: return launch_conv_tma_t<R, NC, NS, COL_CLAMP, EPL>(g, b, weights, num_sms, s);
-            default: return launch_conv_tma_t<R, NC, NS, COL_ZERO, EPL>(g, b, weights, num_sms, s);
+            case COL_WRAP: return launch_conv_tma_t<R, NC, NS, COL_WRAP, EPL>(g, b, weights, num_sms, s, link);
+            case COL_CLAMP: return launch_conv_tma_t<R, NC, NS, COL_CLAMP, EPL>(g, b, weights, num_sms, s, link);
+            default: return launch_conv_tma_t<R, NC, NS, COL_ZERO, EPL>(g, b, weights, num_sms, s, link);
         }
     };
     if constexpr (R <= 2 || kConvBigNC == 16) {
@@ -514,13 +555,14 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
 
 template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
-                               cudaStream_t s) {
+                               cudaStream_t s, const FusedLink* link) {
     constexpr int kNS = R == 1 ? 12 : R == 2 ? 10 : R == 3 ? 14 : 9;  // multiples of 2R+1
     constexpr int kPF = R <= 2 ? 2 : 1;
 #ifndef MAPSM_CONV_REGS
     if (g.w % 4 == 0 && g.w >= 4 && g.pitch % 16 == 0)
-        return conv_detail::launch_conv_tma<R, kNS>(g, b, weights, num_sms, s);
+        return conv_detail::launch_conv_tma<R, kNS>(g, b, weights, num_sms, s, link);
 #endif
+    if (link || b.nbands > 2) return cudaErrorInvalidValue;  // fused exchange needs the TMA kernel
     return conv_detail::launch_conv_t<R, kPF>(g, b, weights, num_sms, s);
 }
 

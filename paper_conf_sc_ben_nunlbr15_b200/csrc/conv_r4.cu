@@ -2,5 +2,6 @@
 #include "conv_impl.cuh"
 
 namespace mapsm {
-template cudaError_t launch_conv_radius<4>(const StencilGeom&, const RowBands&, const float*, int, cudaStream_t);
+template cudaError_t launch_conv_radius<4>(const StencilGeom&, const RowBands&, const float*, int, cudaStream_t,
+                                               const FusedLink*);
 }  // namespace mapsm

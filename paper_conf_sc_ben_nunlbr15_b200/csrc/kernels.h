@@ -31,14 +31,26 @@ struct StencilGeom {
 // Output-row bands computed by one launch (1 band = all rows or interior;
 // 2 bands = the boundary rows [0,r) and [rows-r,rows)).
 struct RowBands {
-    int64_t begin[2], end[2];
+    int64_t begin[3], end[3];
     int nbands;
+};
+
+// Fused peer-memory halo exchange of one launch (see tma_rows.cuh); all-null
+// = plain launch.  Pointers may address a peer GPU's memory (CUDA IPC).
+struct FusedLink {
+    void* mailbox;          // this slab's tma::Mailbox
+    void* dst_up;           // up neighbour: out-parity buffer at its bottom-halo row 0
+    void* dst_down;         // down neighbour: out-parity buffer at its top-halo row -r
+    unsigned int* sig_up;   // up neighbour's mailbox.recv_bot
+    unsigned int* sig_down; // down neighbour's mailbox.recv_top
+    int wait_top, wait_bot;
 };
 
 // Life (bit-packed: bit j of 32-bit word m of a row = column 32m + j).
 // `resident_warps` = warps the device keeps resident for this kernel
 // (persistent-style row chunking); 0 = compute from the occupancy API.
-cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s);
+cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
+                             const FusedLink* link = nullptr);
 // n generations of a whole slab (no exchanged halos) in ONE cooperative
 // launch with a grid barrier between generations; g.in/g.out are the buffers
 // of generation 0 / 1 (generation n ends in g.in if n is even, else g.out).
@@ -51,7 +63,7 @@ cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst,
 
 // fp32 window convolution, radius r in 1..4, weights (2r+1)^2 row-major.
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
-                             int num_sms, cudaStream_t s);
+                             int num_sms, cudaStream_t s, const FusedLink* link = nullptr);
 
 // Reductive (Static) output: 256-bin histogram of a u8 slab into out[256]
 // (zeroed here; 64-bit counts); and the sum of g partial histograms.

@@ -336,7 +336,7 @@ __global__ void __launch_bounds__(kPersistThreads) life_persist_kernel(const __g
 // neighbouring strips' edge words, or the WRAP source at the row ends), do the
 // bit-sliced update, and store straight to HBM.
 
-template <int NC, int NS, int CM>
+template <int NC, int NS, int CM, bool FUSED>
 __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_constant__ tma::RowStream p) {
     using G = tma::Geom<NC>;
     extern __shared__ __align__(128) uint8_t smem[];
@@ -347,104 +347,138 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
     tma::SegIter it = tma::seg_iter(p);
     tma::Seg sg;
     tma::RingPos ring;  // CTA-wide ring position (same sequence in producer and consumers)
+    const tma::HaloLink& L = p.link;
 
     if (warp == NC) {
         if (lane == 0) {
+            const unsigned int halo_target =
+                FUSED ? (unsigned int)(L.mine->gen * (unsigned long long)(L.r * p.nstrips)) : 0u;
             while (tma::seg_next<NC>(p, it, sg)) {
-                tma::produce_align<NS>(full, empty, ring);
-                tma::produce<NC, NS, CM == COL_WRAP>(p, sg, smem, full, empty, sg.ys - 1, sg.ye - sg.ys + 2, ring);
+                tma::produce_align<NS, 1>(full, empty, ring, lane);
+                tma::produce<NC, NS, CM == COL_WRAP, 4, 1>(p, sg, smem, full, empty, sg.ys - 1, sg.ye - sg.ys + 2, ring,
+                                                     halo_target, lane);
             }
         }
+        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32);
         return;
     }
+    {
+        // ------------------------------------------------------ consumers
+        // Input row j of a segment (global row ys-1+j) sits in stage (base+j) % NS
+        // with base a multiple of NS; the loop is unrolled by NS (a multiple of 3)
+        // so stage indices and the 3-row rotation of the row sums are
+        // compile-time register renames.
+        static_assert(NS % 3 == 0, "NS must be a multiple of 3");
+        const int t = warp * 32 + lane;  // vector index within the strip
+        uint32_t r0[3][4], r1[3][4], xs[3][4];  // row sums and raw words of 3 rows
+        while (tma::seg_next<NC>(p, it, sg)) {
+            tma::consume_align<NS>(full, empty, ring, lane);
+            uint32_t ph = ring.phase;  // segment starts at stage 0
+            const int n_in = (int)(sg.ye - sg.ys + 2);  // input rows ys-1 .. ye
+            const bool active = t * 4 < (int)sg.seg;
+            const bool row_first = sg.first_strip && t == 0;
+            const bool row_last = sg.last_strip && (t + 1) * 4 == (int)sg.seg;
+            const bool whole = sg.first_strip && sg.last_strip;
+            uint32_t* out_row = static_cast<uint32_t*>(p.out) + sg.ys * p.pitch + sg.e0 + t * 4;
+            int64_t yo = sg.ys;  // slab row of the next output
 
-    // ------------------------------------------------------ consumers
-    // Input row j of a segment (global row ys-1+j) sits in stage (base+j) % NS
-    // with base a multiple of NS; the loop is unrolled by NS (a multiple of 3)
-    // so stage indices and the 3-row rotation of the row sums are
-    // compile-time register renames.
-    static_assert(NS % 3 == 0, "NS must be a multiple of 3");
-    const int t = warp * 32 + lane;  // vector index within the strip
-    uint32_t r0[3][4], r1[3][4], xs[3][4];  // row sums and raw words of 3 rows
-    while (tma::seg_next<NC>(p, it, sg)) {
-        tma::consume_align<NS>(full, empty, ring, lane);
-        uint32_t ph = ring.phase;  // segment starts at stage 0
-        const int n_in = (int)(sg.ye - sg.ys + 2);  // input rows ys-1 .. ye
-        const bool active = t * 4 < (int)sg.seg;
-        const bool row_first = sg.first_strip && t == 0;
-        const bool row_last = sg.last_strip && (t + 1) * 4 == (int)sg.seg;
-        uint32_t* out_row = static_cast<uint32_t*>(p.out) + sg.ys * p.pitch + sg.e0 + t * 4;
+            auto consume = [&](int j, int k, int slot) {
+                // k = j % NS (static), slot = j % 3 (static)
+                tma::mbar_wait(&full[k], ph);
+                const uint32_t* st = reinterpret_cast<const uint32_t*>(smem + k * G::kStageBytes);
+                const uint4 v = *reinterpret_cast<const uint4*>(st + 4 + t * 4);
+                // neighbour words; at the row ends: WRAP -> the other end (from
+                // the stage itself when the strip is the whole row, else from
+                // the margin copy), CLAMP -> replicate, ZERO -> 0
+                uint32_t lw = st[(CM == COL_WRAP && row_first && whole) ? 4 + (int)sg.seg - 1 : 4 + t * 4 - 1];
+                uint32_t rw = st[(CM == COL_WRAP && row_last && whole) ? 4 : 4 + t * 4 + 4];
+                __syncwarp();
+                if (lane == 0) tma::mbar_arrive(&empty[k]);
+                if (CM != COL_WRAP) {
+                    if (row_first) lw = (CM == COL_CLAMP) ? (v.x << 31) : 0u;  // column -1 := column 0 / 0
+                    if (row_last) rw = (CM == COL_CLAMP) ? (v.w >> 31) : 0u;   // column w := column w-1 / 0
+                }
+                xs[slot][0] = v.x; xs[slot][1] = v.y; xs[slot][2] = v.z; xs[slot][3] = v.w;
+#pragma unroll
+                for (int q = 0; q < 4; ++q) {
+                    const uint32_t ls = (q == 0) ? lw : xs[slot][q - 1];
+                    const uint32_t rs = (q == 3) ? rw : xs[slot][q + 1];
+                    const uint32_t Lf = __funnelshift_l(ls, xs[slot][q], 1);
+                    const uint32_t Rf = __funnelshift_r(xs[slot][q], rs, 1);
+                    r0[slot][q] = Lf ^ xs[slot][q] ^ Rf;
+                    r1[slot][q] = maj3(Lf, xs[slot][q], Rf);
+                }
+            };
+            auto emit = [&](int slot) {
+                // centre row in slot (slot+2)%3, row above in (slot+1)%3, row below in slot
+                const int A = (slot + 1) % 3, B = (slot + 2) % 3, C = slot;
+                uint32_t o[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q)
+                    o[q] = life_word(r0[A][q], r1[A][q], r0[B][q], r1[B][q], r0[C][q], r1[C][q], xs[B][q]);
+                if (active) {
+                    const uint4 ov = make_uint4(o[0], o[1], o[2], o[3]);
+                    *reinterpret_cast<uint4*>(out_row) = ov;
+                    if constexpr (FUSED) {  // boundary rows also go to the neighbours' halos
+                        if (L.dst_up && yo < L.r)
+                            *reinterpret_cast<uint4*>(L.dst_up + yo * p.pitch + sg.e0 + t * 4) = ov;
+                        if (L.dst_down && yo >= p.rows - L.r)
+                            *reinterpret_cast<uint4*>(L.dst_down + (yo - (p.rows - L.r)) * p.pitch + sg.e0 + t * 4) =
+                                ov;
+                    }
+                }
+                out_row += p.pitch;
+                ++yo;
+            };
 
-        auto consume = [&](int j, int k, int slot) {
-            // k = j % NS (static), slot = j % 3 (static)
-            tma::mbar_wait(&full[k], ph);
-            const uint32_t* st = reinterpret_cast<const uint32_t*>(smem + k * G::kStageBytes);
-            const uint4 v = *reinterpret_cast<const uint4*>(st + 4 + t * 4);
-            uint32_t lw = st[4 + t * 4 - 1];
-            uint32_t rw = st[4 + t * 4 + 4];
-            __syncwarp();
-            if (lane == 0) tma::mbar_arrive(&empty[k]);
-            if (CM != COL_WRAP) {
-                if (row_first) lw = (CM == COL_CLAMP) ? (v.x << 31) : 0u;  // column -1 := column 0 / 0
-                if (row_last) rw = (CM == COL_CLAMP) ? (v.w >> 31) : 0u;   // column w := column w-1 / 0
-            }
-            xs[slot][0] = v.x; xs[slot][1] = v.y; xs[slot][2] = v.z; xs[slot][3] = v.w;
-#pragma unroll
-            for (int q = 0; q < 4; ++q) {
-                const uint32_t ls = (q == 0) ? lw : xs[slot][q - 1];
-                const uint32_t rs = (q == 3) ? rw : xs[slot][q + 1];
-                const uint32_t L = __funnelshift_l(ls, xs[slot][q], 1);
-                const uint32_t R = __funnelshift_r(xs[slot][q], rs, 1);
-                r0[slot][q] = L ^ xs[slot][q] ^ R;
-                r1[slot][q] = maj3(L, xs[slot][q], R);
-            }
-        };
-        auto emit = [&](int slot) {
-            // centre row in slot (slot+2)%3, row above in (slot+1)%3, row below in slot
-            const int A = (slot + 1) % 3, B = (slot + 2) % 3, C = slot;
-            uint32_t o[4];
-#pragma unroll
-            for (int q = 0; q < 4; ++q)
-                o[q] = life_word(r0[A][q], r1[A][q], r0[B][q], r1[B][q], r0[C][q], r1[C][q], xs[B][q]);
-            if (active) *reinterpret_cast<uint4*>(out_row) = make_uint4(o[0], o[1], o[2], o[3]);
-            out_row += p.pitch;
-        };
-
-        const uint32_t ph0 = ph;
-        int j = 0;
-        if (n_in >= NS) {
-            // first trip: input rows 0,1 only fill the window
-#pragma unroll
-            for (int k = 0; k < NS; ++k) {
-                consume(k, k, k % 3);
-                if (k >= 2) emit(k % 3);
-            }
-            ph ^= 1u;
-            for (j = NS; j + NS <= n_in; j += NS) {
+            const uint32_t ph0 = ph;
+            int j = 0;
+            if (n_in >= NS) {
+                // first trip: input rows 0,1 only fill the window
 #pragma unroll
                 for (int k = 0; k < NS; ++k) {
-                    consume(j + k, k, k % 3);
-                    emit(k % 3);
+                    consume(k, k, k % 3);
+                    if (k >= 2) emit(k % 3);
                 }
                 ph ^= 1u;
-            }
-        }
-        // last (partial) trip; j is a multiple of NS (and of 3)
+                for (j = NS; j + NS <= n_in; j += NS) {
 #pragma unroll
-        for (int k = 0; k < NS; ++k) {
-            if (j + k < n_in) {
-                consume(j + k, k, k % 3);
-                if (j + k >= 2) emit(k % 3);
+                    for (int k = 0; k < NS; ++k) {
+                        consume(j + k, k, k % 3);
+                        emit(k % 3);
+                    }
+                    ph ^= 1u;
+                }
+            }
+            // last (partial) trip; j is a multiple of NS (and of 3)
+#pragma unroll
+            for (int k = 0; k < NS; ++k) {
+                if (j + k < n_in) {
+                    consume(j + k, k, k % 3);
+                    if (j + k >= 2) emit(k % 3);
+                }
+            }
+            ring.stage = n_in % NS;
+            ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
+            ring.count += n_in;
+            if constexpr (FUSED) {
+                if (L.dst_up && sg.ys < L.r) {
+                    const int64_t e = sg.ye < L.r ? sg.ye : L.r;
+                    tma::publish_delivery(L.sig_up, (unsigned int)(e - sg.ys), NC);
+                }
+                if (L.dst_down && sg.ye > p.rows - L.r) {
+                    const int64_t b0 = sg.ys > p.rows - L.r ? sg.ys : p.rows - L.r;
+                    tma::publish_delivery(L.sig_down, (unsigned int)(sg.ye - b0), NC);
+                }
             }
         }
-        ring.stage = n_in % NS;
-        ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
-        ring.count += n_in;
     }
+    if constexpr (FUSED) tma::finish_launch_consumers(L.mine, (NC + 1) * 32);
 }
 
 template <int NC, int NS, int CM>
-cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
+                              const FusedLink* link) {
     using G = tma::Geom<NC>;
     tma::RowStream p;
     p.in = static_cast<const uint32_t*>(g.in);
@@ -457,27 +491,35 @@ cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_s
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
     static int ctas_per_sm = 0;
     if (ctas_per_sm == 0) {
-        cudaError_t e = cudaFuncSetAttribute(life_tma_kernel<NC, NS, CM>, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
-        if (e != cudaSuccess) return e;
-        e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, life_tma_kernel<NC, NS, CM>, (NC + 1) * 32, smem);
+        // occupancy of the plain kernel; the fused variant is launched with the same grid
+        for (auto kfn : {life_tma_kernel<NC, NS, CM, false>, life_tma_kernel<NC, NS, CM, true>}) {
+            cudaError_t e = cudaFuncSetAttribute(kfn, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+            if (e != cudaSuccess) return e;
+        }
+        cudaError_t e = cudaOccupancyMaxActiveBlocksPerMultiprocessor(&ctas_per_sm, life_tma_kernel<NC, NS, CM, false>,
+                                                                      (NC + 1) * 32, smem);
         if (e != cudaSuccess) return e;
         if (ctas_per_sm < 1) ctas_per_sm = 1;
         const int want = kTmaCtasPerSm > 0 ? kTmaCtasPerSm : (16 / NC > 0 ? 16 / NC : 1);
         if (want < ctas_per_sm) ctas_per_sm = want;
     }
-    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems);
+    tma_set_link(p, link, 1);
+    const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems, link != nullptr);
     if (ctas == 0) return cudaSuccess;
-    dim3 grid((unsigned)ctas, (unsigned)b.nbands);
-    life_tma_kernel<NC, NS, CM><<<grid, (NC + 1) * 32, smem, s>>>(p);
+    if (link)
+        life_tma_kernel<NC, NS, CM, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(p);
+    else
+        life_tma_kernel<NC, NS, CM, false><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(p);
     return cudaGetLastError();
 }
 
 template <int NC, int NS>
-cudaError_t launch_life_tma_nc(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+cudaError_t launch_life_tma_nc(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
+                               const FusedLink* link) {
     switch (g.col_mode) {
-        case COL_WRAP: return launch_life_tma_t<NC, NS, COL_WRAP>(g, b, num_sms, s);
-        case COL_CLAMP: return launch_life_tma_t<NC, NS, COL_CLAMP>(g, b, num_sms, s);
-        default: return launch_life_tma_t<NC, NS, COL_ZERO>(g, b, num_sms, s);
+        case COL_WRAP: return launch_life_tma_t<NC, NS, COL_WRAP>(g, b, num_sms, s, link);
+        case COL_CLAMP: return launch_life_tma_t<NC, NS, COL_CLAMP>(g, b, num_sms, s, link);
+        default: return launch_life_tma_t<NC, NS, COL_ZERO>(g, b, num_sms, s, link);
     }
 }
 
@@ -486,12 +528,13 @@ cudaError_t launch_life_tma_nc(const StencilGeom& g, const RowBands& b, int num_
 // ~16 consumer warps per SM in total (measured best: fewer, longer streams
 // keep HBM pages open — tools/membench.cu, profiles/).
 template <int NS>
-cudaError_t launch_life_tma(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+cudaError_t launch_life_tma(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
+                            const FusedLink* link) {
     const int64_t nvec = g.w / 128;  // 16-byte vectors per row
-    if (nvec > 8 * 32) return launch_life_tma_nc<16, NS>(g, b, num_sms, s);
-    if (nvec > 4 * 32) return launch_life_tma_nc<8, NS>(g, b, num_sms, s);
-    if (nvec > 2 * 32) return launch_life_tma_nc<4, NS>(g, b, num_sms, s);
-    return launch_life_tma_nc<2, NS>(g, b, num_sms, s);
+    if (nvec > 8 * 32) return launch_life_tma_nc<16, NS>(g, b, num_sms, s, link);
+    if (nvec > 4 * 32) return launch_life_tma_nc<8, NS>(g, b, num_sms, s, link);
+    if (nvec > 2 * 32) return launch_life_tma_nc<4, NS>(g, b, num_sms, s, link);
+    return launch_life_tma_nc<2, NS>(g, b, num_sms, s, link);
 }
 
 // ------------------------------------------------------------ pack / unpack
@@ -641,13 +684,11 @@ cudaError_t launch_life_persist_v(const StencilGeom& g, int64_t n, unsigned int*
     }
 }
 
-cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s) {
+cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
+                             const FusedLink* link) {
     const int64_t nw = g.w / 32;
-#ifdef MAPSM_LIFE_REGS
-    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_cm<4, kLifeP>(g, b, num_sms, s);
-#else
-    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_tma<kTmaNS>(g, b, num_sms, s);
-#endif
+    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_tma<kTmaNS>(g, b, num_sms, s, link);
+    if (link || b.nbands > 2) return cudaErrorInvalidValue;  // fused exchange needs the TMA kernel
     return launch_life_cm<2, kLifeP>(g, b, num_sms, s);
 }
 

@@ -74,6 +74,33 @@ struct Geom {
     static constexpr int kStageBytes = kStripElems * 4 + 32;  // + 16 B margin each side
 };
 
+constexpr int kMaxBands = 3;
+
+// Fused halo exchange over peer memory (MAPSM_OPT_EXCHANGE_P2P): the CTAs
+// that compute a slab's first / last r rows also store them into the
+// neighbours' halo rows (NVLink peer stores, or plain stores between slabs
+// on one device) and then add the number of rows delivered to the
+// neighbour's mailbox; a CTA that needs a halo row waits until its own
+// mailbox shows this generation's delivery.  Counters are monotonic; the
+// generation is kept in device memory so CUDA-graph replays stay correct.
+struct Mailbox {
+    unsigned long long gen;  // iterations completed since bind (incremented by the last CTA of each launch)
+    unsigned int done;       // CTAs finished in the current launch
+    unsigned int recv_top;   // rows delivered into my top halo since bind (all strips)
+    unsigned int recv_bot;   // rows delivered into my bottom halo since bind
+    unsigned int pad[3];
+};
+
+struct HaloLink {
+    Mailbox* mine;           // null: no fused exchange in this launch
+    uint32_t* dst_up;        // up neighbour's `out`-parity buffer at its bottom-halo row 0 (null: no up link)
+    uint32_t* dst_down;      // down neighbour's `out`-parity buffer at its top-halo row -r (null: no down link)
+    unsigned int* sig_up;    // &up.mailbox.recv_bot
+    unsigned int* sig_down;  // &down.mailbox.recv_top
+    int wait_top, wait_bot;  // my top / bottom halo is delivered by a neighbour
+    int r;                   // rows per delivery
+};
+
 struct RowStream {
     const uint32_t* in;   // owned row 0 of the input slab (4-byte elements)
     void* out;            // owned row 0 of the output slab
@@ -81,8 +108,11 @@ struct RowStream {
     int64_t rows;         // owned rows of the slab
     int64_t n;            // elements per row (multiple of 4)
     int64_t nstrips;
-    int64_t begin[2], end[2];  // output-row bands of this launch
+    int nbands;
+    int64_t begin[kMaxBands], end[kMaxBands];  // output-row bands of this launch
+    int cta_begin[kMaxBands + 1];              // CTAs [cta_begin[b], cta_begin[b+1]) work on band b
     int top_map, bot_map;
+    HaloLink link;
 };
 
 __device__ __forceinline__ int64_t map_row(const RowStream& p, int64_t y) {
@@ -100,11 +130,12 @@ __device__ __forceinline__ int64_t map_row(const RowStream& p, int64_t y) {
     return y;  // ROWMAP_HALO: the halo row itself (exchanged or zeroed)
 }
 
-// Work distribution.  The (strip, output row) space of a band is flattened
-// strip-major and split into gridDim.x equal contiguous ranges; a CTA's range
-// is a short list of segments (one strip, a run of rows each), so every SM
-// gets the same number of rows whatever the strip count (no idle SMs when
-// 148 is not a multiple of the number of strips).
+// Work distribution.  Each band owns a range of CTAs (1-D grid).  The
+// (strip, output row) space of a band is flattened strip-major and split into
+// equal contiguous ranges, one per CTA of the band; a CTA's range is a short
+// list of segments (one strip, a run of rows each), so every SM gets the same
+// number of rows whatever the strip count (no idle SMs when 148 is not a
+// multiple of the number of strips).
 struct Seg {
     int64_t ys, ye;     // output rows [ys, ye)
     int64_t e0, seg;    // first element and element count of the strip
@@ -117,13 +148,66 @@ struct SegIter {
 
 __device__ __forceinline__ SegIter seg_iter(const RowStream& p) {
     SegIter it;
-    const int band = blockIdx.y;
+    int band = 0;
+    while (band + 1 < p.nbands && (int)blockIdx.x >= p.cta_begin[band + 1]) ++band;
+    const int64_t c = (int64_t)blockIdx.x - p.cta_begin[band];
+    const int64_t C = p.cta_begin[band + 1] - p.cta_begin[band];
     it.rb = p.begin[band];
     it.nr = p.end[band] - it.rb;
     const int64_t T = p.nstrips * it.nr;
-    it.pos = (int64_t)blockIdx.x * T / gridDim.x;
-    it.hi = (int64_t)(blockIdx.x + 1) * T / gridDim.x;
+    it.pos = C > 0 ? c * T / C : 0;
+    it.hi = C > 0 ? (c + 1) * T / C : 0;
     return it;
+}
+
+// ---- fused exchange helpers -------------------------------------------------
+
+__device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* p) {
+    unsigned int v;
+    asm volatile("ld.acquire.sys.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// Producer side: before the TMA load of a halo row, wait for its delivery.
+// Bounded spin: a protocol failure traps (kernel error) instead of hanging.
+__device__ __forceinline__ void wait_delivery(const unsigned int* counter, unsigned int target) {
+    unsigned int spins = 0;
+    while (ld_acquire_sys(counter) < target) {
+        __nanosleep(64);
+        if (++spins > (1u << 26)) __trap();  // ~seconds: the neighbour never delivered
+    }
+    asm volatile("fence.proxy.async.global;" ::: "memory");  // make the peer's stores visible to TMA reads
+}
+
+// Consumer side, after this CTA's consumer warps stored `rows_sent` boundary
+// rows into a neighbour's halo: one thread publishes them (system-scope
+// release; the named barrier orders the other warps' stores before it).
+__device__ __forceinline__ void publish_delivery(unsigned int* counter, unsigned int rows_sent, int consumers) {
+    asm volatile("bar.sync 1, %0;" ::"r"(consumers * 32) : "memory");
+    if (threadIdx.x == 0) {
+        __threadfence_system();
+        asm volatile("red.release.sys.global.add.u32 [%0], %1;" ::"l"(counter), "r"(rows_sent) : "memory");
+    }
+}
+
+// At exit the last CTA of the launch advances gen.  The producer warp only
+// arrives (named barrier 2) and leaves, so the consumer code stays free of
+// CTA-wide divergence; the consumers wait on barrier 2, then thread 0 counts.
+__device__ __forceinline__ void finish_launch_producer(int threads) {
+    __syncwarp();
+    asm volatile("bar.arrive 2, %0;" ::"r"(threads) : "memory");
+}
+
+__device__ __forceinline__ void finish_launch_consumers(Mailbox* mb, int threads) {
+    asm volatile("bar.sync 2, %0;" ::"r"(threads) : "memory");
+    if (threadIdx.x == 0) {
+        __threadfence();
+        if (atomicAdd(&mb->done, 1u) == gridDim.x - 1) {
+            mb->done = 0;
+            __threadfence();
+            atomicAdd(&mb->gen, 1ull);
+        }
+    }
 }
 
 template <int NC, int EPL = 4>
@@ -174,11 +258,19 @@ struct RingPos {
     }
 };
 
-template <int NS>
-__device__ __forceinline__ void produce_align(uint64_t* full, uint64_t* empty, RingPos& r) {
+// The producer is the first PL lanes of the producer warp; lane l issues the
+// rows whose ring position is l mod PL (each lane tracks the whole ring
+// position, so stage and phase are always known).  Measured
+// (profiles/r01_producer_lanes.txt): PL = 2 speeds up the 5x5 conv (8
+// strips per row, 3 bulk copies per row at the row ends) by 6%, while Life
+// (one whole-row copy per row) is fastest with PL = 1.
+template <int NS, int PL>
+__device__ __forceinline__ void produce_align(uint64_t* full, uint64_t* empty, RingPos& r, int plane) {
     while (r.stage != 0) {
-        if (r.count >= NS) mbar_wait(&empty[r.stage], r.phase ^ 1u);
-        mbar_arrive(&full[r.stage]);
+        if ((int)(r.count % PL) == plane) {
+            if (r.count >= NS) mbar_wait(&empty[r.stage], r.phase ^ 1u);
+            mbar_arrive(&full[r.stage]);
+        }
         r.advance(NS);
     }
 }
@@ -197,50 +289,94 @@ __device__ __forceinline__ void consume_align(uint64_t* full, uint64_t* empty, R
 // segment's strip into the ring, continuing the CTA-wide row counter i.  Row
 // i goes to stage i % NS; before reusing a stage it waits until all consumer
 // warps released the row that occupied it.
-template <int NC, int NS, bool WRAP_COLS, int EPL = 4>
+template <int NC, int NS, bool WRAP_COLS, int EPL, int PL>
 __device__ __forceinline__ void produce(const RowStream& p, const Seg& t, uint8_t* smem, uint64_t* full,
-                                        uint64_t* empty, int64_t y_first, int64_t n_in, RingPos& r) {
+                                        uint64_t* empty, int64_t y_first, int64_t n_in, RingPos& r,
+                                        unsigned int halo_target, int plane) {
     using G = Geom<NC, EPL>;
+    // A strip that is the whole row needs no margin copies: under WRAP the
+    // consumers read the row's other end from the stage itself.
+    const bool whole = t.first_strip && t.last_strip;
+    const bool wrap_l = WRAP_COLS && t.first_strip && !whole;
+    const bool wrap_r = WRAP_COLS && t.last_strip && !whole;
     const uint32_t main_bytes = (uint32_t)(t.seg * 4) + (t.first_strip ? 0u : 16u) + (t.last_strip ? 0u : 16u);
-    uint32_t tx = main_bytes;
-    if (WRAP_COLS) tx += (t.first_strip ? 16u : 0u) + (t.last_strip ? 16u : 0u);
-    const uint32_t* src_main = p.in + t.e0 - (t.first_strip ? 0 : 4);
+    const uint32_t tx = main_bytes + (wrap_l ? 16u : 0u) + (wrap_r ? 16u : 0u);
+    const int64_t src_off = t.e0 - (t.first_strip ? 0 : 4);  // element offset of the main copy in a row
     const uint32_t dst_main = t.first_strip ? 16u : 0u;
-    for (int64_t j = 0; j < n_in; ++j) {
+    const uint32_t dst_r = 16u + (uint32_t)(t.seg * 4);
+    // this lane's first row, then every kProducerLanes-th row
+    int64_t j = (plane - r.count % PL + PL) % PL;
+    for (int64_t k = 0; k < j && k < n_in; ++k) r.advance(NS);
+    const uint32_t* rowp = p.in + (y_first + j) * p.pitch;  // in-slab rows: pointer walk
+    const int64_t rstep = (int64_t)PL * p.pitch;
+    for (; j < n_in; j += PL, rowp += rstep) {
         // phase of the release we wait for = the previous round's (r.phase ^ 1)
         if (r.count >= NS) mbar_wait(&empty[r.stage], r.phase ^ 1u);
         const int64_t row = y_first + j;
-        const int64_t rr = (row >= 0 && row < p.rows) ? row : map_row(p, row);
-        const int64_t roff = rr * p.pitch;
+        const uint32_t* rp = rowp;
+        if (row < 0 || row >= p.rows) {  // halo / wrapped / clamped rows: slab edges only
+            if (row < 0 && p.link.wait_top) wait_delivery(&p.link.mine->recv_top, halo_target);
+            if (row >= p.rows && p.link.wait_bot) wait_delivery(&p.link.mine->recv_bot, halo_target);
+            rp = p.in + map_row(p, row) * p.pitch;
+        }
         uint8_t* st = smem + r.stage * G::kStageBytes;
         uint64_t* bar = &full[r.stage];
         mbar_arrive_expect_tx(bar, tx);
-        bulk_g2s(st + dst_main, src_main + roff, main_bytes, bar);
-        if (WRAP_COLS) {
-            if (t.first_strip) bulk_g2s(st, p.in + roff + p.n - 4, 16, bar);            // elements n-4..n-1
-            if (t.last_strip) bulk_g2s(st + 16 + t.seg * 4, p.in + roff, 16, bar);     // elements 0..3
-        }
-        r.advance(NS);
+        bulk_g2s(st + dst_main, rp + src_off, main_bytes, bar);
+        if (wrap_l) bulk_g2s(st, rp + p.n - 4, 16, bar);   // elements n-4..n-1
+        if (wrap_r) bulk_g2s(st + dst_r, rp, 16, bar);     // elements 0..3
+        // advance the ring position past this row and the other lanes' rows
+        for (int q = 0; q < PL && j + q < n_in; ++q) r.advance(NS);
     }
 }
 
 }  // namespace tma
 
+// Host side: copy a FusedLink (or none) into the kernel parameters.
+inline void tma_set_link(tma::RowStream& p, const FusedLink* l, int r) {
+    p.link.mine = l ? static_cast<tma::Mailbox*>(l->mailbox) : nullptr;
+    p.link.dst_up = l ? static_cast<uint32_t*>(l->dst_up) : nullptr;
+    p.link.dst_down = l ? static_cast<uint32_t*>(l->dst_down) : nullptr;
+    p.link.sig_up = l ? l->sig_up : nullptr;
+    p.link.sig_down = l ? l->sig_down : nullptr;
+    p.link.wait_top = l ? l->wait_top : 0;
+    p.link.wait_bot = l ? l->wait_bot : 0;
+    p.link.r = r;
+}
+
 // Host side: fill the band table of a RowStream for a launch of
-// `ctas_per_sm` CTAs per SM; returns the grid x size (0 = nothing to do).
-inline int64_t tma_plan_grid(tma::RowStream& p, const RowBands& b, int num_sms, int ctas_per_sm, int strip_elems) {
+// `ctas_per_sm` CTAs per SM; returns the 1-D grid size (0 = nothing to do).
+// Plain launches split the resident CTAs evenly over the bands; fused
+// launches (bands = top boundary, bottom boundary, interior) give each
+// boundary band one CTA per strip so the exchanged rows are produced first.
+inline int64_t tma_plan_grid(tma::RowStream& p, const RowBands& b, int num_sms, int ctas_per_sm, int strip_elems,
+                             bool boundary_first = false) {
     p.nstrips = (p.n + strip_elems - 1) / strip_elems;
-    int64_t maxT = 0;
-    for (int i = 0; i < 2; ++i) p.begin[i] = p.end[i] = 0;
+    p.nbands = b.nbands;
+    for (int i = 0; i < tma::kMaxBands; ++i) p.begin[i] = p.end[i] = 0;
+    const int64_t resident = (int64_t)num_sms * ctas_per_sm;
+    int64_t total = 0;
+    p.cta_begin[0] = 0;
     for (int i = 0; i < b.nbands; ++i) {
         p.begin[i] = b.begin[i];
         p.end[i] = b.end[i];
         const int64_t T = p.nstrips * (b.end[i] - b.begin[i]);
-        if (T > maxT) maxT = T;
+        int64_t c;
+        if (boundary_first && i + 1 < b.nbands) {
+            c = p.nstrips;
+        } else if (boundary_first) {
+            c = resident - total;
+        } else {
+            c = resident / (b.nbands > 0 ? b.nbands : 1);
+        }
+        if (c > T) c = T;
+        if (c < 1 && T > 0) c = 1;
+        if (T <= 0) c = 0;
+        total += c;
+        p.cta_begin[i + 1] = (int)total;
     }
-    int64_t ctas = (int64_t)num_sms * ctas_per_sm / (b.nbands > 0 ? b.nbands : 1);
-    if (ctas > maxT) ctas = maxT;
-    return ctas;
+    for (int i = b.nbands; i < tma::kMaxBands; ++i) p.cta_begin[i + 1] = (int)total;
+    return total;
 }
 
 }  // namespace mapsm

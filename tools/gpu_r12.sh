@@ -1,0 +1,9 @@
+cd $GRAFT_REPO_ROOT
+for wl in life64k conv5 conv9; do bash tools/gpu_tune.sh $wl pre_p2p pl1 pl2 pl4; done 2>&1 | python -c "
+import sys,json
+for l in sys.stdin:
+    n,_,j=l.partition(' ')
+    try: d=json.loads(j); print(n, d['workload'], round(d['ms_per_launch']*1000,1),'us', round(d['GBps']),'GB/s')
+    except Exception: print(l.strip()[:300])
+"
+
