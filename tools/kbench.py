@@ -15,15 +15,24 @@ import torch
 import mapsm_inputs as mi
 from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
 
-wl = sys.argv[1] if len(sys.argv) > 1 else "life64k"
-iters = int(sys.argv[2]) if len(sys.argv) > 2 else 20
+import argparse
+
+ap = argparse.ArgumentParser()
+ap.add_argument("wl", nargs="?", default="life64k")
+ap.add_argument("iters", nargs="?", type=int, default=20)
+ap.add_argument("--local", type=int, default=0, help="g slabs in one process on cuda:0")
+ap.add_argument("--exchange", default="copy", choices=["copy", "p2p"])
+args = ap.parse_args()
+wl, iters = args.wl, args.iters
 cfg = {"life64k": ("life", 65536, 65536, 1, "wrap", 0.25), "life8k": ("life", 8192, 8192, 1, "wrap", 0.25),
        "conv5": ("conv", 16384, 16384, 2, "clamp", 8.0), "conv9": ("conv", 32768, 4096, 4, "zero", 8.0)}[wl]
 op, w, h, r, b, bc = cfg
 torch.cuda.set_device(0)
-ctx = M.mapsm_ctx_create(0, 1, 0, None, None)
+ctx = M.mapsm_ctx_create_local([0] * args.local) if args.local else M.mapsm_ctx_create(0, 1, 0, None, None)
 W = mi.weights_f32(1, r) if op == "conv" else None
 g = M.Grid(ctx, w, h, op, r, b, W)
+if args.exchange == "p2p":
+    g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
 if op == "life":
     x = torch.randint(0, 2, (h, w), dtype=torch.uint8, device="cuda")
 else:
@@ -31,26 +40,28 @@ else:
 g.bind(x)
 g.iterate(4)
 g.sync()
-per_l = []
-for rep in range(5):
-    g.set_option(M.OPT_TIMING, 1)
-    g.iterate(iters)
-    ms, n, bms, bn = M.mapsm_get_timing(g.handle)
-    per_l.append(ms / n)
-per = sorted(per_l)[len(per_l) // 2]
-gbs = bc * w * h / (per / 1e3) / 1e9
-g.set_option(M.OPT_TIMING, 0)
+if args.local:
+    per, gbs = float("nan"), float("nan")  # per-kernel events only for one slab
+else:
+    per_l = []
+    for rep in range(5):
+        g.set_option(M.OPT_TIMING, 1)
+        g.iterate(iters)
+        ms, n, bms, bn = M.mapsm_get_timing(g.handle)
+        per_l.append(ms / n)
+    per = sorted(per_l)[len(per_l) // 2]
+    gbs = bc * w * h / (per / 1e3) / 1e9
+    g.set_option(M.OPT_TIMING, 0)
 # graphs region
 g.iterate(16)
 g.sync()
-e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-s = torch.cuda.ExternalStream(M.mapsm_grid_stream(g.handle))
-e0.record(s)
+torch.cuda.synchronize()
+t0 = time.perf_counter()
 g.iterate(iters * 2)
-e1.record(s)
-e1.synchronize()
-reg = e0.elapsed_time(e1) / (iters * 2)
-print(json.dumps({"lib": os.environ.get("MAPSM_LIB", "default"), "workload": wl, "ms_per_launch": per,
+g.sync()
+reg = (time.perf_counter() - t0) * 1e3 / (iters * 2)  # wall: all slabs' streams
+print(json.dumps({"lib": os.environ.get("MAPSM_LIB", "default"), "workload": wl, "local": args.local,
+                  "exchange": args.exchange, "ms_per_launch": per,
                   "GBps": gbs, "region_ms_per_iter": reg, "region_GBps": bc * w * h / (reg / 1e3) / 1e9,
                   "cells_per_s": w * h / (reg / 1e3)}))
 g.close()
