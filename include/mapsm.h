@@ -208,6 +208,8 @@ typedef struct {
     int64_t exchanges;       /* halo messages received by this process since bind */
     int64_t device_bytes;    /* device memory owned by the grid */
     int used_graphs;         /* 1 if iterate replays CUDA graphs */
+    int gens_per_pass;       /* generations per compute pass (K with MAPSM_OPT_DEEP_HALO, else 1) */
+    int64_t halo_rows;       /* halo rows allocated above/below each slab (r, or K*r) */
 } mapsm_grid_info;
 
 mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
@@ -234,7 +236,23 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         through a device mailbox; the neighbour's CTAs that
  *                         need those rows wait on it.  Needs rows per slab >
  *                         2r and the TMA kernels (Life w % 128 == 0, conv
- *                         w % 4 == 0); set before bind.                       */
+ *                         w % 4 == 0); set before bind.
+ *   MAPSM_OPT_DEEP_HALO   K in {2,3,4,6,8} (1 = off, default): Life grids keep
+ *                         K*r halo rows per side and run K generations per
+ *                         pass of ONE temporally blocked kernel (each CTA
+ *                         carries its rows through K generations in
+ *                         registers), exchanging K*r rows once per pass
+ *                         instead of r rows every generation (SURVEY §8(f)
+ *                         NEXT-2; the per-iteration exchange of P:L461 made
+ *                         K-fold coarser).  HBM traffic per generation drops
+ *                         K-fold; results are bit-identical.  Set before bind
+ *                         (re-partitions and re-allocates: every slab needs
+ *                         >= K*r rows when g > 1, else EINVAL).  n % K
+ *                         trailing generations of an iterate call, slabs of
+ *                         fewer than K rows, and w % 128 != 0 use the
+ *                         per-generation kernels.  EUNSUPPORTED for non-Life
+ *                         grids or other K; not combined with EXCHANGE_P2P
+ *                         (the fused path then runs per generation).         */
 typedef enum { MAPSM_EXCHANGE_COPY = 0, MAPSM_EXCHANGE_P2P = 1 } mapsm_exchange;
 typedef enum {
     MAPSM_OPT_GRAPHS = 1,
@@ -242,7 +260,8 @@ typedef enum {
     MAPSM_OPT_NO_EXCHANGE = 3,
     MAPSM_OPT_TIMING = 4,
     MAPSM_OPT_PERSISTENT = 5,
-    MAPSM_OPT_EXCHANGE = 6
+    MAPSM_OPT_EXCHANGE = 6,
+    MAPSM_OPT_DEEP_HALO = 7
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

@@ -150,6 +150,8 @@ struct Slab {
     cudaEvent_t ev_b = nullptr, ev_h = nullptr;
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int64_t graph_iters = 0;
+    cudaGraphExec_t graph_tb[2] = {nullptr, nullptr};  // deep-halo passes (K generations each)
+    int64_t graph_tb_passes = 0;
     unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
     unsigned int* gbar = nullptr;        // grid-barrier word of the persistent Life kernel
     // fused peer-memory exchange (MAPSM_OPT_EXCHANGE = P2P): my mailbox and
@@ -185,6 +187,9 @@ struct mapsm_grid_s {
     int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
     bool opt_graphs = true, opt_no_exchange = false, opt_timing = false, opt_persistent = true;
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
+    int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
+    int64_t halo = 0;           // halo rows allocated above/below each slab (r, or K*r with deep halos)
+    bool deep_valid = false;    // the current buffer's halos are valid to depth `halo` (else only r)
     bool p2p_linked = false;    // peer pointers resolved
     int64_t opt_graph_iters = 16;
     bool used_graphs = false;
@@ -194,7 +199,7 @@ struct mapsm_grid_s {
 static const size_t kMailboxBytes = 64;  // >= sizeof(tma::Mailbox)
 
 static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
-    return s.base[b] + (y + g->r) * g->pitch;
+    return s.base[b] + (y + g->halo) * g->pitch;
 }
 
 static bool has_exchange(const Slab& s) {
@@ -326,8 +331,10 @@ static void free_slab(Slab& s) {
     if (s.gbar) cudaFree(s.gbar);
     if (s.mailbox) cudaFree(s.mailbox);
     for (void* q : s.ipc_opened) cudaIpcCloseMemHandle(q);
-    for (int b = 0; b < 2; ++b)
+    for (int b = 0; b < 2; ++b) {
         if (s.graph[b]) cudaGraphExecDestroy(s.graph[b]);
+        if (s.graph_tb[b]) cudaGraphExecDestroy(s.graph_tb[b]);
+    }
     for (auto& t : s.t_bulk) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
     for (auto& t : s.t_bnd) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
     if (s.ev_b) cudaEventDestroy(s.ev_b);
@@ -337,34 +344,39 @@ static void free_slab(Slab& s) {
     s = Slab();
 }
 
-extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundary boundary) {
-    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
-    if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "window_set after bind (allocation depends on r)");
-    if (boundary != MAPSM_WRAP && boundary != MAPSM_CLAMP && boundary != MAPSM_ZERO && boundary != MAPSM_NO_CHECKS)
-        return fail(MAPSM_EINVAL, "boundary %d", (int)boundary);
-    if ((radius == 0) != (boundary == MAPSM_NO_CHECKS))
-        return fail(MAPSM_EUNSUPPORTED, "NO_CHECKS goes with radius 0 (histogram input), got r=%d b=%d", radius,
-                    (int)boundary);
-    if (g->dtype == MAPSM_U8) {
-        if (radius != 1 && radius != 0)
-            return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
-        if (radius == 1 && g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
-    } else {
-        if (radius < 1 || radius > 4) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..4, got %d", radius);
-    }
+// Halo rows per side: r, or K*r for a Life grid with deep halos (K
+// generations per pass, MAPSM_OPT_DEEP_HALO).
+static int64_t halo_rows(const mapsm_grid_s* g, int radius) {
+    const bool life = g->dtype == MAPSM_U8 && radius == 1;
+    return (int64_t)radius * (life && g->tb_k > 1 ? g->tb_k : 1);
+}
+
+static void drop_graphs(mapsm_grid_s* g) {
+    for (auto& s : g->slabs)
+        for (int b = 0; b < 2; ++b) {
+            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+            if (s.graph_tb[b]) { cudaGraphExecDestroy(s.graph_tb[b]); s.graph_tb[b] = nullptr; }
+        }
+}
+
+// Partition (plan.cpp) and allocate both buffers of every local slab with
+// g->halo rows above and below (the Memory Analyzer's bounding box).
+static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boundary) {
     mapsm_ctx c = g->ctx;
+    const int64_t halo = halo_rows(g, radius);
     // validate the partition for every slab before allocating anything
     for (int k = 0; k < c->g; ++k) {
         mapsm_slab_plan p;
-        if (compute_plan(g->h, c->g, radius, boundary, k, &p) != MAPSM_OK)
-            return fail(MAPSM_EINVAL, "cannot split %lld rows over %d slabs with radius %d (need >= r rows each)",
-                        (long long)g->h, c->g, radius);
+        if (compute_plan(g->h, c->g, (int)halo, boundary, k, &p) != MAPSM_OK)
+            return fail(MAPSM_EINVAL, "cannot split %lld rows over %d slabs with %lld halo rows (need >= that many rows each)",
+                        (long long)g->h, c->g, (long long)halo);
     }
     DeviceGuard dg;
     for (auto& s : g->slabs) free_slab(s);
     g->slabs.clear();
     g->device_bytes = 0;
     g->r = radius;
+    g->halo = halo;
     g->boundary = boundary;
     const int64_t row_bytes = g->packed() ? g->w / 8 : g->w * g->elem;
     const int64_t align = row_bytes >= 128 ? 128 : 16;
@@ -375,7 +387,9 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         Slab& s = g->slabs[i];
         s.rank = c->local ? i : c->first_slab;
         s.device = c->devices[c->local ? i : 0];
-        compute_plan(g->h, c->g, radius, boundary, s.rank, &s.plan);
+        // the plan's kinds / neighbours / rows do not depend on the halo
+        // depth; alloc_rows does (rows + 2 * halo)
+        compute_plan(g->h, c->g, (int)halo, boundary, s.rank, &s.plan);
         CK(cudaSetDevice(s.device));
         CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
         const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
@@ -416,6 +430,26 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         if (same > 1) s.num_sms = s.num_sms / same > 0 ? s.num_sms / same : 1;
     }
     CK(cudaDeviceSynchronize());
+    g->p2p_linked = false;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundary boundary) {
+    if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "window_set after bind (allocation depends on r)");
+    if (boundary != MAPSM_WRAP && boundary != MAPSM_CLAMP && boundary != MAPSM_ZERO && boundary != MAPSM_NO_CHECKS)
+        return fail(MAPSM_EINVAL, "boundary %d", (int)boundary);
+    if ((radius == 0) != (boundary == MAPSM_NO_CHECKS))
+        return fail(MAPSM_EUNSUPPORTED, "NO_CHECKS goes with radius 0 (histogram input), got r=%d b=%d", radius,
+                    (int)boundary);
+    if (g->dtype == MAPSM_U8) {
+        if (radius != 1 && radius != 0)
+            return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
+        if (radius == 1 && g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
+    } else {
+        if (radius < 1 || radius > 4) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..4, got %d", radius);
+    }
+    TRY(alloc_slabs(g, radius, boundary));
     g->state = ST_WINDOW;
     if (g->dtype == MAPSM_U8) {  // one operator per u8 radius: op_set is optional
         g->op = radius == 1 ? MAPSM_OP_LIFE : MAPSM_OP_HISTOGRAM;
@@ -443,9 +477,7 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
         return fail(MAPSM_EUNSUPPORTED, "op %d", (int)op);
     }
     g->op = op;
-    for (auto& s : g->slabs)
-        for (int b = 0; b < 2; ++b)
-            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+    drop_graphs(g);
     if (g->state < ST_OP) g->state = ST_OP;
     return MAPSM_OK;
 }
@@ -463,14 +495,14 @@ extern "C" mapsm_status mapsm_grid_slab(mapsm_grid g, int i, int64_t* y0, int64_
 
 // Local mode: slab i pulls its halos of buffer b from its neighbours with
 // device/peer copies on its side stream, after the neighbours' ev_b.
-static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events) {
-    const int64_t bytes = (int64_t)g->r * g->pitch;
+static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events, int64_t depth) {
+    const int64_t bytes = depth * g->pitch;
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
         if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
             Slab& u = g->slabs[s.plan.up];
             if (wait_events) CK(cudaStreamWaitEvent(s.side, u.ev_b, 0));
-            CK(cudaMemcpyAsync(row_ptr(g, s, b, -g->r), row_ptr(g, u, b, u.plan.rows - g->r), bytes,
+            CK(cudaMemcpyAsync(row_ptr(g, s, b, -depth), row_ptr(g, u, b, u.plan.rows - depth), bytes,
                                cudaMemcpyDefault, s.side));
             g->exchanges++;
         }
@@ -490,18 +522,18 @@ static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events) {
 // order send-up, send-down, recv-bottom (from down), recv-top (from up): with
 // g == 2 under WRAP both neighbours are the same peer, and this order makes
 // the peer's first recv (its bottom halo) match my first send (my top rows).
-static mapsm_status exchange_nccl(mapsm_grid_s* g, int b) {
+static mapsm_status exchange_nccl(mapsm_grid_s* g, int b, int64_t depth) {
     Slab& s = g->slabs[0];
-    const size_t bytes = (size_t)g->r * (size_t)g->pitch;
+    const size_t bytes = (size_t)depth * (size_t)g->pitch;
     NK(g_nccl.groupStart());
     if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
         NK(g_nccl.send(row_ptr(g, s, b, 0), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
     if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.send(row_ptr(g, s, b, s.plan.rows - g->r), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
+        NK(g_nccl.send(row_ptr(g, s, b, s.plan.rows - depth), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
     if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
         NK(g_nccl.recv(row_ptr(g, s, b, s.plan.rows), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
     if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.recv(row_ptr(g, s, b, -g->r), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
+        NK(g_nccl.recv(row_ptr(g, s, b, -depth), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
     NK(g_nccl.groupEnd());
     g->exchanges += s.plan.n_recv;
     return MAPSM_OK;
@@ -510,7 +542,7 @@ static mapsm_status exchange_nccl(mapsm_grid_s* g, int b) {
 // ------------------------------------------------------------- compute step
 
 static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk,
-                                const FusedLink* link = nullptr) {
+                                const FusedLink* link = nullptr, int K = 1) {
     StencilGeom geom;
     geom.in = row_ptr(g, s, b_in, 0);
     geom.out = row_ptr(g, s, b_in ^ 1, 0);
@@ -534,7 +566,10 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
         CK(cudaEventRecord(tp->a, s.main));
     }
     cudaError_t e;
-    if (g->op == MAPSM_OP_LIFE)
+    if (g->op == MAPSM_OP_LIFE && K > 1)
+        e = launch_life_tb(geom, bands, K, s.plan.top_kind == MAPSM_HALO_ZERO, s.plan.bottom_kind == MAPSM_HALO_ZERO,
+                           s.num_sms, s.main);
+    else if (g->op == MAPSM_OP_LIFE)
         e = launch_life_step(geom, bands, s.num_sms, s.main, link);
     else
         e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main, link);
@@ -545,8 +580,8 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
 }
 
 // Output-row bands: rows sent to neighbours (boundary) and the rest (interior).
-static void split_bands(const mapsm_grid_s* g, const Slab& s, RowBands& bnd, RowBands& inner) {
-    const int64_t rows = s.plan.rows, r = g->r;
+static void split_bands(const Slab& s, int64_t r, RowBands& bnd, RowBands& inner) {
+    const int64_t rows = s.plan.rows;
     const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
     bnd.nbands = inner.nbands = 0;
     if (rows <= 2 * r) {  // tiny slab: everything is boundary
@@ -561,8 +596,12 @@ static void split_bands(const mapsm_grid_s* g, const Slab& s, RowBands& bnd, Row
 }
 
 // One iteration for all local slabs, reading buffer b_in.
-static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
+// One pass for all local slabs, reading buffer b_in: one generation (K == 1,
+// halos of depth r), or K generations of the deep-halo kernel (halos of
+// depth K*r, exchanged once per pass).
+static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1) {
     mapsm_ctx c = g->ctx;
+    const int64_t depth = (int64_t)g->r * K;
     const bool exch = !g->opt_no_exchange;
     bool any_exchange = false;
     for (auto& s : g->slabs) any_exchange |= has_exchange(s);
@@ -573,7 +612,7 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
             all.nbands = 1;
             all.begin[0] = 0;
             all.end[0] = s.plan.rows;
-            TRY(launch_step(g, s, b_in, all, true));
+            TRY(launch_step(g, s, b_in, all, true, nullptr, K));
         }
         return MAPSM_OK;
     }
@@ -583,18 +622,18 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
         Slab& s = g->slabs[i];
         CK(cudaSetDevice(s.device));
         RowBands bnd;
-        split_bands(g, s, bnd, inner[i]);
-        TRY(launch_step(g, s, b_in, bnd, false));
+        split_bands(s, depth, bnd, inner[i]);
+        TRY(launch_step(g, s, b_in, bnd, false, nullptr, K));
         CK(cudaEventRecord(s.ev_b, s.main));
     }
     // 2. halo exchange of the freshly computed rows on the side streams
     if (exch) {
         if (c->local) {
-            TRY(exchange_local(g, b_in ^ 1, true));
+            TRY(exchange_local(g, b_in ^ 1, true, depth));
         } else {
             Slab& s = g->slabs[0];
             CK(cudaStreamWaitEvent(s.side, s.ev_b, 0));
-            TRY(exchange_nccl(g, b_in ^ 1));
+            TRY(exchange_nccl(g, b_in ^ 1, depth));
             CK(cudaEventRecord(s.ev_h, s.side));
         }
     }
@@ -602,7 +641,8 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in) {
     for (size_t i = 0; i < g->slabs.size(); ++i) {
         Slab& s = g->slabs[i];
         CK(cudaSetDevice(s.device));
-        if (inner[i].nbands > 0 && inner[i].end[0] > inner[i].begin[0]) TRY(launch_step(g, s, b_in, inner[i], true));
+        if (inner[i].nbands > 0 && inner[i].end[0] > inner[i].begin[0])
+            TRY(launch_step(g, s, b_in, inner[i], true, nullptr, K));
         if (exch) CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
     }
     return MAPSM_OK;
@@ -718,8 +758,8 @@ static mapsm_status iterate_fused(mapsm_grid_s* g, int b_in) {
         bands.nbands++;
         FusedLink L;
         L.mailbox = s.mailbox;
-        L.dst_up = top ? s.up_base[bo] + (s.up_rows + r) * g->pitch : nullptr;  // up's row up_rows (bottom halo)
-        L.dst_down = bot ? s.down_base[bo] : nullptr;                           // down's row -r (top halo)
+        L.dst_up = top ? s.up_base[bo] + (s.up_rows + g->halo) * g->pitch : nullptr;  // up's row up_rows (bottom halo)
+        L.dst_down = bot ? s.down_base[bo] + (g->halo - r) * g->pitch : nullptr;      // down's row -r (top halo)
         L.sig_up = top ? reinterpret_cast<unsigned int*>(s.up_mail + 16) : nullptr;      // recv_bot
         L.sig_down = bot ? reinterpret_cast<unsigned int*>(s.down_mail + 12) : nullptr;  // recv_top
         L.wait_top = top;
@@ -734,14 +774,49 @@ static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
     return fused_now(g) ? iterate_fused(g, b_in) : iterate_once(g, b_in);
 }
 
-static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters) {
+// Deep-halo passes apply: Life, TMA-kernel rows (w % 128 == 0), every slab at
+// least K rows (mirror rows at CLAMP edges), copy/NCCL exchange.
+static bool tb_active(const mapsm_grid_s* g) {
+    if (g->op != MAPSM_OP_LIFE || g->tb_k <= 1 || g->opt_p2p) return false;
+    if ((g->w / 32) % 4 != 0 || g->pitch % 16 != 0) return false;
+    for (auto& s : g->slabs)
+        if (s.plan.rows < g->tb_k) return false;
+    return true;
+}
+
+// Re-fill the current buffer's halos to depth g->halo (after per-generation
+// steps, which only exchange r rows), ordered after the work already enqueued.
+static mapsm_status refresh_deep_halos(mapsm_grid_s* g) {
+    bool any = false;
+    for (auto& s : g->slabs) any |= has_exchange(s);
+    if (!any || g->opt_no_exchange) return MAPSM_OK;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaEventRecord(s.ev_b, s.main));
+    }
+    if (g->ctx->local) {
+        TRY(exchange_local(g, g->cur, true, g->halo));
+    } else {
+        Slab& s = g->slabs[0];
+        CK(cudaStreamWaitEvent(s.side, s.ev_b, 0));
+        TRY(exchange_nccl(g, g->cur, g->halo));
+        CK(cudaEventRecord(s.ev_h, s.side));
+    }
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
+    }
+    return MAPSM_OK;
+}
+
+static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters, int K = 1) {
     CK(cudaSetDevice(s.device));
     const int64_t l0 = g->launches, x0 = g->exchanges;
     CK(cudaStreamBeginCapture(s.main, cudaStreamCaptureModeThreadLocal));
     mapsm_status st = MAPSM_OK;
     int cur = start_cur;
     for (int64_t k = 0; k < iters && st == MAPSM_OK; ++k) {
-        st = step_all(g, cur);
+        st = K > 1 ? iterate_once(g, cur, K) : step_all(g, cur);
         cur ^= 1;
     }
     cudaGraph_t graph = nullptr;
@@ -753,10 +828,13 @@ static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64
         return st;
     }
     if (e != cudaSuccess) return fail(MAPSM_ECUDA, "graph capture: %s", cudaGetErrorString(e));
-    e = cudaGraphInstantiate(&s.graph[start_cur], graph, 0);
+    e = cudaGraphInstantiate(K > 1 ? &s.graph_tb[start_cur] : &s.graph[start_cur], graph, 0);
     cudaGraphDestroy(graph);
     if (e != cudaSuccess) return fail(MAPSM_ECUDA, "graph instantiate: %s", cudaGetErrorString(e));
-    s.graph_iters = iters;
+    if (K > 1)
+        s.graph_tb_passes = iters;
+    else
+        s.graph_iters = iters;
     return MAPSM_OK;
 }
 
@@ -767,9 +845,53 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     if (n == 0) return MAPSM_OK;
     if (g->op == MAPSM_OP_HISTOGRAM) return fail(MAPSM_EUNSUPPORTED, "a Reductive (histogram) grid is not iterated");
     DeviceGuard dg;
+    const bool graphs = g->opt_graphs && !g->opt_timing && !g->ctx->local;
+    // Deep halos: K generations per pass (one halo exchange of K*r rows per
+    // pass), then any remainder with the per-generation path below.
+    if (tb_active(g) && n >= g->tb_k) {
+        const int K = g->tb_k;
+        int64_t passes = n / K;
+        if (!g->deep_valid) TRY(refresh_deep_halos(g));
+        Slab& s0 = g->slabs[0];
+        int64_t per_pass_launches = 1, per_pass_exch = 0;
+        {
+            RowBands bnd, inner;
+            split_bands(s0, g->halo, bnd, inner);
+            if (has_exchange(s0)) per_pass_launches = 1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0);
+            per_pass_exch = (has_exchange(s0) && !g->opt_no_exchange) ? s0.plan.n_recv : 0;
+        }
+        if (graphs) {
+            int64_t gp = g->opt_graph_iters / K;  // passes per graph (even)
+            if (gp < 2) gp = 2;
+            if (gp % 2) gp++;
+            if (s0.graph_tb_passes != gp)
+                for (int b = 0; b < 2; ++b)
+                    if (s0.graph_tb[b]) { cudaGraphExecDestroy(s0.graph_tb[b]); s0.graph_tb[b] = nullptr; }
+            while (passes >= gp) {
+                if (!s0.graph_tb[g->cur]) TRY(capture_graph(g, s0, g->cur, gp, K));
+                CK(cudaSetDevice(s0.device));
+                CK(cudaGraphLaunch(s0.graph_tb[g->cur], s0.main));
+                passes -= gp;
+                n -= gp * K;
+                g->launches += per_pass_launches * gp;
+                g->exchanges += per_pass_exch * gp;
+                g->gen += gp * K;
+                g->used_graphs = true;
+            }
+        }
+        for (; passes > 0; --passes) {
+            TRY(iterate_once(g, g->cur, K));
+            g->cur ^= 1;
+            g->gen += K;
+            n -= K;
+        }
+        g->deep_valid = true;
+        if (n == 0) return MAPSM_OK;
+    }
+    if (n > 0) g->deep_valid = false;  // per-generation steps exchange only r rows
     // L2-resident Life slabs with no exchanged halos: persistent kernel, up to
     // kPersistChunk generations per cooperative launch.
-    if (g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 &&
+    if (g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 && g->tb_k <= 1 &&
         !has_exchange(g->slabs[0]) && 2 * g->slabs[0].plan.alloc_rows * g->pitch <= (64ll << 20)) {
         Slab& s = g->slabs[0];
         CK(cudaSetDevice(s.device));
@@ -797,7 +919,6 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     }
     // CUDA graphs for the single-stream-per-process modes (g == 1 and NCCL);
     // local multi-slab mode issues directly (it is the single-GPU test vehicle).
-    const bool graphs = g->opt_graphs && !g->opt_timing && !g->ctx->local;
     int64_t done = 0;
     if (graphs) {
         Slab& s = g->slabs[0];
@@ -812,7 +933,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
         {
             // launches per iteration (for the counters; graphs replay them)
             RowBands bnd, inner;
-            split_bands(g, s, bnd, inner);
+            split_bands(s, g->r, bnd, inner);
             per_graph_launches = (has_exchange(s) && !fused_now(g))
                                      ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0))
                                      : 1;
@@ -945,12 +1066,13 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     for (auto& s : g->slabs) any |= has_exchange(s);
     if (any) {
         if (g->ctx->local) {
-            TRY(exchange_local(g, 0, false));
+            TRY(exchange_local(g, 0, false, g->halo));
         } else {
-            TRY(exchange_nccl(g, 0));
+            TRY(exchange_nccl(g, 0, g->halo));
         }
         g->exchanges = 0;
     }
+    g->deep_valid = true;
     return check_async(g);
 }
 
@@ -1041,7 +1163,7 @@ extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int
         // Reuse read_slab's copy-out path on a view of the received rows.
         Slab view = s;
         view.plan = pk;
-        view.base[g->cur] = tmp - (int64_t)g->r * g->pitch;
+        view.base[g->cur] = tmp - g->halo * g->pitch;
         view.staging = s.staging;
         view.staging_bytes = s.staging_bytes;
         st = read_slab(g, view, dst, pitch, on_dev);
@@ -1133,6 +1255,8 @@ extern "C" mapsm_status mapsm_get_info(mapsm_grid g, mapsm_grid_info* o) {
     o->exchanges = g->exchanges;
     o->device_bytes = g->device_bytes;
     o->used_graphs = g->used_graphs ? 1 : 0;
+    o->halo_rows = g->halo;
+    o->gens_per_pass = tb_active(g) ? g->tb_k : 1;
     return MAPSM_OK;
 }
 
@@ -1156,11 +1280,30 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;
             break;
+        case MAPSM_OPT_DEEP_HALO: {
+            const int k = v <= 1 ? 1 : (int)v;
+            if (k > 1 && !life_tb_supported(k))
+                return fail(MAPSM_EUNSUPPORTED, "deep halo: K must be 1 (off) or one of 2, 3, 4, 6, 8 (got %lld)", (long long)v);
+            if (k == g->tb_k) break;
+            if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "set MAPSM_OPT_DEEP_HALO before bind (it sizes the halos)");
+            if (g->dtype != MAPSM_U8) return fail(MAPSM_EUNSUPPORTED, "deep halos are implemented for Life grids");
+            const int old = g->tb_k;
+            g->tb_k = k;
+            if (g->state >= ST_WINDOW && g->r == 1) {  // re-partition and re-allocate with the new halo depth
+                const int st = g->state;
+                mapsm_status e = alloc_slabs(g, g->r, g->boundary);
+                if (e != MAPSM_OK) {
+                    g->tb_k = old;
+                    if (alloc_slabs(g, g->r, g->boundary) == MAPSM_OK) g->state = st;
+                    return e;
+                }
+                g->state = st;
+            }
+            break;
+        }
         default: return fail(MAPSM_EINVAL, "unknown option %d", (int)opt);
     }
-    for (auto& s : g->slabs)
-        for (int b = 0; b < 2; ++b)
-            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+    drop_graphs(g);
     return MAPSM_OK;
 }
 

@@ -56,6 +56,14 @@ cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sm
 // of generation 0 / 1 (generation n ends in g.in if n is even, else g.out).
 // `bar` = one device word of barrier state.
 cudaError_t launch_life_persistent(const StencilGeom& g, int64_t n, unsigned int* bar, int num_sms, cudaStream_t s);
+// K generations of Life in ONE temporally blocked launch (life_tb.cu): reads
+// input rows [-K, rows+K) of g.in (halo rows must be valid to depth K; under
+// ROWMAP_CLAMP the rows outside are the MIRROR image), writes owned rows of
+// the bands of generation t+K to g.out.  zero_top / zero_bot: ZERO global
+// edges (rows outside the slab forced to 0 at every generation).
+bool life_tb_supported(int k);
+cudaError_t launch_life_tb(const StencilGeom& g, const RowBands& b, int k, int zero_top, int zero_bot, int num_sms,
+                           cudaStream_t s);
 cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, int64_t dst_pitch,
                              int64_t rows, int64_t w, cudaStream_t s);
 cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst, int64_t dst_pitch,

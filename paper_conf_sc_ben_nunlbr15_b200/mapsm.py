@@ -23,7 +23,7 @@ U8, F32 = 1, 2
 WRAP, CLAMP, ZERO, NO_CHECKS = 0, 1, 2, 3
 OP_LIFE, OP_CONV, OP_HISTOGRAM = 0, 1, 2
 HALO_EXCHANGE, HALO_WRAP_LOCAL, HALO_CLAMP, HALO_ZERO = 0, 1, 2, 3
-OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING, OPT_PERSISTENT, OPT_EXCHANGE = 1, 2, 3, 4, 5, 6
+OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING, OPT_PERSISTENT, OPT_EXCHANGE, OPT_DEEP_HALO = 1, 2, 3, 4, 5, 6, 7
 EXCHANGE_COPY, EXCHANGE_P2P = 0, 1
 
 BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO, "no_checks": NO_CHECKS}
@@ -55,7 +55,7 @@ class mapsm_grid_info(ctypes.Structure):
                 ("radius", ctypes.c_int), ("boundary", ctypes.c_int), ("world", ctypes.c_int),
                 ("local_slabs", ctypes.c_int), ("pitch_bytes", ctypes.c_int64), ("generation", ctypes.c_int64),
                 ("launches", ctypes.c_int64), ("exchanges", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
-                ("used_graphs", ctypes.c_int)]
+                ("used_graphs", ctypes.c_int), ("gens_per_pass", ctypes.c_int), ("halo_rows", ctypes.c_int64)]
 
 
 _lib = None
@@ -260,7 +260,7 @@ class Grid:
     bind -> iterate -> gather, as in Fig 2a."""
 
     def __init__(self, ctx: int, w: int, h: int, op: str = "life", radius: int = 1, boundary: str = "wrap",
-                 weights=None):
+                 weights=None, deep_halo: int = 1):
         self.ctx, self.w, self.h = ctx, w, h
         self.op = op
         self.dtype = F32 if op == "conv" else U8
@@ -269,6 +269,8 @@ class Grid:
         self.handle = mapsm_grid_create(ctx, w, h, self.dtype)
         try:
             mapsm_window_set(self.handle, radius, BOUNDARY[boundary] if isinstance(boundary, str) else boundary)
+            if deep_halo > 1:
+                mapsm_set_option(self.handle, OPT_DEEP_HALO, deep_halo)
             if op == "life":
                 mapsm_op_set(self.handle, OP_LIFE, None)
             elif op == "histogram":

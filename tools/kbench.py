@@ -22,6 +22,7 @@ ap.add_argument("wl", nargs="?", default="life64k")
 ap.add_argument("iters", nargs="?", type=int, default=20)
 ap.add_argument("--local", type=int, default=0, help="g slabs in one process on cuda:0")
 ap.add_argument("--exchange", default="copy", choices=["copy", "p2p"])
+ap.add_argument("--deep", type=int, default=1, help="MAPSM_OPT_DEEP_HALO (generations per pass)")
 args = ap.parse_args()
 wl, iters = args.wl, args.iters
 cfg = {"life64k": ("life", 65536, 65536, 1, "wrap", 0.25), "life8k": ("life", 8192, 8192, 1, "wrap", 0.25),
@@ -30,7 +31,7 @@ op, w, h, r, b, bc = cfg
 torch.cuda.set_device(0)
 ctx = M.mapsm_ctx_create_local([0] * args.local) if args.local else M.mapsm_ctx_create(0, 1, 0, None, None)
 W = mi.weights_f32(1, r) if op == "conv" else None
-g = M.Grid(ctx, w, h, op, r, b, W)
+g = M.Grid(ctx, w, h, op, r, b, W, deep_halo=args.deep)
 if args.exchange == "p2p":
     g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
 if op == "life":
@@ -48,7 +49,7 @@ else:
         g.set_option(M.OPT_TIMING, 1)
         g.iterate(iters)
         ms, n, bms, bn = M.mapsm_get_timing(g.handle)
-        per_l.append(ms / n)
+        per_l.append(ms / n / max(1, g.info().gens_per_pass))  # per generation
     per = sorted(per_l)[len(per_l) // 2]
     gbs = bc * w * h / (per / 1e3) / 1e9
     g.set_option(M.OPT_TIMING, 0)
@@ -61,7 +62,7 @@ g.iterate(iters * 2)
 g.sync()
 reg = (time.perf_counter() - t0) * 1e3 / (iters * 2)  # wall: all slabs' streams
 print(json.dumps({"lib": os.environ.get("MAPSM_LIB", "default"), "workload": wl, "local": args.local,
-                  "exchange": args.exchange, "ms_per_launch": per,
+                  "exchange": args.exchange, "deep": args.deep, "ms_per_launch": per,
                   "GBps": gbs, "region_ms_per_iter": reg, "region_GBps": bc * w * h / (reg / 1e3) / 1e9,
                   "cells_per_s": w * h / (reg / 1e3)}))
 g.close()
