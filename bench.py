@@ -21,6 +21,10 @@ configs[2] at N=1 (``life64k``); ``--workload`` selects the other configs
               cell-update, 8 B per conv cell-update, 1 B per histogram pixel.
 * cpu_baseline = the CPU oracle (oracle/, OpenMP) timed on a bounded sample of
               the same workload on rank 0 only.
+* deep_halo = (Life) the same workload on the deep-halo path (MAPSM_OPT_DEEP_HALO
+              = --deep-halo K, default 8: K generations per pass of the
+              temporally blocked kernel, K-row halos exchanged once per pass),
+              reported separately with its ALU-pipe roofline.
 ``--impl reference`` times only the oracle (this tier's reference arm).
 """
 from __future__ import annotations
@@ -221,6 +225,9 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--graph-iters", type=int, default=0)
+    ap.add_argument("--deep-halo", type=int, default=8,
+                    help="Life workloads: also measure the deep-halo path with K generations per pass "
+                         "(reported under 'deep_halo'; 0/1 = skip)")
     args = ap.parse_args()
     wl = dict(WORKLOADS[args.workload])
 
@@ -414,6 +421,61 @@ def main():
     d2h = 256 * 8 * world if op == "histogram" else h * w * elem
 
     grid.close()
+
+    # Deep halos (MAPSM_OPT_DEEP_HALO): the same workload
+    # with K generations per pass and K-row halos exchanged once per pass —
+    # reported separately because it is not the per-iteration exchange of the
+    # north_star design and is bound by the ALU pipe, not HBM.
+    deep = None
+    if op == "life" and args.deep_halo > 1:
+        K = args.deep_halo
+        dg = M.Grid(ctx, w, h, op, wl["r"], wl["b"], None, deep_halo=K)
+        dg.bind(h_in)
+        for _ in range(args.warmup):
+            dg.iterate(n)
+        barrier()
+        d_ms = 0.0
+        for _ in range(args.steps):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            dg.iterate(n)
+            e1.record(stream)
+            e1.synchronize()
+            d_ms += e0.elapsed_time(e1)
+        dinfo = dg.info()
+        # per-launch kernel time of the temporally blocked kernel (direct launches)
+        dg.set_option(M.OPT_TIMING, 1)
+        dg.iterate(n - n % K)
+        b_ms, b_n, bb_ms, bb_n = M.mapsm_get_timing(dg.handle)
+        dg.set_option(M.OPT_TIMING, 0)
+        dg.close()
+        td = torch.tensor([d_ms], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(td, op=dist.ReduceOp.MAX)
+        d_ms = float(td.item())
+        d_value = units_per_step * args.steps / (d_ms / 1e3)
+        # ALU roofline: 12 ALU-pipe ops (2 funnel shifts + 2 LOP3 for the
+        # 3-cell row sum, 8 LOP3 for the rule) per 32-cell word per generation;
+        # the ALU pipe retires 64 lanes/clk/SM (tools/pipebench.cu: LOP3 and
+        # SHF ~1.9 warp-instructions/clk/SM).
+        sm_mhz = clocks.get("sm_mhz") or 1965.0
+        alu_peak = 148 * 64 * sm_mhz * 1e6 / 1e12  # T lane-ops/s
+        kern_s = (b_ms / 1e3) / max(1, b_n)
+        bulk_rows = rows if bb_n == 0 else rows - 2 * K
+        cells_per_launch = bulk_rows * w * K
+        alu_achieved = cells_per_launch * 12 / 32 / kern_s / 1e12
+        deep = {"generations_per_pass": int(dinfo.gens_per_pass), "halo_rows": int(dinfo.halo_rows),
+                "value": d_value, "unit": metric_of(wl)[1], "ms_per_step": d_ms / args.steps,
+                "vs_per_generation_path": d_value / value,
+                "roofline": {"bound": "alu", "kernel": "life_tb_kernel", "achieved": alu_achieved,
+                             "peak": alu_peak, "unit": "T ALU lane-ops/s", "frac": alu_achieved / alu_peak,
+                             "ops_per_cell_update": 12 / 32, "kernel_ms_per_launch": kern_s * 1e3,
+                             "peak_source": "148 SMs x 64 ALU lanes/clk x sampled SM clock (B300_MICROARCH.md "
+                                            "alu rt=2/SMSP; tools/pipebench.cu)",
+                             "hbm_bytes_per_cell_update": 0.25 / K,
+                             "hbm_achieved_GBps": cells_per_launch * 0.25 / K / kern_s / 1e9}}
     M.mapsm_ctx_destroy(ctx)
 
     if rank == 0:
@@ -444,6 +506,8 @@ def main():
         }
         if exposure is not None:
             line["halo_exposure"] = exposure
+        if deep is not None:
+            line["deep_halo"] = deep
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier(device_ids=[local_rank])
