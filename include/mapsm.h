@@ -17,7 +17,7 @@
  *     bit-packed 32 cells per 32-bit word on the device;
  *   - MAPSM_OP_CONV: fp32 window convolution (Table 1, "N-dimensional
  *     convolution"), cross-correlation with (2r+1)^2 row-major weights,
- *     1 <= r <= 4, one fmaf per tap in row-major (dy, dx) order starting from
+ *     1 <= r <= 8, one fmaf per tap in row-major (dy, dx) order starting from
  *     +0.0f (reading c11) so results are reproducible bit for bit;
  *   - MAPSM_OP_HISTOGRAM: the Reductive (Static) output pattern (P:L104,
  *     Fig 4): 256-bin histogram of a u8 image (bin = pixel value,
@@ -149,10 +149,14 @@ mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, mapsm_dtype 
  * the slabs and allocates both buffers of every local slab with 2r halo rows
  * (the Memory Analyzer's bounding box after both AnalyzeCalls, P:L167-169,
  * P:L281).  U8 grids: radius 1 = Life (bit-packed storage), radius 0 with
- * NO_CHECKS = histogram input (byte storage, one buffer).  F32: radius 1..4.
- * EUNSUPPORTED: any other radius/boundary combination.  EINVAL: a slab would
- * have fewer than r rows (g > 1), or Life with w % 64 != 0.  ENOMEM on
- * allocation failure.                                                        */
+ * NO_CHECKS = histogram input (byte storage, one buffer).  F32: radius 1..8
+ * (r <= 4: TMA row-pipeline kernels; r = 5..8: a
+ * shared-memory tile kernel, not eligible for MAPSM_EXCHANGE_P2P).
+ * Life takes any width w >= 1 (rows of ceil(w/32) words, the unused bits of
+ * the last word kept 0); w % 128 == 0 runs the TMA kernels, w % 64 == 0 a
+ * register kernel, other widths a word-per-thread kernel (SURVEY §8(f)
+ * NEXT-2).  EUNSUPPORTED: any other radius/boundary combination.  EINVAL: a
+ * slab would have fewer than r rows (g > 1).  ENOMEM on allocation failure. */
 mapsm_status mapsm_window_set(mapsm_grid grid, int radius, mapsm_boundary boundary);
 
 /* Operator: LIFE (weights must be NULL, dtype U8, r = 1), CONV (weights =

@@ -178,7 +178,7 @@ struct mapsm_grid_s {
     int r = 0;
     mapsm_boundary boundary = MAPSM_WRAP;
     mapsm_op op = MAPSM_OP_LIFE;
-    float wt[81] = {0};
+    float wt[17 * 17] = {0};       // conv weights, up to r = 8
     int state = ST_CREATED;
     int64_t pitch = 0;
     int64_t elem = 1;               // host bytes per cell
@@ -378,7 +378,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
     g->r = radius;
     g->halo = halo;
     g->boundary = boundary;
-    const int64_t row_bytes = g->packed() ? g->w / 8 : g->w * g->elem;
+    const int64_t row_bytes = g->packed() ? (g->w + 31) / 32 * 4 : g->w * g->elem;
     const int64_t align = row_bytes >= 128 ? 128 : 16;
     g->pitch = (row_bytes + align - 1) / align * align;
     const int nloc = c->local ? c->g : 1;
@@ -445,9 +445,8 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     if (g->dtype == MAPSM_U8) {
         if (radius != 1 && radius != 0)
             return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
-        if (radius == 1 && g->w % 64 != 0) return fail(MAPSM_EINVAL, "Life needs w %% 64 == 0 (w=%lld)", (long long)g->w);
     } else {
-        if (radius < 1 || radius > 4) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..4, got %d", radius);
+        if (radius < 1 || radius > 8) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..8, got %d", radius);
     }
     TRY(alloc_slabs(g, radius, boundary));
     g->state = ST_WINDOW;
@@ -653,7 +652,8 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1) {
 // Can this grid run the fused exchange?  (TMA kernels, every slab > 2r rows.)
 static bool p2p_eligible(const mapsm_grid_s* g) {
     if (g->op != MAPSM_OP_LIFE && g->op != MAPSM_OP_CONV) return false;
-    if (g->op == MAPSM_OP_LIFE && ((g->w / 32) % 4 != 0 || g->pitch % 16 != 0)) return false;
+    if (g->op == MAPSM_OP_CONV && g->r > 4) return false;  // r = 5..8 run the shared-memory tile kernel
+    if (g->op == MAPSM_OP_LIFE && (g->w % 128 != 0 || g->pitch % 16 != 0)) return false;
     if (g->op == MAPSM_OP_CONV && (g->w % 4 != 0 || g->pitch % 16 != 0)) return false;
     return g->h / g->ctx->g > 2 * (int64_t)g->r;
 }
@@ -778,7 +778,7 @@ static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
 // least K rows (mirror rows at CLAMP edges), copy/NCCL exchange.
 static bool tb_active(const mapsm_grid_s* g) {
     if (g->op != MAPSM_OP_LIFE || g->tb_k <= 1 || g->opt_p2p) return false;
-    if ((g->w / 32) % 4 != 0 || g->pitch % 16 != 0) return false;
+    if (g->w % 128 != 0 || g->pitch % 16 != 0) return false;
     for (auto& s : g->slabs)
         if (s.plan.rows < g->tb_k) return false;
     return true;
@@ -892,7 +892,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     // L2-resident Life slabs with no exchanged halos: persistent kernel, up to
     // kPersistChunk generations per cooperative launch.
     if (g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 && g->tb_k <= 1 &&
-        !has_exchange(g->slabs[0]) && 2 * g->slabs[0].plan.alloc_rows * g->pitch <= (64ll << 20)) {
+        !has_exchange(g->slabs[0]) && g->w % 64 == 0 && 2 * g->slabs[0].plan.alloc_rows * g->pitch <= (64ll << 20)) {
         Slab& s = g->slabs[0];
         CK(cudaSetDevice(s.device));
         if (!s.gbar) CK(cudaMalloc(&s.gbar, sizeof(unsigned int)));

@@ -1,5 +1,6 @@
 // conv.cu — radius dispatch of the fp32 window convolution (kernels in
-// conv_impl.cuh, one translation unit per radius: conv_r1.cu .. conv_r4.cu).
+// conv_impl.cuh, one translation unit per radius: conv_r1.cu .. conv_r4.cu;
+// radii 5..8 in conv_wide.cu).
 #include <cuda_runtime.h>
 
 #include "kernels.h"
@@ -17,6 +18,9 @@ cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, con
         case 2: return launch_conv_radius<2>(g, b, weights, num_sms, s, link);
         case 3: return launch_conv_radius<3>(g, b, weights, num_sms, s, link);
         case 4: return launch_conv_radius<4>(g, b, weights, num_sms, s, link);
+        case 5: case 6: case 7: case 8:
+            if (link) return cudaErrorInvalidValue;  // the fused exchange needs the TMA kernels (r <= 4)
+            return launch_conv_wide(g, b, r, weights, s);
         default: return cudaErrorInvalidValue;
     }
 }

@@ -69,9 +69,13 @@ cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, i
 cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst, int64_t dst_pitch,
                                int64_t rows, int64_t w, cudaStream_t s);
 
-// fp32 window convolution, radius r in 1..4, weights (2r+1)^2 row-major.
+// fp32 window convolution, radius r in 1..8, weights (2r+1)^2 row-major
+// (r <= 4: TMA row pipeline, conv_impl.cuh; r = 5..8: shared-memory tiles,
+// conv_wide.cu).
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
                              int num_sms, cudaStream_t s, const FusedLink* link = nullptr);
+
+cudaError_t launch_conv_wide(const StencilGeom& g, const RowBands& b, int r, const float* weights, cudaStream_t s);
 
 // Reductive (Static) output: 256-bin histogram of a u8 slab into out[256]
 // (zeroed here; 64-bit counts); and the sum of g partial histograms.

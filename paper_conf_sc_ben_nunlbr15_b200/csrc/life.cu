@@ -537,17 +537,92 @@ cudaError_t launch_life_tma(const StencilGeom& g, const RowBands& b, int num_sms
     return launch_life_tma_nc<2, NS>(g, b, num_sms, s, link);
 }
 
+// ------------------------------------------------ any width
+// Widths that are not a multiple of 64 cells: a row has nw = ceil(w/32) words,
+// the last one holding b = w - 32(nw-1) cells in bits 0..b-1 (bits >= b are
+// kept 0).  One thread per output word; the neighbour bits across word ends
+// come from the adjacent words, and at the row ends from the boundary rule:
+// WRAP pairs column w-1 (bit b-1 of the last word) with column 0.  A
+// correctness path (the configs' widths all take the TMA kernel).
+template <int CM>
+__global__ void life_anyw_kernel(const __grid_constant__ LifeParams p, int tail_bits) {
+    const int64_t m = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    const int band = blockIdx.z;
+    if (m >= p.nw) return;
+    const int64_t last = p.nw - 1;
+    const uint32_t tail_mask = tail_bits == 32 ? ~0u : ((1u << tail_bits) - 1u);
+    for (int64_t y = p.begin[band] + blockIdx.y; y < p.end[band]; y += gridDim.y) {
+        uint32_t r0[3], r1[3], mid = 0;
+#pragma unroll
+        for (int k = 0; k < 3; ++k) {
+            const uint32_t* row = p.in + map_row(p, y + k - 1) * p.pitch_w;
+            const uint32_t x = __ldg(row + m);
+            const uint32_t first = __ldg(row);
+            const uint32_t lastw = __ldg(row + last);
+            // cell left of bit 0 of word m, and right of the word's last cell
+            uint32_t lbit, rbit;
+            if (m > 0) {
+                lbit = __ldg(row + m - 1) >> 31;
+            } else {
+                lbit = CM == COL_WRAP ? (lastw >> (tail_bits - 1)) & 1u : CM == COL_CLAMP ? (x & 1u) : 0u;
+            }
+            uint32_t R;
+            if (m < last) {
+                R = (x >> 1) | (__ldg(row + m + 1) << 31);
+            } else {
+                const uint32_t e = CM == COL_WRAP ? (first & 1u) : CM == COL_CLAMP ? ((x >> (tail_bits - 1)) & 1u) : 0u;
+                R = (x >> 1) | (e << (tail_bits - 1));  // bits >= tail_bits of x are 0
+            }
+            const uint32_t L = (x << 1) | lbit;
+            r0[k] = L ^ x ^ R;
+            r1[k] = maj3(L, x, R);
+            if (k == 1) mid = x;
+        }
+        uint32_t o = life_word(r0[0], r1[0], r0[1], r1[1], r0[2], r1[2], mid);
+        if (m == last) o &= tail_mask;
+        p.out[y * p.pitch_w + m] = o;
+    }
+}
+
+template <int CM>
+cudaError_t launch_life_anyw_t(const StencilGeom& g, const RowBands& b, cudaStream_t s) {
+    LifeParams p;
+    p.in = static_cast<const uint32_t*>(g.in);
+    p.out = static_cast<uint32_t*>(g.out);
+    p.pitch_w = g.pitch / 4;
+    p.rows = g.rows;
+    p.nw = (g.w + 31) / 32;
+    p.nvec = p.nw;
+    p.warps_per_row = 0;
+    p.top_map = g.top_map;
+    p.bot_map = g.bot_map;
+    p.col_mode = g.col_mode;
+    int64_t maxr = 0;
+    for (int i = 0; i < 2; ++i) {
+        p.begin[i] = i < b.nbands ? b.begin[i] : 0;
+        p.end[i] = i < b.nbands ? b.end[i] : 0;
+        p.nchunks[i] = 0;
+        if (p.end[i] - p.begin[i] > maxr) maxr = p.end[i] - p.begin[i];
+    }
+    if (maxr <= 0) return cudaSuccess;
+    const int tail = (int)(g.w - 32 * (p.nw - 1));
+    dim3 grid((unsigned)((p.nw + 127) / 128), (unsigned)(maxr < 8192 ? maxr : 8192), (unsigned)b.nbands);
+    life_anyw_kernel<CM><<<grid, 128, 0, s>>>(p, tail);
+    return cudaGetLastError();
+}
+
 // ------------------------------------------------------------ pack / unpack
 // u8 (nonzero = alive) -> bits; one thread per 32-bit word (32 bytes in).
 __global__ void pack_life_kernel(const uint8_t* __restrict__ src, int64_t src_pitch,
                                  uint32_t* __restrict__ dst, int64_t dst_pitch_w, int64_t rows,
-                                 int64_t nw, bool vec) {
+                                 int64_t nw, int64_t w, bool vec) {
     const int64_t wi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t y = blockIdx.y + (int64_t)blockIdx.z * gridDim.y;
     if (wi >= nw || y >= rows) return;
     const uint8_t* s = src + y * src_pitch + wi * 32;
     uint32_t word = 0;
-    if (vec) {
+    const int64_t nb = w - wi * 32;  // cells in this word (< 32 only for the last word of an odd width)
+    if (vec && nb >= 32) {
         const uint4 q0 = __ldg(reinterpret_cast<const uint4*>(s));
         const uint4 q1 = __ldg(reinterpret_cast<const uint4*>(s + 16));
         const uint32_t v[8] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w};
@@ -559,7 +634,7 @@ __global__ void pack_life_kernel(const uint8_t* __restrict__ src, int64_t src_pi
             word |= ((m * 0x00204081u) >> 28) << (4 * q);
         }
     } else {
-        for (int j = 0; j < 32; ++j) word |= (uint32_t)(s[j] != 0) << j;
+        for (int j = 0; j < 32 && j < nb; ++j) word |= (uint32_t)(s[j] != 0) << j;
     }
     dst[y * dst_pitch_w + wi] = word;
 }
@@ -567,7 +642,7 @@ __global__ void pack_life_kernel(const uint8_t* __restrict__ src, int64_t src_pi
 // bits -> u8 0/1; one thread per 32-bit word (32 bytes out).
 __global__ void unpack_life_kernel(const uint32_t* __restrict__ src, int64_t src_pitch_w,
                                    uint8_t* __restrict__ dst, int64_t dst_pitch, int64_t rows,
-                                   int64_t nw, bool vec) {
+                                   int64_t nw, int64_t w, bool vec) {
     const int64_t wi = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
     const int64_t y = blockIdx.y + (int64_t)blockIdx.z * gridDim.y;
     if (wi >= nw || y >= rows) return;
@@ -576,11 +651,12 @@ __global__ void unpack_life_kernel(const uint32_t* __restrict__ src, int64_t src
     uint32_t v[8];
 #pragma unroll
     for (int q = 0; q < 8; ++q) v[q] = (((word >> (4 * q)) & 0xFu) * 0x00204081u) & 0x01010101u;
-    if (vec) {
+    const int64_t nb = w - wi * 32;
+    if (vec && nb >= 32) {
         *reinterpret_cast<uint4*>(d) = make_uint4(v[0], v[1], v[2], v[3]);
         *reinterpret_cast<uint4*>(d + 16) = make_uint4(v[4], v[5], v[6], v[7]);
     } else {
-        for (int j = 0; j < 32; ++j) d[j] = (uint8_t)((word >> j) & 1u);
+        for (int j = 0; j < 32 && j < nb; ++j) d[j] = (uint8_t)((word >> j) & 1u);
     }
 }
 
@@ -686,39 +762,44 @@ cudaError_t launch_life_persist_v(const StencilGeom& g, int64_t n, unsigned int*
 
 cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sms, cudaStream_t s,
                              const FusedLink* link) {
-    const int64_t nw = g.w / 32;
-    if (nw % 4 == 0 && g.pitch % 16 == 0) return launch_life_tma<kTmaNS>(g, b, num_sms, s, link);
+    if (g.w % 128 == 0 && g.pitch % 16 == 0) return launch_life_tma<kTmaNS>(g, b, num_sms, s, link);
     if (link || b.nbands > 2) return cudaErrorInvalidValue;  // fused exchange needs the TMA kernel
-    return launch_life_cm<2, kLifeP>(g, b, num_sms, s);
+    if (g.w % 64 == 0) return launch_life_cm<2, kLifeP>(g, b, num_sms, s);
+    switch (g.col_mode) {
+        case COL_WRAP: return launch_life_anyw_t<COL_WRAP>(g, b, s);
+        case COL_CLAMP: return launch_life_anyw_t<COL_CLAMP>(g, b, s);
+        default: return launch_life_anyw_t<COL_ZERO>(g, b, s);
+    }
 }
 
 cudaError_t launch_life_persistent(const StencilGeom& g, int64_t n, unsigned int* bar, int num_sms, cudaStream_t s) {
     if (n <= 0) return cudaSuccess;
-    if ((g.w / 32) % 4 == 0 && g.pitch % 16 == 0) return launch_life_persist_v<4>(g, n, bar, num_sms, s);
+    if (g.w % 64 != 0) return cudaErrorInvalidValue;  // odd widths: per-generation launches
+    if (g.w % 128 == 0 && g.pitch % 16 == 0) return launch_life_persist_v<4>(g, n, bar, num_sms, s);
     return launch_life_persist_v<2>(g, n, bar, num_sms, s);
 }
 
 cudaError_t launch_pack_life(const uint8_t* src, int64_t src_pitch, void* dst, int64_t dst_pitch,
                              int64_t rows, int64_t w, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
-    const int64_t nw = w / 32;
+    const int64_t nw = (w + 31) / 32;
     const bool vec = (src_pitch % 16 == 0) && ((uintptr_t)src % 16 == 0);
     const unsigned ty = (unsigned)(rows < 32768 ? rows : 32768);
     dim3 grid((unsigned)((nw + 255) / 256), ty, (unsigned)((rows + ty - 1) / ty));
     pack_life_kernel<<<grid, 256, 0, s>>>(src, src_pitch, static_cast<uint32_t*>(dst), dst_pitch / 4,
-                                          rows, nw, vec);
+                                          rows, nw, w, vec);
     return cudaGetLastError();
 }
 
 cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst, int64_t dst_pitch,
                                int64_t rows, int64_t w, cudaStream_t s) {
     if (rows <= 0) return cudaSuccess;
-    const int64_t nw = w / 32;
+    const int64_t nw = (w + 31) / 32;
     const bool vec = (dst_pitch % 16 == 0) && ((uintptr_t)dst % 16 == 0);
     const unsigned ty = (unsigned)(rows < 32768 ? rows : 32768);
     dim3 grid((unsigned)((nw + 255) / 256), ty, (unsigned)((rows + ty - 1) / ty));
     unpack_life_kernel<<<grid, 256, 0, s>>>(static_cast<const uint32_t*>(src), src_pitch / 4, dst,
-                                            dst_pitch, rows, nw, vec);
+                                            dst_pitch, rows, nw, w, vec);
     return cudaGetLastError();
 }
 

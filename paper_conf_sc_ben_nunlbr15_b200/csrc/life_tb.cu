@@ -54,7 +54,15 @@ namespace mapsm {
 namespace tb {
 
 constexpr int kOut = 30;     // words stored per warp (lanes 1..30)
-constexpr int kMaxNC = 15;   // consumer warps per CTA (16 warps x 128 registers = the register file; 4 warps x 128 per SMSP)
+#ifndef MAPSM_TB_MAXNC
+#define MAPSM_TB_MAXNC 15
+#endif
+#ifndef MAPSM_TB_REGS
+#define MAPSM_TB_REGS 128
+#endif
+// consumer warps per CTA: 16 warps x 128 registers fill the register file
+// (4 warps x 128 registers x 32 lanes = one SMSP's 16K registers)
+constexpr int kMaxNC = MAPSM_TB_MAXNC;
 #ifndef MAPSM_TB_NS
 #define MAPSM_TB_NS 8
 #endif
@@ -262,7 +270,7 @@ __device__ __forceinline__ void tb_consume_segment(const TbParams& P, const TbSe
 }
 
 template <int K, int NS, int CM>
-__global__ void __maxnreg__(128) life_tb_kernel(const __grid_constant__ TbParams P) {
+__global__ void __maxnreg__(MAPSM_TB_REGS) life_tb_kernel(const __grid_constant__ TbParams P) {
     static_assert(K >= 1 && K <= 31, "ghost words stay exact for at most 31 generations");
     constexpr int RPS = rows_per_stage(K);
     const tma::RowStream& p = P.s;
@@ -379,7 +387,7 @@ cudaError_t launch_life_tb(const StencilGeom& g, const RowBands& b, int k, int z
                            cudaStream_t s) {
     using namespace tb;
     const int64_t W = g.w / 32;
-    if (W % 4 != 0 || g.pitch % 16 != 0 || !life_tb_supported(k)) return cudaErrorInvalidValue;
+    if (g.w % 128 != 0 || g.pitch % 16 != 0 || !life_tb_supported(k)) return cudaErrorInvalidValue;
     TbParams P;
     tma::RowStream& p = P.s;
     p.in = static_cast<const uint32_t*>(g.in);

@@ -117,3 +117,48 @@ def test_config5_9x9_zero_single_gpu_slab_sampled(ctx):
         exp = cone_eval("conv", gen, h, w, r, n, "zero", ys, ys + 4, xs, xs + 8, W)
         got = dev[ys:ys + 4, xs:xs + 8].cpu().numpy()
         gate(got, exp)
+
+
+# ------------------------------------------- radii 5..8
+
+@pytest.mark.parametrize("r", [5, 6, 7, 8])
+@pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
+@pytest.mark.parametrize("shape", [(128, 40), (300, 70), (5, 17), (17, 9), (257, 33)])
+def test_wide_radius_vs_oracle(ctx, r, b, shape):
+    """The shared-memory tile kernel: tiles of 32 x 128 outputs, ragged in
+    both directions, windows wider than the grid under WRAP (multiplicity)."""
+    w, h = shape
+    f0 = mi.field_f32(500 + w + r, w, h)
+    W = mi.weights_f32(600 + r, r)
+    for n in (1, 2):
+        out, _ = run(ctx, f0, W, n, b)
+        gate(out, oracle.conv(f0, W, n, b))
+
+
+@pytest.mark.parametrize("g", [2, 3])
+@pytest.mark.parametrize("b", ["wrap", "zero"])
+def test_wide_radius_local_multislab(local_ctx, g, b):
+    """r = 8 halos of 8 rows exchanged between slabs every iteration."""
+    r = 8
+    h, w = g * 20 + 3, 160
+    f0 = mi.field_f32(77 + g, w, h)
+    W = mi.weights_f32(78, r)
+    out, info = run(local_ctx(g), f0, W, 3, b)
+    gate(out, oracle.conv(f0, W, 3, b))
+    assert info.radius == r
+
+
+def test_wide_radius_limits(ctx, local_ctx):
+    gh = M.mapsm_grid_create(ctx, 64, 64, M.F32)
+    try:
+        with pytest.raises(M.MapsmError) as e:
+            M.mapsm_window_set(gh, 9, M.WRAP)
+        assert e.value.status == M.EUNSUPPORTED
+    finally:
+        M.mapsm_grid_destroy(gh)
+    # the fused peer-memory exchange needs the TMA kernels (r <= 4)
+    with M.Grid(local_ctx(2), 128, 64, "conv", 5, "wrap", mi.weights_f32(1, 5)) as g:
+        g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
+        with pytest.raises(M.MapsmError) as e:
+            g.bind(mi.field_f32(1, 128, 64))
+        assert e.value.status == M.EUNSUPPORTED

@@ -151,11 +151,10 @@ def test_state_machine_and_errors(ctx):
         assert e.value.status == M.ESTATE
     finally:
         M.mapsm_grid_destroy(gh)
-    gh = M.mapsm_grid_create(ctx, 100, 10, M.U8)
+    gh = M.mapsm_grid_create(ctx, 100, 10, M.U8)  # any width is accepted (NEXT-2)
     try:
-        with pytest.raises(M.MapsmError) as e:
-            M.mapsm_window_set(gh, 1, M.WRAP)
-        assert e.value.status == M.EINVAL
+        M.mapsm_window_set(gh, 1, M.WRAP)
+        assert M.mapsm_get_info(gh).pitch_bytes == 16
     finally:
         M.mapsm_grid_destroy(gh)
 
@@ -202,3 +201,38 @@ def test_config3_65536_bench_size_sampled(ctx):
         assert np.array_equal(got, exp), (ys, xs)
     # population sanity at any size: 0/1 only
     assert int(dev.max()) <= 1
+
+
+# ------------------------------------------- any width
+
+@pytest.mark.parametrize("w", [1, 2, 3, 31, 32, 33, 63, 65, 96, 100, 161, 1000])
+@pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
+def test_any_width_vs_oracle(ctx, w, b):
+    """Rows of ceil(w/32) words with a partial last word: WRAP pairs column
+    w-1 (bit (w-1) % 32 of the last word) with column 0; unused bits stay 0."""
+    h = 37
+    g0 = mi.life_u8(900 + w, w, h)
+    for n in (1, 5):
+        out, info = run(ctx, g0, n, b)
+        assert np.array_equal(out, oracle.life(g0, n, b)), n
+
+
+@pytest.mark.parametrize("g", [2, 3])
+def test_any_width_local_multislab(local_ctx, g):
+    g0 = mi.life_u8(55, 77, 40)
+    out, _ = run(local_ctx(g), g0, 9, "wrap")
+    assert np.array_equal(out, oracle.life(g0, 9, "wrap"))
+
+
+def test_any_width_device_pointers(ctx):
+    import torch
+
+    g0 = mi.life_u8(8, 45, 30)
+    t = torch.from_numpy(g0).cuda()
+    with M.Grid(ctx, 45, 30, "life", 1, "clamp") as g:
+        g.bind(t)
+        g.iterate(4)
+        o = torch.full_like(t, 7)
+        M.mapsm_read(g.handle, o)
+        torch.cuda.synchronize()
+    assert np.array_equal(o.cpu().numpy(), oracle.life(g0, 4, "clamp"))

@@ -83,7 +83,7 @@ def test_min_slab_height_equals_r():
         assert all(p.rows == r for p in ps)
 
 
-@pytest.mark.parametrize("g,h", itertools.product([2, 4, 8], [65536, 16384, 32768]))
+@pytest.mark.parametrize("g,h", list(itertools.product([2, 4, 8], [65536, 16384, 32768])))
 def test_bench_configs_partition(g, h):
     for p in plans(h, g, 4 if h == 32768 else 1, M.WRAP):
         assert p.rows == h // g
