@@ -27,6 +27,8 @@ SEED_CONV9_FIELD = 0x5EED0005
 SEED_CONV9_W = 0x5EED0055
 SEED_HIST_UNIFORM = 0x5EED0006
 SEED_HIST_SKEWED = 0x5EED0066
+SEED_CONV3D_FIELD = 0x5EED0007
+SEED_CONV3D_W = 0x5EED0077
 
 
 def build(force: bool = False) -> str:
@@ -51,6 +53,8 @@ def _L():
         _lib.mapsm_gen_field_f32.restype = None
         _lib.mapsm_gen_weights_f32.argtypes = [u64, ctypes.c_int, p]
         _lib.mapsm_gen_weights_f32.restype = None
+        _lib.mapsm_gen_weights_n_f32.argtypes = [u64, ctypes.c_int, p]
+        _lib.mapsm_gen_weights_n_f32.restype = ctypes.c_int
         _lib.mapsm_gen_image_u8.argtypes = [u64, i64, i64, i64, p, i64, ctypes.c_int]
         _lib.mapsm_gen_image_u8.restype = None
     return _lib
@@ -84,6 +88,21 @@ def weights_f32(seed: int, r: int) -> np.ndarray:
     out = np.empty(k * k, dtype=np.float32)
     _L().mapsm_gen_weights_f32(seed, r, out.ctypes.data)
     return out.reshape(k, k)
+
+
+def weights3d_f32(seed: int, r: int) -> np.ndarray:
+    """(2r+1)^3 non-negative asymmetric weights summing to ~1, (dz, dy, dx) order."""
+    k = 2 * r + 1
+    out = np.empty(k ** 3, dtype=np.float32)
+    assert _L().mapsm_gen_weights_n_f32(seed, k ** 3, out.ctypes.data) == 0
+    return out.reshape(k, k, k)
+
+
+def volume_f32(seed: int, w: int, h: int, d: int, z0: int = 0) -> np.ndarray:
+    """Planes [z0, z0+d) of a synthetic (depth, h, w) fp32 volume: the 2-D
+    field recipe over global row index z*h + y, so plane z of the volume is
+    rows [z*h, (z+1)*h) of field_f32(seed, w, ...)."""
+    return field_f32(seed, w, d * h, y0=z0 * h).reshape(d, h, w)
 
 
 def image_u8(seed: int, w: int, h: int, y0: int = 0, kind: str = "uniform",

@@ -57,6 +57,18 @@ void mapsm_gen_weights_f32(uint64_t seed, int r, float* out) {
     for (int t = 0; t < taps; ++t) out[t] = (float)(raw[t] / sum);
 }
 
+/* `taps` weights by the same recipe (Window(3D): (2r+1)^3, ordered (dz,dy,dx)). */
+int mapsm_gen_weights_n_f32(uint64_t seed, int taps, float* out) {
+    double raw[4096], sum = 0.0;
+    if (taps < 1 || taps > 4096) return -1;
+    for (int t = 0; t < taps; ++t) {
+        raw[t] = (double)((splitmix64(seed + (uint64_t)t) >> 40) + 1) * (1.0 / 16777216.0);
+        sum += raw[t];
+    }
+    for (int t = 0; t < taps; ++t) out[t] = (float)(raw[t] / sum);
+    return 0;
+}
+
 /* u8 images for the histogram (Reductive-Static) path, rows [y0, y0+rows),
  * row stride `pitch` bytes.  kind 0: uniform, pixel = v >> 56.
  * kind 1: skewed ("natural-image-like" concentration around 128 that makes

@@ -12,7 +12,11 @@ Parity status: Life pinned (closed forms, scipy neighbour count,
 known methuselah, exhaustive tiny tori); fp32 conv pinned (exact-rational fma
 chain, scipy correlate in fp64, roll/identity closed forms, mass invariant);
 fp64 conv pinned (scipy correlate); histogram pinned (numpy.bincount, closed
-forms, invariants).  No function is "parity unpinned".
+forms, invariants); fp32-field histogram pinned (closed forms at bin edges,
+numpy.floor/clip binning); Segment Location Monitor (``oracle/locmon.py``)
+pinned by the paper's worked cases (Fig 3 halos, Reductive aggregation,
+upToDate reuse) and brute-force cell enumeration.  No function is "parity
+unpinned".
 """
 from __future__ import annotations
 
@@ -54,6 +58,10 @@ def _L():
         _lib.oracle_num_threads.restype = ci
         _lib.oracle_histogram.argtypes = [p, i64, i64, i64, ci, p]
         _lib.oracle_histogram.restype = ci
+        _lib.oracle_conv3d_ex.argtypes = [p, p, i64, i64, i64, i64, ci, p, p]
+        _lib.oracle_conv3d_ex.restype = ci
+        _lib.oracle_histogram_f32.argtypes = [p, i64, i64, i64, ci, p]
+        _lib.oracle_histogram_f32.restype = ci
     return _lib
 
 
@@ -110,6 +118,25 @@ def conv_f64(field: np.ndarray, weights: np.ndarray, n: int, boundary="wrap", si
     return out
 
 
+def conv3d(vol: np.ndarray, weights: np.ndarray, n: int, boundary="wrap", sides=None) -> np.ndarray:
+    """n steps of the fp32 Window(3D) convolution of a (d, h, w) volume with
+    (2r+1)^3 weights ordered (dz, dy, dx); `sides` = 6 modes (z lo, z hi, y lo,
+    y hi, x lo, x hi) overriding `boundary`."""
+    v = np.ascontiguousarray(vol, dtype=np.float32)
+    wt = np.ascontiguousarray(weights, dtype=np.float32).ravel()
+    k = round(len(wt) ** (1 / 3))
+    assert k ** 3 == len(wt) and k % 2 == 1
+    d, h, w = v.shape
+    modes = np.array(sides if sides is not None else [_mode(boundary)] * 6, dtype=np.int32)
+    modes = np.array([_mode(m) for m in modes], dtype=np.int32)
+    out = np.empty_like(v)
+    rc = _L().oracle_conv3d_ex(v.ctypes.data, out.ctypes.data, w, h, d, n, k // 2, wt.ctypes.data,
+                               modes.ctypes.data)
+    if rc != 0:
+        raise ValueError("oracle_conv3d_ex rejected its arguments")
+    return out
+
+
 def histogram(img: np.ndarray, nbins: int = 256) -> np.ndarray:
     """256-bin histogram of a u8 image (Reductive-Static pattern, Fig 4)."""
     a = np.asarray(img)
@@ -119,6 +146,18 @@ def histogram(img: np.ndarray, nbins: int = 256) -> np.ndarray:
     rc = _L().oracle_histogram(a.ctypes.data, w, h, a.strides[0] if h > 0 else w, nbins, out.ctypes.data)
     if rc != 0:
         raise ValueError("oracle_histogram rejected its arguments")
+    return out
+
+
+def histogram_f32(field: np.ndarray, nbins: int = 256) -> np.ndarray:
+    """256-bin histogram of an fp32 field over [0, 1): bin = floor(v * 256),
+    clamped to [0, 255], NaN -> 0 (reading h4)."""
+    a = np.ascontiguousarray(field, dtype=np.float32)
+    h, w = a.shape
+    out = np.zeros(nbins, dtype=np.uint64)
+    rc = _L().oracle_histogram_f32(a.ctypes.data, w, h, w, nbins, out.ctypes.data)
+    if rc != 0:
+        raise ValueError("oracle_histogram_f32 rejected its arguments")
     return out
 
 

@@ -222,6 +222,67 @@ int oracle_conv_f64(const float* in, double* out, int64_t w, int64_t h, int64_t 
     return oracle_conv_f64_ex(in, out, w, h, n, r, weights, boundary, boundary, boundary, boundary);
 }
 
+/* ------------------------------------------------------ Window (3D) */
+
+/* Window (3D) input pattern (§5.3: "each image in the batch is
+ * separately convolved in three dimensions ... This corresponds to the Window
+ * (3D) input memory access pattern, using the Structured Injective output";
+ * Table 1 P:L87-88 "N-dimensional convolution").  A d x h
+ * x w fp32 volume (plane-major: index (z*h + y)*w + x), cross-correlation with
+ * (2r+1)^3 weights ordered (dz, dy, dx) row-major, one correctly rounded fmaf
+ * per tap starting from +0.0f (the 3-D extension of reading c11, DESIGN.md
+ * reading v1):
+ *     acc = +0.0f
+ *     for dz = -r..r: for dy = -r..r: for dx = -r..r:
+ *         acc = fmaf(W[((dz+r)(2r+1) + (dy+r))(2r+1) + (dx+r)], cell(z+dz, y+dy, x+dx), acc)
+ * cell() resolves each axis with its own side modes exactly as in 2-D. */
+static float conv3_cell(const float* G, int64_t w, int64_t h, int64_t d, int64_t z, int64_t y, int64_t x,
+                        const int* m) {
+    int64_t zz = resolve(z, d, m[0], m[1]);
+    int64_t yy = resolve(y, h, m[2], m[3]);
+    int64_t xx = resolve(x, w, m[4], m[5]);
+    if (zz < 0 || yy < 0 || xx < 0) return 0.0f;
+    return G[(zz * h + yy) * w + xx];
+}
+
+static void conv3_step_f32(const float* G, float* out, int64_t w, int64_t h, int64_t d, int r, const float* W,
+                           const int* m) {
+    int k = 2 * r + 1;
+#pragma omp parallel for schedule(static) collapse(2)
+    for (int64_t z = 0; z < d; ++z)
+        for (int64_t y = 0; y < h; ++y)
+            for (int64_t x = 0; x < w; ++x) {
+                float acc = 0.0f;
+                for (int dz = -r; dz <= r; ++dz)
+                    for (int dy = -r; dy <= r; ++dy)
+                        for (int dx = -r; dx <= r; ++dx)
+                            acc = fmaf(W[((dz + r) * k + (dy + r)) * k + (dx + r)],
+                                       conv3_cell(G, w, h, d, z + dz, y + dy, x + dx, m), acc);
+                out[(z * h + y) * w + x] = acc;
+            }
+}
+
+/* n steps; modes[6] = (z lo, z hi, y lo, y hi, x lo, x hi).  Returns 0 or -1. */
+int oracle_conv3d_ex(const float* in, float* out, int64_t w, int64_t h, int64_t d, int64_t n, int r,
+                     const float* weights, const int* modes) {
+    if (w <= 0 || h <= 0 || d <= 0 || n < 0 || r < 0 || !modes) return -1;
+    if (!check_modes(modes[0], modes[1], modes[2], modes[3]) || !check_modes(modes[4], modes[5], modes[4], modes[5]))
+        return -1;
+    size_t cells = (size_t)w * (size_t)h * (size_t)d;
+    float* a = (float*)malloc(cells * sizeof(float));
+    float* b = (float*)malloc(cells * sizeof(float));
+    if (!a || !b) { free(a); free(b); return -1; }
+    memcpy(a, in, cells * sizeof(float));
+    for (int64_t t = 0; t < n; ++t) {
+        conv3_step_f32(a, b, w, h, d, r, weights, modes);
+        float* tmp = a; a = b; b = tmp;
+    }
+    memcpy(out, a, cells * sizeof(float));
+    free(a);
+    free(b);
+    return 0;
+}
+
 /* ------------------------------------------------------------ Histogram */
 
 /* Reductive (Static) output pattern (§3.2; Fig 4 P:L359-403 §4.5.3,
@@ -234,6 +295,24 @@ int oracle_histogram(const uint8_t* img, int64_t w, int64_t h, int64_t pitch, in
     for (int b = 0; b < nbins; ++b) bins[b] = 0;
     for (int64_t y = 0; y < h; ++y)
         for (int64_t x = 0; x < w; ++x) bins[img[y * pitch + x]] += 1;
+    return 0;
+}
+
+/* Histogram task over an fp32 field (reading h4): 256
+ * bins over [0, 1), bin = floor(v * 256) evaluated in double (v * 256 is
+ * exact), below 0 (and NaN) -> bin 0, at or above 256 -> bin 255. */
+int oracle_histogram_f32(const float* img, int64_t w, int64_t h, int64_t pitch_floats, int nbins, uint64_t* bins) {
+    if (w < 0 || h < 0 || pitch_floats < w || nbins != 256 || !bins) return -1;
+    for (int b = 0; b < nbins; ++b) bins[b] = 0;
+    for (int64_t y = 0; y < h; ++y)
+        for (int64_t x = 0; x < w; ++x) {
+            const double s = floor((double)img[y * pitch_floats + x] * 256.0);
+            int b;
+            if (!(s >= 0.0)) b = 0;
+            else if (s > 255.0) b = 255;
+            else b = (int)s;
+            bins[b] += 1;
+        }
     return 0;
 }
 
