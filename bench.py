@@ -420,7 +420,40 @@ def main():
     h2d = h * w * elem
     d2h = 256 * 8 * world if op == "histogram" else h * w * elem
 
+    # Chained task: a Reductive-Static histogram task over
+    # the current generation, its data movement inferred by the Segment Location
+    # Monitor (Alg 2) — 0 bytes on the grid's own partition.  Timed per call
+    # (memset + kernel + aggregation + bins copy), after an L2 flush.
+    chained = None
+    if op != "histogram":
+        d_b = torch.zeros(256, dtype=torch.int64, device=dev)
+        _, moved = M.mapsm_task_histogram(grid.handle, 0, d_b)
+        c_ms = 0.0
+        for _ in range(args.steps):
+            flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            M.mapsm_task_histogram(grid.handle, 0, d_b)
+            e1.record(stream)
+            e1.synchronize()
+            c_ms += e0.elapsed_time(e1)
+        tc = torch.tensor([c_ms], dtype=torch.float64, device=dev)
+        if world > 1:
+            dist.all_reduce(tc, op=dist.ReduceOp.MAX)
+        c_s = float(tc.item()) / 1e3 / args.steps
+        tb = 0.125 if op == "life" else 4.0   # bytes read per cell (1 bit / one fp32)
+        ach = tb * rows * w / c_s / 1e9
+        chained = {"task": "histogram of the current generation (mapsm_task_histogram, grid's own partition)",
+                   "moved_bytes": int(moved), "ms_per_call": c_s * 1e3, "cells_per_s": h * w / c_s,
+                   "roofline": {"bound": "hbm", "kernel": "histogram_life_kernel" if op == "life"
+                                else "histogram_f32_kernel", "bytes_per_unit": tb, "achieved": ach,
+                                "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
+                                "note": "whole call timed (memset + kernel + bins copy + sync)"}}
+
     grid.close()
+
+    # Deep halos    grid.close()
 
     # Deep halos (MAPSM_OPT_DEEP_HALO): the same workload
     # with K generations per pass and K-row halos exchanged once per pass —
@@ -508,6 +541,8 @@ def main():
             line["halo_exposure"] = exposure
         if deep is not None:
             line["deep_halo"] = deep
+        if chained is not None:
+            line["chained_task"] = chained
         print(json.dumps(line), flush=True)
     if world > 1:
         dist.barrier(device_ids=[local_rank])

@@ -116,6 +116,53 @@ typedef struct {
 mapsm_status mapsm_plan_query(int64_t h, int g, int radius, mapsm_boundary boundary, int rank,
                               mapsm_slab_plan* out);
 
+/* ------------------------------------------------- segment location monitor
+ * Alg 2 (§4.4): tracks, per datum, `lastOutput` (the segments the
+ * last task wrote, per location, and whether they are partials that still
+ * need aggregation) and `upToDate` (every location holding an unmodified
+ * instance of a segment, "to avoid unnecessary memory transfers"),
+ * and answers "which copies bring this segment up to date on that target".
+ * Pure host code, needs no GPU.  The runtime uses one monitor per grid for
+ * chained tasks (mapsm_task_histogram); these entry points expose the same
+ * monitor for tests and for callers composing their own tasks.
+ * Boxes are half-open N-D rectangles, dimension 0 = rows (slowest); unused
+ * dimensions must be [0, 1).  Locations are caller-chosen ints (the runtime
+ * uses the global slab index for slab buffers; -1 conventionally = host).
+ * Readings (DESIGN.md l1-l3): "up to date on the target" is tested on the
+ * union of the target's up-to-date boxes, and only the part of the segment
+ * the target lacks is copied; partials awaiting aggregation are never up to
+ * date, and every overlapping partial is copied with needs_aggregation = 1. */
+#define MAPSM_MAX_DIMS 3
+typedef struct {
+    int64_t lo[MAPSM_MAX_DIMS], hi[MAPSM_MAX_DIMS];
+} mapsm_box;
+typedef struct {
+    int src, dst;   /* locations */
+    mapsm_box box;  /* the segment to copy (global coordinates) */
+} mapsm_copy_op;
+typedef struct mapsm_locmon_s* mapsm_locmon;
+
+/* ndims in 1..3, else EINVAL.                                                */
+mapsm_status mapsm_locmon_create(int ndims, mapsm_locmon* out);
+mapsm_status mapsm_locmon_destroy(mapsm_locmon m);
+/* A task wrote a new version of `datum` (>= 0): segment i at locs[i] covers
+ * boxes[i] (arrays of nseg, copied).  lastOutput := these segments; upToDate
+ * := the same unless needs_aggregation (duplicated partial outputs, the
+ * Reductive pattern).                                            */
+mapsm_status mapsm_locmon_output(mapsm_locmon m, int datum, int nseg, const int* locs, const mapsm_box* boxes,
+                                 int needs_aggregation);
+/* Alg 2 for segment `required` of `datum` on location `target`: writes the
+ * copy list to ops[0..*n_ops) (*n_ops is set even when it exceeds max_ops, in
+ * which case ENOMEM is returned and nothing is written) and the
+ * needsAggregation flag.  ESTATE: unknown datum (never output).  EINVAL: part
+ * of `required` lies outside every lastOutput segment.                      */
+mapsm_status mapsm_locmon_query(mapsm_locmon m, int datum, const mapsm_box* required, int target,
+                                mapsm_copy_op* ops, int max_ops, int* n_ops, int* needs_aggregation);
+/* The copies in ops[0..nops) completed: their destinations now hold
+ * up-to-date instances (the closing step of Alg 2).  No effect on a
+ * datum whose lastOutput needs aggregation.                                  */
+mapsm_status mapsm_locmon_copied(mapsm_locmon m, int datum, int nops, const mapsm_copy_op* ops);
+
 /* ------------------------------------------------------------------- context */
 
 /* Multi-process mode: one process (rank of world) per GPU.  `nccl_unique_id`
@@ -144,6 +191,22 @@ mapsm_status mapsm_nccl_unique_id(void* out128);
 /* Declare a w x h datum.  dtype U8 for Life, F32 for conv.          */
 mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, mapsm_dtype dtype,
                                mapsm_grid* out);
+
+/* Window(3D) datum (§5.3 "convolved in three
+ * dimensions ... the Window (3D) input memory access pattern", Table 1
+ * P:L87-88): a d x h x w fp32 volume, plane-major (host layout: plane z, row
+ * y at row index z*h + y of a row-pitched 2-D buffer of d*h rows).  Only
+ * dtype F32 (EUNSUPPORTED otherwise).  The volume is partitioned in PLANES
+ * over the slabs (like the rows of a 2-D grid), with r halo planes exchanged
+ * per iteration; every call below then counts planes where it says rows for
+ * partition purposes (mapsm_grid_slab returns (z0, planes); mapsm_bind /
+ * mapsm_read take this process's planes [z0, z0+planes) as planes*h rows).
+ * mapsm_window_set: radius 1..2, boundary WRAP / CLAMP / ZERO on all three
+ * axes.  mapsm_op_set(CONV): (2r+1)^3 weights ordered (dz, dy, dx),
+ * one fmaf per tap in that order from +0.0f (reading v1).  The
+ * fused P2P exchange and deep halos are 2-D only.                           */
+mapsm_status mapsm_grid_create_3d(mapsm_ctx ctx, int64_t w, int64_t h, int64_t d, mapsm_dtype dtype,
+                                  mapsm_grid* out);
 
 /* Window(2D) pattern: radius and boundary.  Partitions the rows over
  * the slabs and allocates both buffers of every local slab with 2r halo rows
@@ -193,6 +256,34 @@ mapsm_status mapsm_gather(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, i
  * must be HISTOGRAM (else ESTATE).  Collective; synchronises.              */
 mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
 
+/* Chained task: a Reductive (Static) histogram task
+ * over the grid's CURRENT generation, as a second task on the same datum with
+ * a different access pattern (radius-0 Window in, ReductiveStatic out, Fig 4
+ * P:L359-403).  The task partitions the rows over `target_slabs` slabs (0 =
+ * the grid's own partition; k >= 1 = rows split evenly over k slabs, slab j
+ * on the device of global slab j, k <= total slabs), and the grid's Segment
+ * Location Monitor (Alg 2) infers which rows each target slab must receive
+ * and from where; rows already up to date on a target (its own slab, or a
+ * copy made by an earlier task on the unmodified datum) are not moved.
+ * Copies: peer cudaMemcpy (one process) or NCCL send/recv (multi-process).
+ * Bins (nbins must be 256, 64-bit counts, written on every process):
+ *   HISTOGRAM grids (u8): bin = pixel value (as mapsm_histogram);
+ *   Life grids: bin = cell state, so bins[0] = dead, bins[1] = alive cells;
+ *   F32 grids: bin = floor(v * 256) for 0 <= v < 1, v < 0 (and NaN) -> 0,
+ *              v >= 1 -> 255 (v * 256 is exact in fp32; DESIGN.md h4).
+ * `moved_bytes` (may be NULL) receives the bytes this process received for
+ * the task.  EINVAL: target_slabs out of range.  ESTATE: grid not bound.
+ * Collective; synchronises.                                                  */
+mapsm_status mapsm_task_histogram(mapsm_grid grid, int target_slabs, uint64_t* bins, int nbins,
+                                  int64_t* moved_bytes);
+
+/* GatherAsync (Table 2): like mapsm_gather but returns once the
+ * copies are enqueued; `ptr` is complete after mapsm_sync (Wait).  Use pinned
+ * host or device memory for a truly asynchronous copy (pageable memory makes
+ * the device-to-host step synchronous).  Do not iterate the grid before the
+ * mapsm_sync.  Collective.                                                   */
+mapsm_status mapsm_gather_async(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, int root);
+
 /* Copy only this process's own rows (same row range as mapsm_bind) to `ptr`;
  * not collective; synchronises.                                              */
 mapsm_status mapsm_read(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes);
@@ -214,6 +305,7 @@ typedef struct {
     int used_graphs;         /* 1 if iterate replays CUDA graphs */
     int gens_per_pass;       /* generations per compute pass (K with MAPSM_OPT_DEEP_HALO, else 1) */
     int64_t halo_rows;       /* halo rows allocated above/below each slab (r, or K*r) */
+    int64_t d;               /* planes of a Window(3D) grid, 0 for a 2-D grid */
 } mapsm_grid_info;
 
 mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);

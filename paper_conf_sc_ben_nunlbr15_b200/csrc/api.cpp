@@ -10,7 +10,9 @@
 //       host thread issuing to per-slab streams (local mode).
 //   Memory Analyzer + Allocator     -> mapsm_window_set (plan.cpp + cudaMalloc
 //       of both buffers with 2r halo rows each, once).
-//   Location Monitor + Alg 2        -> the static halo plan (plan.cpp).
+//   Location Monitor + Alg 2        -> the static halo plan (plan.cpp) on the
+//       iterated path; the general monitor (locmon.cpp) for chained tasks
+//       (mapsm_task_histogram) whose partition differs from the grid's.
 //   P2P copies      -> ncclSend/ncclRecv over NVLink (NCCL
 //       mode) or cudaMemcpyAsync peer copies (local mode).
 #include <cuda_runtime.h>
@@ -25,6 +27,7 @@
 
 #include "mapsm.h"
 #include "kernels.h"
+#include "locmon.h"
 #include "nccl.h"
 
 namespace mapsm {
@@ -174,6 +177,8 @@ enum GridState { ST_CREATED = 0, ST_WINDOW = 1, ST_OP = 2, ST_BOUND = 3 };
 struct mapsm_grid_s {
     mapsm_ctx ctx = nullptr;
     int64_t w = 0, h = 0;
+    int64_t d = 0;                  // planes of a Window(3D) grid (0 = 2-D grid)
+    int64_t rpitch = 0;             // device row pitch (== pitch for 2-D; pitch = h * rpitch for 3-D)
     mapsm_dtype dtype = MAPSM_U8;
     int r = 0;
     mapsm_boundary boundary = MAPSM_WRAP;
@@ -193,7 +198,22 @@ struct mapsm_grid_s {
     bool p2p_linked = false;    // peer pointers resolved
     int64_t opt_graph_iters = 16;
     bool used_graphs = false;
-    bool packed() const { return dtype == MAPSM_U8 && r == 1; }   // Life: bit-packed rows
+    // Segment Location Monitor of this datum (Alg 2) and the buffers of the
+    // last re-partitioned chained task (location kTaskLoc + j).
+    mapsm::LocationMonitor lm{2};
+    bool lm_dirty = true;       // the datum changed since the monitor last saw it
+    struct TaskBuf {
+        int device = 0;
+        int64_t y0 = 0, rows = 0;
+        char* ptr = nullptr;    // rows x pitch
+        unsigned long long* hist = nullptr;
+    };
+    int task_slabs = 0;         // target partition the task buffers belong to
+    std::vector<TaskBuf> tbufs;  // one per target slab this process owns
+    bool packed() const { return dtype == MAPSM_U8 && r == 1; }
+    // partition units: rows of a 2-D grid, planes of a 3-D grid (each unit is `pitch` bytes)
+    int64_t units() const { return d ? d : h; }
+    int64_t rows_per_unit() const { return d ? h : 1; }   // Life: bit-packed rows
 };
 
 static const size_t kMailboxBytes = 64;  // >= sizeof(tma::Mailbox)
@@ -322,6 +342,17 @@ extern "C" mapsm_status mapsm_grid_create(mapsm_ctx ctx, int64_t w, int64_t h, m
     return MAPSM_OK;
 }
 
+extern "C" mapsm_status mapsm_grid_create_3d(mapsm_ctx ctx, int64_t w, int64_t h, int64_t d, mapsm_dtype dtype,
+                                             mapsm_grid* out) {
+    if (!ctx || !out) return fail(MAPSM_EINVAL, "NULL argument");
+    *out = nullptr;
+    if (w < 1 || h < 1 || d < 1) return fail(MAPSM_EINVAL, "volume must be at least 1x1x1");
+    if (dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "Window(3D) grids are F32 (convolution)");
+    TRY(mapsm_grid_create(ctx, w, h, dtype, out));
+    (*out)->d = d;
+    return MAPSM_OK;
+}
+
 static void free_slab(Slab& s) {
     cudaSetDevice(s.device);
     for (int b = 0; b < 2; ++b)
@@ -367,9 +398,9 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
     // validate the partition for every slab before allocating anything
     for (int k = 0; k < c->g; ++k) {
         mapsm_slab_plan p;
-        if (compute_plan(g->h, c->g, (int)halo, boundary, k, &p) != MAPSM_OK)
+        if (compute_plan(g->units(), c->g, (int)halo, boundary, k, &p) != MAPSM_OK)
             return fail(MAPSM_EINVAL, "cannot split %lld rows over %d slabs with %lld halo rows (need >= that many rows each)",
-                        (long long)g->h, c->g, (long long)halo);
+                        (long long)g->units(), c->g, (long long)halo);
     }
     DeviceGuard dg;
     for (auto& s : g->slabs) free_slab(s);
@@ -380,7 +411,8 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
     g->boundary = boundary;
     const int64_t row_bytes = g->packed() ? (g->w + 31) / 32 * 4 : g->w * g->elem;
     const int64_t align = row_bytes >= 128 ? 128 : 16;
-    g->pitch = (row_bytes + align - 1) / align * align;
+    g->rpitch = (row_bytes + align - 1) / align * align;
+    g->pitch = g->rpitch * g->rows_per_unit();  // a unit = one row (2-D) or one plane of h rows (3-D)
     const int nloc = c->local ? c->g : 1;
     g->slabs.resize(nloc);
     for (int i = 0; i < nloc; ++i) {
@@ -389,17 +421,15 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
         s.device = c->devices[c->local ? i : 0];
         // the plan's kinds / neighbours / rows do not depend on the halo
         // depth; alloc_rows does (rows + 2 * halo)
-        compute_plan(g->h, c->g, (int)halo, boundary, s.rank, &s.plan);
+        compute_plan(g->units(), c->g, (int)halo, boundary, s.rank, &s.plan);
         CK(cudaSetDevice(s.device));
         CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
         const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
         const int nbuf = radius == 0 ? 1 : 2;  // a reductive (non-iterated) task needs no double buffer
         CK(cudaMalloc(&s.mailbox, kMailboxBytes));
         CK(cudaMemset(s.mailbox, 0, kMailboxBytes));
-        if (radius == 0) {
-            CK(cudaMalloc(&s.hist, 256 * sizeof(unsigned long long)));
-            g->device_bytes += 256 * sizeof(unsigned long long);
-        }
+        CK(cudaMalloc(&s.hist, 256 * sizeof(unsigned long long)));  // histogram / chained-task partials
+        g->device_bytes += 256 * sizeof(unsigned long long);
         for (int b = 0; b < nbuf; ++b) {
             cudaError_t e = cudaMalloc(&s.base[b], bytes);
             if (e != cudaSuccess) {
@@ -445,6 +475,9 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     if (g->dtype == MAPSM_U8) {
         if (radius != 1 && radius != 0)
             return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
+    } else if (g->d) {
+        if (radius < 1 || radius > 2)
+            return fail(MAPSM_EUNSUPPORTED, "Window(3D) conv radius must be 1..2, got %d", radius);
     } else {
         if (radius < 1 || radius > 8) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..8, got %d", radius);
     }
@@ -471,7 +504,7 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
         if (g->dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "conv needs dtype F32");
         if (!weights) return fail(MAPSM_EINVAL, "conv needs (2r+1)^2 weights");
         const int k = 2 * g->r + 1;
-        memcpy(g->wt, weights, sizeof(float) * k * k);
+        memcpy(g->wt, weights, sizeof(float) * k * k * (g->d ? k : 1));
     } else {
         return fail(MAPSM_EUNSUPPORTED, "op %d", (int)op);
     }
@@ -551,6 +584,8 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
     geom.top_map = rowmap_of(s.plan.top_kind);
     geom.bot_map = rowmap_of(s.plan.bottom_kind);
     geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+    geom.plane_rows = g->d ? g->h : 0;
+    geom.rpitch = g->rpitch;
     TimingPair* tp = nullptr;
     if (g->opt_timing && &s == &g->slabs[0]) {
         auto& vec = bulk ? s.t_bulk : s.t_bnd;
@@ -570,6 +605,8 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
                            s.num_sms, s.main);
     else if (g->op == MAPSM_OP_LIFE)
         e = launch_life_step(geom, bands, s.num_sms, s.main, link);
+    else if (g->d)
+        e = launch_conv3d(geom, bands, g->r, g->wt, s.num_sms, s.main);
     else
         e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main, link);
     if (e != cudaSuccess) return fail(MAPSM_ECUDA, "stencil launch: %s", cudaGetErrorString(e));
@@ -655,6 +692,7 @@ static bool p2p_eligible(const mapsm_grid_s* g) {
     if (g->op == MAPSM_OP_CONV && g->r > 4) return false;  // r = 5..8 run the shared-memory tile kernel
     if (g->op == MAPSM_OP_LIFE && (g->w % 128 != 0 || g->pitch % 16 != 0)) return false;
     if (g->op == MAPSM_OP_CONV && (g->w % 4 != 0 || g->pitch % 16 != 0)) return false;
+    if (g->d) return false;  // Window(3D): copy exchange only
     return g->h / g->ctx->g > 2 * (int64_t)g->r;
 }
 
@@ -720,7 +758,7 @@ static mapsm_status p2p_link(mapsm_grid_s* g) {
         s.up_base[1] = static_cast<char*>(p[1]);
         s.up_mail = static_cast<char*>(p[2]);
         mapsm_slab_plan up;
-        compute_plan(g->h, c->g, g->r, g->boundary, s.plan.up, &up);
+        compute_plan(g->units(), c->g, g->r, g->boundary, s.plan.up, &up);
         s.up_rows = up.rows;
     }
     if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
@@ -844,6 +882,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     if (n < 0) return fail(MAPSM_EINVAL, "n < 0");
     if (n == 0) return MAPSM_OK;
     if (g->op == MAPSM_OP_HISTOGRAM) return fail(MAPSM_EUNSUPPORTED, "a Reductive (histogram) grid is not iterated");
+    g->lm_dirty = true;  // a new version of the datum (Alg 2's lastOutput changes)
     DeviceGuard dg;
     const bool graphs = g->opt_graphs && !g->opt_timing && !g->ctx->local;
     // Deep halos: K generations per pass (one halo exchange of K*r rows per
@@ -1018,11 +1057,11 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
         CK(cudaSetDevice(s.device));
         for (int b = 0; b < 2; ++b)
             if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
-        const char* src = static_cast<const char*>(ptr) + (s.plan.y0 - y_first) * pitch;
+        const char* src = static_cast<const char*>(ptr) + (s.plan.y0 - y_first) * g->rows_per_unit() * pitch;
         const int64_t rows = s.plan.rows;
-        if (!g->packed()) {
-            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->pitch, src, pitch, g->w * g->elem, rows, cudaMemcpyDefault,
-                                 s.main));
+        if (!g->packed()) {  // planes of a 3-D slab are rows_per_unit contiguous device rows each
+            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->rpitch, src, pitch, g->w * g->elem, rows * g->rows_per_unit(),
+                                 cudaMemcpyDefault, s.main));
         } else if (on_dev && pdev == s.device) {
             CK(launch_pack_life(reinterpret_cast<const uint8_t*>(src), pitch, row_ptr(g, s, 0, 0), g->pitch, rows,
                                 g->w, s.main));
@@ -1048,6 +1087,7 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     g->gen = 0;
     g->launches = 0;
     g->exchanges = 0;
+    g->lm_dirty = true;
     g->state = ST_BOUND;
     if (g->opt_p2p) {
         if (!p2p_eligible(g))
@@ -1080,8 +1120,8 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
 static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitch, bool dst_on_dev) {
     const int64_t rows = s.plan.rows;
     if (!g->packed()) {
-        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->pitch, g->w * g->elem, rows, cudaMemcpyDefault,
-                             s.main));
+        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->rpitch, g->w * g->elem,
+                             rows * g->rows_per_unit(), cudaMemcpyDefault, s.main));
         return MAPSM_OK;
     }
     if (dst_on_dev) {
@@ -1103,7 +1143,7 @@ static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitc
     return MAPSM_OK;
 }
 
-extern "C" mapsm_status mapsm_read(mapsm_grid g, void* ptr, int64_t pitch) {
+static mapsm_status read_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, bool async) {
     if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
     if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "read before bind");
     if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch too small");
@@ -1113,44 +1153,48 @@ extern "C" mapsm_status mapsm_read(mapsm_grid g, void* ptr, int64_t pitch) {
     const int64_t y_first = g->slabs[0].plan.y0;
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
-        char* dst = static_cast<char*>(ptr) + (s.plan.y0 - y_first) * pitch;
+        char* dst = static_cast<char*>(ptr) + (s.plan.y0 - y_first) * g->rows_per_unit() * pitch;
         TRY(read_slab(g, s, dst, pitch, on_dev && pdev == s.device));
     }
-    return check_async(g);
+    return async ? MAPSM_OK : check_async(g);
 }
 
-extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int root) {
+extern "C" mapsm_status mapsm_read(mapsm_grid g, void* ptr, int64_t pitch) { return read_impl(g, ptr, pitch, false); }
+
+// Gather / GatherAsync (Table 2).  `async`: only enqueue (the caller
+// waits with mapsm_sync); the root's receive buffer is stream-ordered memory.
+static mapsm_status gather_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, int root, bool async) {
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
     if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "gather before bind");
     mapsm_ctx c = g->ctx;
     if (root < 0 || root >= c->world) return fail(MAPSM_EINVAL, "root %d", root);
     if (c->world == 1) {
         if (!ptr) return fail(MAPSM_EINVAL, "ptr is NULL");
-        return mapsm_read(g, ptr, pitch);
+        return read_impl(g, ptr, pitch, async);
     }
     if (c->rank == root && (!ptr || pitch < g->w * g->elem)) return fail(MAPSM_EINVAL, "root needs ptr and pitch");
     DeviceGuard dg;
     Slab& s = g->slabs[0];
     CK(cudaSetDevice(s.device));
-    TRY(check_async(g));
+    if (!async) TRY(check_async(g));
     const int64_t slab_bytes_row = g->pitch;
     if (c->rank != root) {
         NK(g_nccl.send(row_ptr(g, s, g->cur, 0), (size_t)(s.plan.rows * slab_bytes_row), ncclUint8, root, c->comm,
                        s.main));
-        return check_async(g);
+        return async ? MAPSM_OK : check_async(g);
     }
     int pdev = -1;
     const bool on_dev = is_device_ptr(ptr, &pdev) && pdev == s.device;
     // Root: receive each slab into a temporary buffer, then unpack / copy out.
     mapsm_slab_plan pk;
-    compute_plan(g->h, c->g, g->r, g->boundary, 0, &pk);
+    compute_plan(g->units(), c->g, g->r, g->boundary, 0, &pk);
     const int64_t max_rows = pk.rows;  // slab 0 is never shorter than any other
     char* tmp = nullptr;
-    CK(cudaMalloc(&tmp, (size_t)(max_rows * slab_bytes_row)));
+    CK(cudaMallocAsync(reinterpret_cast<void**>(&tmp), (size_t)(max_rows * slab_bytes_row), s.main));
     mapsm_status st = MAPSM_OK;
     for (int k = 0; k < c->world && st == MAPSM_OK; ++k) {
-        compute_plan(g->h, c->g, g->r, g->boundary, k, &pk);
-        char* dst = static_cast<char*>(ptr) + pk.y0 * pitch;
+        compute_plan(g->units(), c->g, g->r, g->boundary, k, &pk);
+        char* dst = static_cast<char*>(ptr) + pk.y0 * g->rows_per_unit() * pitch;
         if (k == root) {
             st = read_slab(g, s, dst, pitch, on_dev);
             continue;
@@ -1171,13 +1215,22 @@ extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int
         s.staging_bytes = view.staging_bytes;
         view.staging = nullptr;
         view.graph[0] = view.graph[1] = nullptr;
-        cudaError_t e = cudaStreamSynchronize(s.main);
-        if (e != cudaSuccess && st == MAPSM_OK) st = fail(MAPSM_ECUDA, "gather: %s", cudaGetErrorString(e));
+        if (!async) {
+            cudaError_t e = cudaStreamSynchronize(s.main);
+            if (e != cudaSuccess && st == MAPSM_OK) st = fail(MAPSM_ECUDA, "gather: %s", cudaGetErrorString(e));
+        }
     }
-    cudaStreamSynchronize(s.main);
-    cudaFree(tmp);
+    cudaFreeAsync(tmp, s.main);  // stream-ordered: after the last copy-out
     if (st != MAPSM_OK) return st;
-    return check_async(g);
+    return async ? MAPSM_OK : check_async(g);
+}
+
+extern "C" mapsm_status mapsm_gather(mapsm_grid g, void* ptr, int64_t pitch, int root) {
+    return gather_impl(g, ptr, pitch, root, false);
+}
+
+extern "C" mapsm_status mapsm_gather_async(mapsm_grid g, void* ptr, int64_t pitch, int root) {
+    return gather_impl(g, ptr, pitch, root, true);
 }
 
 // ---------------------------------------------------------------- histogram
@@ -1186,28 +1239,73 @@ extern "C" mapsm_status mapsm_histogram(mapsm_grid g, uint64_t* bins, int nbins)
     if (!g || !bins) return fail(MAPSM_EINVAL, "NULL argument");
     if (nbins != 256) return fail(MAPSM_EINVAL, "nbins must be 256");
     if (g->state < ST_BOUND || g->op != MAPSM_OP_HISTOGRAM) return fail(MAPSM_ESTATE, "histogram needs a bound HISTOGRAM grid");
-    DeviceGuard dg;
-    mapsm_ctx c = g->ctx;
-    // 1. per-slab partial histograms (shared-memory bins + one commit per CTA)
-    for (auto& s : g->slabs) {
-        CK(cudaSetDevice(s.device));
-        CK(launch_histogram(reinterpret_cast<const uint8_t*>(row_ptr(g, s, 0, 0)), g->pitch, g->w, s.plan.rows, s.hist,
-                            s.num_sms, s.main));
-        g->launches++;
-        CK(cudaEventRecord(s.ev_b, s.main));
+    // 1. per-slab partial histograms (shared-memory bins + one commit per CTA);
+    // 2. aggregation of the duplicated outputs: local slabs summed
+    //    on slab 0's device, then ncclAllReduce across processes.  This is the
+    //    chained task on the grid's own partition (no data moves).
+    return mapsm_task_histogram(g, 0, bins, nbins, nullptr);
+}
+
+static void free_task_bufs(mapsm_grid_s* g) {
+    for (auto& t : g->tbufs) {
+        cudaSetDevice(t.device);
+        if (t.ptr) cudaFree(t.ptr);
+        if (t.hist) cudaFree(t.hist);
     }
-    // 2. aggregate the duplicated outputs: local slabs summed on
-    //    slab 0's device, then across processes with ncclAllReduce.
+    g->tbufs.clear();
+    g->task_slabs = 0;
+}
+
+// ------------------------------------------------------------ chained tasks
+// a second task with a different access pattern over the
+// same datum (stencil -> histogram of its result), its data movement inferred
+// by the Segment Location Monitor (Alg 2) instead of hard-coded.
+
+static const int kTaskLoc = 1 << 20;  // monitor location of target slab j of a re-partitioned task: kTaskLoc + j
+
+static mapsm::Box rows_box(int64_t y0, int64_t rows, int64_t w) {
+    mapsm::Box b;
+    b.lo[0] = y0, b.hi[0] = y0 + rows;
+    b.lo[1] = 0, b.hi[1] = w;
+    b.lo[2] = 0, b.hi[2] = 1;
+    return b;
+}
+
+// Local slab index of global slab k in this process, -1 if another process owns it.
+static int local_of(const mapsm_grid_s* g, int k) {
+    const int i = k - g->ctx->first_slab;
+    return (i >= 0 && i < (int)g->slabs.size()) ? i : -1;
+}
+
+static mapsm_status launch_task_hist(mapsm_grid_s* g, const Slab& s, const char* rows0, int64_t rows,
+                                     unsigned long long* out, cudaStream_t st) {
+    if (g->op == MAPSM_OP_HISTOGRAM) {
+        CK(launch_histogram(reinterpret_cast<const uint8_t*>(rows0), g->pitch, g->w, rows, out, s.num_sms, st));
+    } else if (g->packed()) {
+        CK(launch_histogram_life(rows0, g->pitch, g->w, rows, out, s.num_sms, st));
+    } else {  // fp32: units of rows_per_unit rows each (3-D planes)
+        CK(launch_histogram_f32(reinterpret_cast<const float*>(rows0), g->rpitch, g->w, rows * g->rows_per_unit(), out,
+                                s.num_sms, st));
+    }
+    g->launches++;
+    return MAPSM_OK;
+}
+
+// Sum the partial histograms parts[i] (device of local slab owner[i]) into
+// slab 0's `hist`, all-reduce across processes, copy to `bins`.  Partials must
+// be complete on their owners' main streams (ev_b recorded by the caller).
+static mapsm_status aggregate_bins(mapsm_grid_s* g, const std::vector<const unsigned long long*>& parts,
+                                   const std::vector<int>& owner, uint64_t* bins) {
+    mapsm_ctx c = g->ctx;
     Slab& s0 = g->slabs[0];
     CK(cudaSetDevice(s0.device));
-    if (g->slabs.size() > 1) {
-        const int n = (int)g->slabs.size();
-        std::vector<const unsigned long long*> parts(n);
-        for (int k = 0; k < n; ++k) {
-            parts[k] = g->slabs[k].hist;
-            if (k) CK(cudaStreamWaitEvent(s0.main, g->slabs[k].ev_b, 0));
-        }
-        TRY(ensure_staging(s0, (int64_t)(n * sizeof(void*) + 256 * sizeof(unsigned long long))));
+    const int n = (int)parts.size();
+    for (int k = 0; k < n; ++k)
+        if (owner[k] != 0) CK(cudaStreamWaitEvent(s0.main, g->slabs[owner[k]].ev_b, 0));
+    if (n == 0) {
+        CK(cudaMemsetAsync(s0.hist, 0, 256 * sizeof(unsigned long long), s0.main));
+    } else if (n > 1 || parts[0] != s0.hist) {
+        TRY(ensure_staging(s0, (int64_t)(n * sizeof(void*) + 8 + 256 * sizeof(unsigned long long))));
         auto* dparts = static_cast<const unsigned long long**>(s0.staging);
         auto* sum = reinterpret_cast<unsigned long long*>(static_cast<char*>(s0.staging) + n * sizeof(void*) +
                                                           (8 - (n * sizeof(void*)) % 8) % 8);
@@ -1217,15 +1315,161 @@ extern "C" mapsm_status mapsm_histogram(mapsm_grid g, uint64_t* bins, int nbins)
         CK(cudaMemcpyAsync(s0.hist, sum, 256 * sizeof(unsigned long long), cudaMemcpyDeviceToDevice, s0.main));
         CK(cudaStreamSynchronize(s0.main));  // `parts` is host memory read by the async copy
     }
-    if (c->world > 1)
-        NK(g_nccl.allReduce(s0.hist, s0.hist, 256, ncclUint64, ncclSum, c->comm, s0.main));
+    if (c->world > 1) NK(g_nccl.allReduce(s0.hist, s0.hist, 256, ncclUint64, ncclSum, c->comm, s0.main));
     CK(cudaMemcpyAsync(bins, s0.hist, 256 * sizeof(unsigned long long), cudaMemcpyDefault, s0.main));
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_task_histogram(mapsm_grid g, int target_slabs, uint64_t* bins, int nbins,
+                                             int64_t* moved_bytes) {
+    if (!g || !bins) return fail(MAPSM_EINVAL, "NULL argument");
+    if (nbins != 256) return fail(MAPSM_EINVAL, "nbins must be 256");
+    if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "task before bind");
+    mapsm_ctx c = g->ctx;
+    const int G = c->g;
+    if (target_slabs < 0 || target_slabs > G)
+        return fail(MAPSM_EINVAL, "target_slabs %d (0..%d)", target_slabs, G);
+    // The even row split does not depend on the radius, so T == G is the grid's own partition.
+    const bool same = target_slabs == 0 || target_slabs == G;
+    const int T = same ? G : target_slabs;
+    DeviceGuard dg;
+    int64_t moved = 0;
+
+    // Allocator: buffers of a re-partitioned task (kept while T is unchanged,
+    // so a later task on the unmodified datum finds its rows up to date).
+    if (!same && g->task_slabs != T) {
+        free_task_bufs(g);
+        g->lm_dirty = true;  // forget up-to-date instances in the freed buffers
+        for (int j = 0; j < T; ++j) {
+            const int li = local_of(g, j);
+            if (li < 0) continue;
+            mapsm_slab_plan pj;
+            compute_plan(g->units(), T, 0, MAPSM_NO_CHECKS, j, &pj);
+            mapsm_grid_s::TaskBuf tb;
+            tb.device = g->slabs[li].device;
+            tb.y0 = pj.y0;
+            tb.rows = pj.rows;
+            CK(cudaSetDevice(tb.device));
+            g->tbufs.push_back(tb);  // pushed first so free_task_bufs releases it on failure
+            CK(cudaMalloc(&g->tbufs.back().hist, 256 * sizeof(unsigned long long)));
+            if (pj.rows > 0) CK(cudaMalloc(&g->tbufs.back().ptr, (size_t)(pj.rows * g->pitch)));
+        }
+        g->task_slabs = T;
+    }
+    // The monitor learns the datum's current version: slab k's owned rows at location k.
+    if (g->lm_dirty) {
+        std::vector<mapsm::LocEntry> segs;
+        for (int k = 0; k < G; ++k) {
+            mapsm_slab_plan pk;
+            compute_plan(g->units(), G, 0, MAPSM_NO_CHECKS, k, &pk);
+            segs.push_back({k, rows_box(pk.y0, pk.rows, g->w)});
+        }
+        g->lm.output(0, segs, false);
+        g->lm_dirty = false;
+    }
+    // Alg 2 for every target slab (every process evaluates all of them, so the
+    // monitors of all processes stay identical and send/recv pairs match).
+    std::vector<std::vector<mapsm::CopyOp>> ops(T);
+    std::vector<mapsm_slab_plan> tp(T);
+    for (int j = 0; j < T; ++j) {
+        compute_plan(g->units(), T, 0, MAPSM_NO_CHECKS, j, &tp[j]);
+        const int loc = same ? j : kTaskLoc + j;
+        mapsm_status st = g->lm.query(0, rows_box(tp[j].y0, tp[j].rows, g->w), loc, ops[j], nullptr);
+        if (st != MAPSM_OK) return fail(st, "location monitor query for target slab %d", j);
+    }
+    auto tbuf_of = [&](int j) -> mapsm_grid_s::TaskBuf* {
+        for (auto& t : g->tbufs)
+            if (t.y0 == tp[j].y0 && t.rows == tp[j].rows && local_of(g, j) >= 0) return &t;
+        return nullptr;
+    };
+    // Copies (P2P copy commands of Alg 1 line 13): the producer slab's stream
+    // has the current generation; each target's stream waits for it.
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaEventRecord(s.ev_b, s.main));
+    }
+    bool any_remote = false;
+    for (int j = 0; j < T; ++j) {
+        const int lj = local_of(g, j);
+        for (const auto& op : ops[j]) {
+            const int lk = local_of(g, op.src);
+            const int64_t nr = op.box.hi[0] - op.box.lo[0];
+            if (lj >= 0 && lk >= 0) {
+                Slab& dst = g->slabs[lj];
+                Slab& src = g->slabs[lk];
+                mapsm_grid_s::TaskBuf* tb = tbuf_of(j);
+                if (!tb) return fail(MAPSM_ESTATE, "no task buffer for target slab %d", j);
+                CK(cudaSetDevice(dst.device));
+                CK(cudaStreamWaitEvent(dst.main, src.ev_b, 0));
+                CK(cudaMemcpyAsync(tb->ptr + (op.box.lo[0] - tb->y0) * g->pitch,
+                                   row_ptr(g, src, g->cur, op.box.lo[0] - src.plan.y0), (size_t)(nr * g->pitch),
+                                   cudaMemcpyDefault, dst.main));
+                moved += nr * g->pitch;
+            } else if (lj >= 0 || lk >= 0) {
+                any_remote = true;
+            }
+        }
+    }
+    if (any_remote) {  // multi-process: one slab per process, NCCL point-to-point in one group
+        Slab& s = g->slabs[0];
+        CK(cudaSetDevice(s.device));
+        NK(g_nccl.groupStart());
+        for (int j = 0; j < T; ++j) {
+            const int lj = local_of(g, j);
+            for (const auto& op : ops[j]) {
+                const int lk = local_of(g, op.src);
+                if ((lj >= 0) == (lk >= 0)) continue;
+                const int64_t nr = op.box.hi[0] - op.box.lo[0];
+                const size_t bytes = (size_t)(nr * g->pitch);
+                if (lk >= 0) {
+                    NK(g_nccl.send(row_ptr(g, s, g->cur, op.box.lo[0] - s.plan.y0), bytes, ncclUint8, j, c->comm,
+                                   s.main));
+                } else {
+                    mapsm_grid_s::TaskBuf* tb = tbuf_of(j);
+                    if (!tb) {
+                        g_nccl.groupEnd();
+                        return fail(MAPSM_ESTATE, "no task buffer for target slab %d", j);
+                    }
+                    NK(g_nccl.recv(tb->ptr + (op.box.lo[0] - tb->y0) * g->pitch, bytes, ncclUint8, op.src, c->comm,
+                                   s.main));
+                    moved += (int64_t)bytes;
+                    g->exchanges++;
+                }
+            }
+        }
+        NK(g_nccl.groupEnd());
+    }
+    for (int j = 0; j < T; ++j) g->lm.copied(0, ops[j]);
+
+    // The Reductive-Static task itself, per local target slab, then aggregation.
+    std::vector<const unsigned long long*> parts;
+    std::vector<int> owner;
+    for (int j = 0; j < T; ++j) {
+        const int lj = local_of(g, j);
+        if (lj < 0) continue;
+        Slab& s = g->slabs[lj];
+        CK(cudaSetDevice(s.device));
+        if (same) {
+            TRY(launch_task_hist(g, s, row_ptr(g, s, g->cur, 0), s.plan.rows, s.hist, s.main));
+            parts.push_back(s.hist);
+        } else {
+            mapsm_grid_s::TaskBuf* tb = tbuf_of(j);
+            if (!tb) return fail(MAPSM_ESTATE, "no task buffer for target slab %d", j);
+            TRY(launch_task_hist(g, s, tb->ptr, tb->rows, tb->hist, s.main));
+            parts.push_back(tb->hist);
+        }
+        owner.push_back(lj);
+        CK(cudaEventRecord(s.ev_b, s.main));
+    }
+    TRY(aggregate_bins(g, parts, owner, bins));
+    if (moved_bytes) *moved_bytes = moved;
     return check_async(g);
 }
 
 extern "C" mapsm_status mapsm_grid_destroy(mapsm_grid g) {
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
     DeviceGuard dg;
+    free_task_bufs(g);
     for (auto& s : g->slabs) {
         cudaSetDevice(s.device);
         cudaStreamSynchronize(s.main);
@@ -1243,6 +1487,7 @@ extern "C" mapsm_status mapsm_get_info(mapsm_grid g, mapsm_grid_info* o) {
     if (!g || !o) return fail(MAPSM_EINVAL, "NULL argument");
     o->w = g->w;
     o->h = g->h;
+    o->d = g->d;
     o->dtype = g->dtype;
     o->op = g->op;
     o->radius = g->r;

@@ -26,6 +26,9 @@ struct StencilGeom {
     int64_t rows;    // owned rows of the slab
     int64_t w;       // columns (cells)
     int top_map, bot_map, col_mode;
+    // Window(3D) grids: `rows` counts planes, `pitch` is the plane pitch, and a
+    // plane holds plane_rows rows of rpitch bytes (0 for 2-D grids)
+    int64_t plane_rows = 0, rpitch = 0;
 };
 
 // Output-row bands computed by one launch (1 band = all rows or interior;
@@ -75,12 +78,24 @@ cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst,
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
                              int num_sms, cudaStream_t s, const FusedLink* link = nullptr);
 
+// Window(3D) fp32 convolution (conv3d.cu), radius 1..2, (2r+1)^3 weights
+// ordered (dz, dy, dx); bands are plane ranges; col_mode is the y/x boundary.
+cudaError_t launch_conv3d(const StencilGeom& g, const RowBands& b, int r, const float* weights, int num_sms,
+                          cudaStream_t s);
+
 cudaError_t launch_conv_wide(const StencilGeom& g, const RowBands& b, int r, const float* weights, cudaStream_t s);
 
 // Reductive (Static) output: 256-bin histogram of a u8 slab into out[256]
 // (zeroed here; 64-bit counts); and the sum of g partial histograms.
 cudaError_t launch_histogram(const uint8_t* img, int64_t pitch, int64_t w, int64_t rows, unsigned long long* out,
                              int num_sms, cudaStream_t s);
+// Chained histogram tasks over stencil grids (api.cpp mapsm_task_histogram):
+// Life (bit-packed rows; bins 0 = dead, 1 = alive) and fp32 (bin =
+// floor(v * 256) clamped).  `out` is zeroed here.
+cudaError_t launch_histogram_life(const void* bits, int64_t pitch, int64_t w, int64_t rows, unsigned long long* out,
+                                  int num_sms, cudaStream_t s);
+cudaError_t launch_histogram_f32(const float* img, int64_t pitch, int64_t w, int64_t rows, unsigned long long* out,
+                                 int num_sms, cudaStream_t s);
 cudaError_t launch_histogram_sum(const unsigned long long* const* parts_dev, int g, unsigned long long* out,
                                  cudaStream_t s);
 

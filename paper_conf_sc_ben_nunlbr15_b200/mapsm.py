@@ -33,8 +33,11 @@ EXPORTED = [
     "mapsm_nccl_unique_id", "mapsm_grid_create", "mapsm_window_set", "mapsm_op_set", "mapsm_grid_slab",
     "mapsm_bind", "mapsm_iterate", "mapsm_sync", "mapsm_gather", "mapsm_read", "mapsm_histogram", "mapsm_grid_destroy",
     "mapsm_get_info", "mapsm_set_option", "mapsm_get_timing", "mapsm_grid_stream", "mapsm_status_string",
-    "mapsm_last_error", "mapsm_version",
+    "mapsm_last_error", "mapsm_version", "mapsm_locmon_create", "mapsm_locmon_destroy", "mapsm_locmon_output",
+    "mapsm_locmon_query", "mapsm_locmon_copied", "mapsm_task_histogram", "mapsm_gather_async",
+    "mapsm_grid_create_3d",
 ]
+MAX_DIMS = 3
 
 
 class MapsmError(RuntimeError):
@@ -55,7 +58,16 @@ class mapsm_grid_info(ctypes.Structure):
                 ("radius", ctypes.c_int), ("boundary", ctypes.c_int), ("world", ctypes.c_int),
                 ("local_slabs", ctypes.c_int), ("pitch_bytes", ctypes.c_int64), ("generation", ctypes.c_int64),
                 ("launches", ctypes.c_int64), ("exchanges", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
-                ("used_graphs", ctypes.c_int), ("gens_per_pass", ctypes.c_int), ("halo_rows", ctypes.c_int64)]
+                ("used_graphs", ctypes.c_int), ("gens_per_pass", ctypes.c_int), ("halo_rows", ctypes.c_int64),
+                ("d", ctypes.c_int64)]
+
+
+class mapsm_box(ctypes.Structure):
+    _fields_ = [("lo", ctypes.c_int64 * MAX_DIMS), ("hi", ctypes.c_int64 * MAX_DIMS)]
+
+
+class mapsm_copy_op(ctypes.Structure):
+    _fields_ = [("src", ctypes.c_int), ("dst", ctypes.c_int), ("box", mapsm_box)]
 
 
 _lib = None
@@ -92,6 +104,14 @@ def lib() -> ctypes.CDLL:
         "mapsm_set_option": [vp, ci, i64],
         "mapsm_get_timing": [vp, P(ctypes.c_double), P(i64), P(ctypes.c_double), P(i64)],
         "mapsm_grid_stream": [vp, ci, P(vp)],
+        "mapsm_locmon_create": [ci, P(vp)],
+        "mapsm_locmon_destroy": [vp],
+        "mapsm_locmon_output": [vp, ci, ci, P(ci), P(mapsm_box), ci],
+        "mapsm_locmon_query": [vp, ci, P(mapsm_box), ci, P(mapsm_copy_op), ci, P(ci), P(ci)],
+        "mapsm_locmon_copied": [vp, ci, ci, P(mapsm_copy_op)],
+        "mapsm_task_histogram": [vp, ci, vp, ci, P(i64)],
+        "mapsm_gather_async": [vp, vp, i64, ci],
+        "mapsm_grid_create_3d": [vp, i64, i64, i64, ci, P(vp)],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -171,6 +191,12 @@ def mapsm_grid_create(ctx: int, w: int, h: int, dtype: int) -> int:
     return out.value
 
 
+def mapsm_grid_create_3d(ctx: int, w: int, h: int, d: int, dtype: int = F32) -> int:
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_grid_create_3d(ctx, w, h, d, dtype, ctypes.byref(out)), "mapsm_grid_create_3d")
+    return out.value
+
+
 def mapsm_window_set(grid: int, radius: int, boundary: int) -> None:
     _check(lib().mapsm_window_set(grid, radius, boundary), "mapsm_window_set")
 
@@ -209,6 +235,13 @@ def mapsm_gather(grid: int, buf, row_pitch_bytes: int | None = None, root: int =
     _check(lib().mapsm_gather(grid, p, pitch, root), "mapsm_gather")
 
 
+def mapsm_gather_async(grid: int, buf, row_pitch_bytes: int | None = None, root: int = 0) -> None:
+    """GatherAsync: enqueue only; `buf` is complete after mapsm_sync."""
+    p = None if buf is None else _ptr(buf)
+    pitch = row_pitch_bytes or (0 if buf is None else _pitch(buf, 0))
+    _check(lib().mapsm_gather_async(grid, p, pitch, root), "mapsm_gather_async")
+
+
 def mapsm_read(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
     _check(lib().mapsm_read(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read")
 
@@ -219,6 +252,73 @@ def mapsm_histogram(grid: int, bins=None) -> np.ndarray:
     out = np.zeros(256, dtype=np.uint64) if bins is None else bins
     _check(lib().mapsm_histogram(grid, _ptr(out), 256), "mapsm_histogram")
     return out
+
+
+def mapsm_task_histogram(grid: int, target_slabs: int = 0, bins=None) -> tuple[np.ndarray, int]:
+    """Chained Reductive-Static task over the grid's current generation with
+    its own partition (0 = the grid's); returns (bins, bytes moved here)."""
+    out = np.zeros(256, dtype=np.uint64) if bins is None else bins
+    moved = ctypes.c_int64()
+    _check(lib().mapsm_task_histogram(grid, target_slabs, _ptr(out), 256, ctypes.byref(moved)),
+           "mapsm_task_histogram")
+    return out, moved.value
+
+
+# Segment Location Monitor (Alg 2).  Boxes are given as sequences of (lo, hi)
+# pairs, one per dimension (missing dimensions are [0, 1)).
+
+def _box(b) -> mapsm_box:
+    x = mapsm_box()
+    for d in range(MAX_DIMS):
+        lo, hi = (b[d] if d < len(b) else (0, 1))
+        x.lo[d], x.hi[d] = lo, hi
+    return x
+
+
+def _unbox(x: mapsm_box, nd: int) -> tuple:
+    return tuple((x.lo[d], x.hi[d]) for d in range(nd))
+
+
+def mapsm_locmon_create(ndims: int) -> int:
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_locmon_create(ndims, ctypes.byref(out)), "mapsm_locmon_create")
+    return out.value
+
+
+def mapsm_locmon_destroy(m: int) -> None:
+    _check(lib().mapsm_locmon_destroy(m), "mapsm_locmon_destroy")
+
+
+def mapsm_locmon_output(m: int, datum: int, segs, needs_aggregation: bool = False) -> None:
+    """segs: [(location, box), ...]"""
+    n = len(segs)
+    locs = (ctypes.c_int * max(n, 1))(*[l for l, _ in segs])
+    boxes = (mapsm_box * max(n, 1))(*[_box(b) for _, b in segs])
+    _check(lib().mapsm_locmon_output(m, datum, n, locs, boxes, int(needs_aggregation)), "mapsm_locmon_output")
+
+
+def mapsm_locmon_query(m: int, datum: int, required, target: int, nd: int = 2) -> tuple[list, bool]:
+    """Alg 2: ([(src, dst, box), ...], needs_aggregation)."""
+    req = _box(required)
+    n, agg = ctypes.c_int(), ctypes.c_int()
+    cap = 16
+    while True:
+        ops = (mapsm_copy_op * cap)()
+        st = lib().mapsm_locmon_query(m, datum, ctypes.byref(req), target, ops, cap, ctypes.byref(n),
+                                      ctypes.byref(agg))
+        if st == ENOMEM and n.value > cap:
+            cap = n.value
+            continue
+        _check(st, "mapsm_locmon_query")
+        return [(ops[i].src, ops[i].dst, _unbox(ops[i].box, nd)) for i in range(n.value)], bool(agg.value)
+
+
+def mapsm_locmon_copied(m: int, datum: int, ops) -> None:
+    n = len(ops)
+    arr = (mapsm_copy_op * max(n, 1))()
+    for i, (src, dst, b) in enumerate(ops):
+        arr[i].src, arr[i].dst, arr[i].box = src, dst, _box(b)
+    _check(lib().mapsm_locmon_copied(m, datum, n, arr), "mapsm_locmon_copied")
 
 
 def mapsm_grid_destroy(grid: int) -> None:
@@ -260,13 +360,15 @@ class Grid:
     bind -> iterate -> gather, as in Fig 2a."""
 
     def __init__(self, ctx: int, w: int, h: int, op: str = "life", radius: int = 1, boundary: str = "wrap",
-                 weights=None, deep_halo: int = 1):
-        self.ctx, self.w, self.h = ctx, w, h
+                 weights=None, deep_halo: int = 1, d: int = 0):
+        """d > 0: a Window(3D) d x h x w fp32 volume (op "conv", (2r+1)^3 weights)."""
+        self.ctx, self.w, self.h, self.d = ctx, w, h, d
         self.op = op
         self.dtype = F32 if op == "conv" else U8
         if op == "histogram":
             radius, boundary = 0, "no_checks"
-        self.handle = mapsm_grid_create(ctx, w, h, self.dtype)
+        self.handle = (mapsm_grid_create_3d(ctx, w, h, d, self.dtype) if d else
+                       mapsm_grid_create(ctx, w, h, self.dtype))
         try:
             mapsm_window_set(self.handle, radius, BOUNDARY[boundary] if isinstance(boundary, str) else boundary)
             if deep_halo > 1:
@@ -289,7 +391,7 @@ class Grid:
         return y0, ylast + rlast - y0
 
     def bind(self, buf, pitch: int | None = None):
-        mapsm_bind(self.handle, buf, pitch)
+        mapsm_bind(self.handle, buf, pitch or self._rp(buf))
 
     def iterate(self, n: int):
         mapsm_iterate(self.handle, n)
@@ -300,18 +402,33 @@ class Grid:
     def read(self, out=None):
         y0, rows = self.local_rows()
         if out is None:
-            out = np.empty((rows, self.w), dtype=np.uint8 if self.dtype == U8 else np.float32)
-        mapsm_read(self.handle, out)
+            shape = (rows, self.h, self.w) if self.d else (rows, self.w)
+            out = np.empty(shape, dtype=np.uint8 if self.dtype == U8 else np.float32)
+        mapsm_read(self.handle, out, self._rp(out))
         return out
+
+    def _rp(self, buf):
+        """Row pitch of a (planes, h, w) volume buffer (None = the binding's default for 2-D)."""
+        if not self.d or buf is None:
+            return None
+        return buf.strides[1] if isinstance(buf, np.ndarray) else buf.stride(1) * buf.element_size()
 
     def gather(self, out=None, root: int = 0, rank: int = 0):
         if out is None and rank == root:
-            out = np.empty((self.h, self.w), dtype=np.uint8 if self.dtype == U8 else np.float32)
-        mapsm_gather(self.handle, out, None, root)
+            shape = (self.d, self.h, self.w) if self.d else (self.h, self.w)
+            out = np.empty(shape, dtype=np.uint8 if self.dtype == U8 else np.float32)
+        mapsm_gather(self.handle, out, self._rp(out), root)
         return out
 
     def histogram(self, bins=None):
         return mapsm_histogram(self.handle, bins)
+
+    def task_histogram(self, target_slabs: int = 0, bins=None):
+        return mapsm_task_histogram(self.handle, target_slabs, bins)
+
+    def gather_async(self, out, root: int = 0):
+        mapsm_gather_async(self.handle, out, self._rp(out), root)
+        return out
 
     def info(self) -> mapsm_grid_info:
         return mapsm_get_info(self.handle)

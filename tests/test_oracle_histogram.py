@@ -52,3 +52,28 @@ def test_generators():
     hu, hs = oracle.histogram(u), oracle.histogram(s)
     assert hu.min() > 0 and hu.max() < 3 * hu.mean()
     assert hs.argmax() in range(100, 156) and hs[:30].sum() < 0.01 * hs.sum() and hs.max() > 2 * hu.max()
+
+
+# ---- fp32-field histogram task (reading h4) ----
+
+def test_f32_histogram_closed_forms():
+    """bin = floor(v * 256) on [0, 1): every bin edge k/256 lands in bin k,
+    the float just below it in bin k-1; < 0, -0.0 and NaN -> 0; >= 1 -> 255."""
+    k = np.arange(256)
+    edges = (k / 256).astype(np.float32)[None, :]
+    out = oracle.histogram_f32(edges)
+    assert np.array_equal(out, np.ones(256, np.uint64))
+    below = np.nextafter(edges[:, 1:], np.float32(-1))
+    out = oracle.histogram_f32(below)
+    assert np.array_equal(out[:255], np.ones(255, np.uint64)) and out[255] == 0
+    special = np.array([[-1.0, -0.0, np.nan, -np.inf, 1.0, 7.5, np.inf, 0.99999994]], np.float32)
+    out = oracle.histogram_f32(special)
+    assert out[0] == 4 and out[255] == 4 and out.sum() == 8
+
+
+def test_f32_histogram_vs_numpy_binning():
+    """Against numpy's floor/clip on a random field in [-0.1, 1.1)."""
+    rng = np.random.default_rng(5)
+    f = (rng.random((37, 101)) * 1.2 - 0.1).astype(np.float32)
+    b = np.clip(np.floor(f.astype(np.float64) * 256), 0, 255).astype(np.int64)
+    assert np.array_equal(oracle.histogram_f32(f), np.bincount(b.ravel(), minlength=256).astype(np.uint64))
