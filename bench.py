@@ -57,6 +57,14 @@ WORKLOADS = {
                   scaling="weak", bcell=8.0,
                   label="fp32 9x9 (r=4) window stencil, 32768 wide x 4096 rows per GPU, ZERO, 100 iterations per "
                         "step (BASELINE configs[4], weak scaling)"),
+    "conv3d": dict(op="conv", w=512, h=512, d=512, r=1, b="zero", n=100, seed=0x5EED0007, wseed=0x5EED0077,
+                   scaling="strong", bcell=8.0,
+                   label="fp32 3x3x3 Window(3D) convolution 512x512x512 ZERO, 100 iterations per step (SURVEY "
+                         "§8(f) NEXT-2; plane-slab partition; not a BASELINE config)"),
+    "conv3d5": dict(op="conv", w=512, h=512, d=512, r=2, b="clamp", n=20, seed=0x5EED0007, wseed=0x5EED0078,
+                    scaling="strong", bcell=8.0,
+                    label="fp32 5x5x5 Window(3D) convolution 512x512x512 CLAMP, 20 iterations per step (SURVEY "
+                          "§8(f) NEXT-2; FMA-bound; not a BASELINE config)"),
     "hist8k": dict(op="histogram", w=8192, h=8192, r=0, b="no_checks", n=1, seed=0x5EED0006, wseed=None,
                    scaling="strong", bcell=1.0,
                    label="256-bin histogram of an 8192x8192 u8 image, uniform pixels (seed 0x5EED0006), one "
@@ -145,6 +153,11 @@ def _oracle_sample(wl):
         rows = 512
         g0 = mi.life_u8(wl["seed"], w, rows)
         return (lambda k: oracle.life(g0, k, wl["b"])), w * rows, f"{w} x {rows} rows"
+    if wl["op"] == "conv" and wl.get("d"):
+        planes = 8
+        v0 = mi.volume_f32(wl["seed"], w, wl["h"], planes)
+        W = mi.weights3d_f32(wl["wseed"], wl["r"])
+        return (lambda k: oracle.conv3d(v0, W, k, wl["b"])), w * wl["h"] * planes, f"{planes} planes of {wl['h']} x {w}"
     if wl["op"] == "conv":
         rows = 256
         g0 = mi.field_f32(wl["seed"], w, rows)
@@ -263,15 +276,23 @@ def main():
     w = wl["w"]
     h = wl["h"] * (world if wl["scaling"] == "weak" else 1)
     n = wl["n"]
-    W = mi.weights_f32(wl["wseed"], wl["r"]) if op == "conv" else None
-    grid = M.Grid(ctx, w, h, op, wl["r"], wl["b"], W)
+    d = wl.get("d", 0)   # Window(3D): partition units are planes of h rows
+    if op == "conv":
+        W = mi.weights3d_f32(wl["wseed"], wl["r"]) if d else mi.weights_f32(wl["wseed"], wl["r"])
+    else:
+        W = None
+    grid = M.Grid(ctx, w, h, op, wl["r"], wl["b"], W, d=d)
+    cpu_ = w * (h if d else 1)             # cells per partition unit (row or plane)
+    cells_total = w * h * (d if d else 1)
     if args.graph_iters:
         grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
     y0, rows = grid.local_rows()
     host_dtype = torch.float32 if op == "conv" else torch.uint8
     # pinned host rows of this rank (input and result buffers for e2e)
-    h_in = torch.empty((rows, w), dtype=host_dtype, pin_memory=True)
-    if op == "life":
+    h_in = torch.empty((rows, h, w) if d else (rows, w), dtype=host_dtype, pin_memory=True)
+    if d:
+        h_in.numpy()[:] = mi.volume_f32(wl["seed"], w, h, rows, z0=y0)
+    elif op == "life":
         mi.life_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
     elif op == "conv":
         mi.field_f32(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
@@ -326,19 +347,20 @@ def main():
         dist.all_reduce(tl, op=dist.ReduceOp.SUM)
     total_ms = float(t.item())
     total_launches = int(tl.item())
-    units_per_step = w * h * n
+    units_per_step = cells_total * n
     value = units_per_step * args.steps / (total_ms / 1e3)
     ms_per_step = total_ms / args.steps
 
     peak_gbs, peak_src = load_peaks()
     bcell = wl["bcell"]
-    slab_cells = rows * w
+    slab_cells = rows * cpu_
     # achieved over the timed region: each stencil step is n back-to-back bulk
     # launches (N == 1), the histogram step one launch (plus its aggregation)
     bulk_launches_per_step = n if op != "histogram" else 1
     per_launch_s = (total_ms / 1e3) / (args.steps * bulk_launches_per_step)
     achieved_region = bcell * slab_cells / per_launch_s / 1e9
-    kernel = {"life": "life_tma_kernel", "conv": "conv_tma_kernel", "histogram": "histogram_kernel"}[op]
+    kernel = {"life": "life_tma_kernel", "conv": "conv3d_kernel" if d else "conv_tma_kernel",
+              "histogram": "histogram_kernel"}[op]
     roofline = {"bound": "hbm", "peak": peak_gbs, "unit": "GB/s", "kernel": kernel,
                 "bytes_per_unit": bcell, "algorithmic_bytes_per_launch": bcell * slab_cells, "peak_source": peak_src}
     per_kernel_s = None
@@ -351,7 +373,7 @@ def main():
         grid.set_option(M.OPT_TIMING, 0)
         bulk_rows = rows if bnd_n == 0 else rows - 2 * wl["r"]
         per_kernel_s = (bulk_ms / 1e3) / max(1, bulk_n)
-        achieved_kernel = bcell * bulk_rows * w / per_kernel_s / 1e9
+        achieved_kernel = bcell * bulk_rows * cpu_ / per_kernel_s / 1e9
         roofline["achieved_events_per_launch_GBps"] = achieved_kernel
         roofline["kernel_ms_per_launch"] = per_kernel_s * 1e3
         achieved = achieved_region if world == 1 else achieved_kernel
@@ -370,12 +392,12 @@ def main():
         except Exception:
             pass
     if op == "conv":
-        fma_per_cell = (2 * wl["r"] + 1) ** 2
+        fma_per_cell = (2 * wl["r"] + 1) ** (3 if d else 2)
         sm_mhz = clocks.get("sm_mhz") or 1965.0
         fma_peak = 148 * 128 * sm_mhz * 1e6
-        roofline["fma_frac_at_sampled_clock"] = (bulk_rows * w * fma_per_cell / per_kernel_s) / fma_peak
-        if wl["r"] >= 3:
-            roofline["note"] = "9x9 is FP32-FMA bound (20.25 FMA/B): fma_frac is the binding fraction"
+        roofline["fma_frac_at_sampled_clock"] = (bulk_rows * cpu_ * fma_per_cell / per_kernel_s) / fma_peak
+        if fma_per_cell / 8.0 > 5.7:   # above the FMA/HBM balance (37.2 TFMA/s / 6.5 TB/s)
+            roofline["note"] = (f"FP32-FMA bound ({fma_per_cell / 8.0:.2f} FMA/B): fma_frac is the binding fraction")
 
     # halo-exchange exposure (N > 1): same steps without the exchange
     exposure = None
@@ -408,7 +430,7 @@ def main():
             M.mapsm_histogram(grid.handle, h_bins)
         else:
             grid.iterate(n)
-            M.mapsm_read(grid.handle, h_out)
+            M.mapsm_read(grid.handle, h_out, grid._rp(h_out))
         e1.record(stream)
         e1.synchronize()
         e2e_ms += e0.elapsed_time(e1)
@@ -417,8 +439,8 @@ def main():
         dist.all_reduce(te, op=dist.ReduceOp.MAX)
     e2e_value = units_per_step * args.e2e_steps / (float(te.item()) / 1e3)
     elem = 4 if op == "conv" else 1
-    h2d = h * w * elem
-    d2h = 256 * 8 * world if op == "histogram" else h * w * elem
+    h2d = cells_total * elem
+    d2h = 256 * 8 * world if op == "histogram" else cells_total * elem
 
     # Chained task: a Reductive-Static histogram task over
     # the current generation, its data movement inferred by the Segment Location
@@ -443,9 +465,9 @@ def main():
             dist.all_reduce(tc, op=dist.ReduceOp.MAX)
         c_s = float(tc.item()) / 1e3 / args.steps
         tb = 0.125 if op == "life" else 4.0   # bytes read per cell (1 bit / one fp32)
-        ach = tb * rows * w / c_s / 1e9
+        ach = tb * rows * cpu_ / c_s / 1e9
         chained = {"task": "histogram of the current generation (mapsm_task_histogram, grid's own partition)",
-                   "moved_bytes": int(moved), "ms_per_call": c_s * 1e3, "cells_per_s": h * w / c_s,
+                   "moved_bytes": int(moved), "ms_per_call": c_s * 1e3, "cells_per_s": cells_total / c_s,
                    "roofline": {"bound": "hbm", "kernel": "histogram_life_kernel" if op == "life"
                                 else "histogram_f32_kernel", "bytes_per_unit": tb, "achieved": ach,
                                 "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
@@ -524,7 +546,8 @@ def main():
             "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
             "scaling": wl["scaling"], "vs_baseline": None, "dtype": dtype, "data": "synthetic",
-            "config": {"workload": wl["label"], "w": w, "h": h, "iterations_per_step": n, "radius": wl["r"],
+            "config": {"workload": wl["label"], "w": w, "h": h, **({"d": d} if d else {}),
+                       "iterations_per_step": n, "radius": wl["r"],
                        "boundary": wl["b"], "parallelism": para,
                        "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU working set "
                              f"{ws_mib:.0f} MiB vs 126 MB L2",

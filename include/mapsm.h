@@ -284,6 +284,74 @@ mapsm_status mapsm_task_histogram(mapsm_grid grid, int target_slabs, uint64_t* b
  * mapsm_sync.  Collective.                                                   */
 mapsm_status mapsm_gather_async(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, int root);
 
+/* ------------------------------------------------- unmodified GPU routines
+ * SURVEY §8(f) NEXT-4; §4.6 ("the scheduler calls the host-level
+ * wrapper functions for each GPU with the device ID, stream, buffer pointers
+ * and their corresponding memory segments"), §5.4.
+ * A matrix datum is a rows x cols fp32 row-major matrix.  A task splits
+ * `task_rows` evenly over the slabs and gives every parameter an
+ * access pattern (Table 1):
+ *   MAPSM_PAT_BLOCK2D    input, the slab's row block (rows == task_rows)
+ *   MAPSM_PAT_BLOCK2D_T  input, the whole matrix (Block (2D-Transposed): a row
+ *                        block of the output needs every column of every row)
+ *   MAPSM_PAT_OUT_SI     output, Structured Injective row block (write only)
+ *   MAPSM_PAT_INOUT_SI   input row block that is also the output row block
+ * The matrix's Segment Location Monitor (Alg 2) infers the copies each slab
+ * needs (segments already up to date are not moved, so chains of calls on
+ * unchanged inputs move nothing — the paper's point against CUBLAS-XT,
+ * P:L497); then `routine` runs once per local slab on the slab's stream and
+ * must only enqueue work on that stream.  Outputs become the datums' new
+ * versions (row blocks on their slabs).  Asynchronous: mapsm_matrix_sync /
+ * mapsm_matrix_gather wait.  Collective in multi-process mode.            */
+#define MAPSM_MAX_PARAMS 8
+typedef enum {
+    MAPSM_PAT_BLOCK2D = 0,
+    MAPSM_PAT_BLOCK2D_T = 1,
+    MAPSM_PAT_OUT_SI = 2,
+    MAPSM_PAT_INOUT_SI = 3
+} mapsm_pattern;
+typedef struct mapsm_matrix_s* mapsm_matrix;
+/* One parameter's segment on the slab's device: rows [row0, row0+rows) of
+ * the datum, `cols` columns, leading dimension `ld` (floats), `ptr` = element
+ * (row0, 0) in device memory.                                               */
+typedef struct {
+    int64_t row0, rows, cols, ld;
+    float* ptr;
+} mapsm_segment;
+/* The wrapper prototype (Fig 5): returns 0 on success.  `context`
+ * is the caller's pointer (the ctx itself if the caller passed NULL).       */
+typedef int (*mapsm_routine)(void* context, int slab, int device, void* stream, const mapsm_segment* segs,
+                             int nsegs, const float* scalars, int nscalars);
+
+mapsm_status mapsm_matrix_create(mapsm_ctx ctx, int64_t rows, int64_t cols, mapsm_matrix* out);
+mapsm_status mapsm_matrix_destroy(mapsm_matrix m);
+/* Bind: every process passes the FULL matrix (host or device memory,
+ * leading dimension ld >= cols floats, copied).  It is uploaded to the
+ * process's first slab; other slabs receive segments on demand.  Collective. */
+mapsm_status mapsm_matrix_bind(mapsm_matrix m, const float* ptr, int64_t ld);
+/* InvokeUnmodified (Table 2).  EINVAL: bad pattern / sizes (row-block
+ * patterns need rows == task_rows), nparams outside 1..MAPSM_MAX_PARAMS.
+ * ESTATE: an input was never bound or written.  ECUDA: the routine returned
+ * nonzero.  `moved_bytes` (may be NULL): bytes this process moved for the task.*/
+mapsm_status mapsm_invoke_unmodified(mapsm_ctx ctx, int64_t task_rows, mapsm_routine routine, void* context,
+                                     int nparams, const mapsm_matrix* params, const int* patterns,
+                                     const float* scalars, int nscalars, int64_t* moved_bytes);
+/* Wait for the matrix's pending work (Wait, Table 2).                       */
+mapsm_status mapsm_matrix_sync(mapsm_matrix m);
+/* Gather the current version to `ptr` (host or device, ld floats) on `root`;
+ * other processes pass NULL.  Collective; synchronises.                     */
+mapsm_status mapsm_matrix_gather(mapsm_matrix m, float* ptr, int64_t ld, int root);
+/* Built-in wrappers over cuBLAS (dlopen'ed libcublas.so.12, plain fp32
+ * math, no TF32), for use as `routine` with context NULL:
+ *   sgemm: params (A BLOCK2D m x k, B BLOCK2D_T k x n, C OUT_SI or INOUT_SI
+ *          m x n), scalars (alpha, beta): C = alpha A B + beta C;
+ *   saxpy: params (x BLOCK2D, y INOUT_SI, same shape), scalars (alpha):
+ *          y = alpha x + y (Fig 5).                                         */
+int mapsm_routine_sgemm(void* context, int slab, int device, void* stream, const mapsm_segment* segs, int nsegs,
+                        const float* scalars, int nscalars);
+int mapsm_routine_saxpy(void* context, int slab, int device, void* stream, const mapsm_segment* segs, int nsegs,
+                        const float* scalars, int nscalars);
+
 /* Copy only this process's own rows (same row range as mapsm_bind) to `ptr`;
  * not collective; synchronises.                                              */
 mapsm_status mapsm_read(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes);

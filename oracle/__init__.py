@@ -127,8 +127,7 @@ def conv3d(vol: np.ndarray, weights: np.ndarray, n: int, boundary="wrap", sides=
     k = round(len(wt) ** (1 / 3))
     assert k ** 3 == len(wt) and k % 2 == 1
     d, h, w = v.shape
-    modes = np.array(sides if sides is not None else [_mode(boundary)] * 6, dtype=np.int32)
-    modes = np.array([_mode(m) for m in modes], dtype=np.int32)
+    modes = np.array([_mode(m) for m in (sides if sides is not None else [boundary] * 6)], dtype=np.int32)
     out = np.empty_like(v)
     rc = _L().oracle_conv3d_ex(v.ctypes.data, out.ctypes.data, w, h, d, n, k // 2, wt.ctypes.data,
                                modes.ctypes.data)

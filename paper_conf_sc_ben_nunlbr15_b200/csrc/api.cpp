@@ -28,11 +28,7 @@
 #include "mapsm.h"
 #include "kernels.h"
 #include "locmon.h"
-#include "nccl.h"
-
-namespace mapsm {
-mapsm_status compute_plan(int64_t h, int g, int r, mapsm_boundary b, int rank, mapsm_slab_plan* out);
-}
+#include "runtime.h"
 
 using namespace mapsm;
 
@@ -40,7 +36,7 @@ using namespace mapsm;
 
 static thread_local std::string g_last_error;
 
-static mapsm_status fail(mapsm_status s, const char* fmt, ...) {
+mapsm_status mapsm::fail(mapsm_status s, const char* fmt, ...) {
     char buf[512];
     va_list ap;
     va_start(ap, fmt);
@@ -50,51 +46,11 @@ static mapsm_status fail(mapsm_status s, const char* fmt, ...) {
     return s;
 }
 
-#define CK(expr)                                                                              \
-    do {                                                                                      \
-        cudaError_t e_ = (expr);                                                              \
-        if (e_ != cudaSuccess)                                                                \
-            return fail(e_ == cudaErrorMemoryAllocation ? MAPSM_ENOMEM : MAPSM_ECUDA,         \
-                        "%s failed: %s (%s:%d)", #expr, cudaGetErrorString(e_), __FILE__, __LINE__); \
-    } while (0)
-
-#define TRY(expr)                          \
-    do {                                   \
-        mapsm_status s_ = (expr);          \
-        if (s_ != MAPSM_OK) return s_;     \
-    } while (0)
-
-// Restores the caller's current device on scope exit (torch relies on it).
-struct DeviceGuard {
-    int prev = -1;
-    DeviceGuard() { cudaGetDevice(&prev); }
-    ~DeviceGuard() {
-        if (prev >= 0) cudaSetDevice(prev);
-    }
-};
-
 // ------------------------------------------------------------------- NCCL
-// Loaded on first use with dlopen("libnccl.so.2"): inside a torch process this
-// resolves to the NCCL torch already loaded (one NCCL per process).
 
-struct NcclApi {
-    void* h = nullptr;
-    decltype(&ncclGetUniqueId) getUniqueId = nullptr;
-    decltype(&ncclCommInitRank) commInitRank = nullptr;
-    decltype(&ncclCommDestroy) commDestroy = nullptr;
-    decltype(&ncclCommAbort) commAbort = nullptr;
-    decltype(&ncclCommGetAsyncError) commGetAsyncError = nullptr;
-    decltype(&ncclSend) send = nullptr;
-    decltype(&ncclRecv) recv = nullptr;
-    decltype(&ncclGroupStart) groupStart = nullptr;
-    decltype(&ncclGroupEnd) groupEnd = nullptr;
-    decltype(&ncclAllReduce) allReduce = nullptr;
-    decltype(&ncclAllGather) allGather = nullptr;
-    decltype(&ncclGetErrorString) errStr = nullptr;
-};
-static NcclApi g_nccl;
+NcclApi mapsm::g_nccl;
 
-static mapsm_status nccl_load() {
+mapsm_status mapsm::nccl_load() {
     if (g_nccl.h) return MAPSM_OK;
     void* h = dlopen("libnccl.so.2", RTLD_NOW | RTLD_GLOBAL);
     if (!h) return fail(MAPSM_ENCCL, "dlopen(libnccl.so.2) failed: %s", dlerror());
@@ -118,25 +74,7 @@ static mapsm_status nccl_load() {
     return MAPSM_OK;
 }
 
-#define NK(expr)                                                                              \
-    do {                                                                                      \
-        ncclResult_t r_ = (expr);                                                             \
-        if (r_ != ncclSuccess)                                                                \
-            return fail(MAPSM_ENCCL, "%s failed: %s", #expr, g_nccl.errStr(r_));              \
-    } while (0)
-
 // ---------------------------------------------------------------- objects
-
-struct mapsm_ctx_s {
-    bool local = false;            // single-process multi-slab mode
-    int rank = 0, world = 1;       // process rank / count (multi-process mode)
-    int g = 1;                     // total slabs
-    int first_slab = 0;            // global index of local slab 0
-    std::vector<int> devices;      // device per local slab
-    cudaStream_t user_stream = nullptr;
-    ncclComm_t comm = nullptr;
-    int live_grids = 0;
-};
 
 struct TimingPair {
     cudaEvent_t a, b;
@@ -318,6 +256,7 @@ extern "C" mapsm_status mapsm_ctx_destroy(mapsm_ctx c) {
     if (!c) return fail(MAPSM_EINVAL, "ctx is NULL");
     if (c->live_grids > 0) return fail(MAPSM_ESTATE, "ctx still has %d grids", c->live_grids);
     if (c->comm) g_nccl.commDestroy(c->comm);
+    blas_release(c);
     delete c;
     return MAPSM_OK;
 }

@@ -17,13 +17,16 @@
 // maps (ROWMAP_*) and double buffering are the 2-D runtime's.  A CTA owns a
 // TX x TY (64 x 16) output tile of the (y, x) plane and streams a chunk of
 // planes in increasing z ("2.5-D blocking"): each input plane's tile plus its
-// r-wide y/x apron is staged ONCE in shared memory (y/x boundary resolved while
-// staging, the next plane's loads in flight in registers during the compute),
-// and feeds the 2r+1 output planes whose accumulators are live in registers.
+// r-wide y/x apron is staged ONCE in shared memory by cp.async (LDGSTS) into a
+// 4-deep plane ring (y/x boundary resolved by the source address, ZERO cells
+// by zero-fill), and feeds the 2r+1 output planes whose accumulators are live
+// in registers.
 // Because planes stream in increasing z, output plane z receives its dz =
 // -r..r tap planes in order — the paper's ILP over rows taken to
 // the third dimension.  Each thread owns 4 consecutive x (one 128-bit store)
-// of one row, reading its (4 + 2r)-wide window rows with three 16-byte LDS.
+// of RY rows (register blocking in y: RY + 2r window rows, three 16-byte LDS
+// each, serve RY x 4 outputs — without it the kernel was shared-memory bound,
+// ncu: 36 wavefronts per 108 FFMA per warp and plane).
 // Weights are a kernel parameter (constant bank).  No tensor cores: a stencil
 // is not a dense contraction and a GEMM reshaping would not be exact.
 #include <cuda_runtime.h>
@@ -34,10 +37,30 @@
 namespace mapsm {
 namespace {
 
-constexpr int TX = 64;       // output columns per CTA (16 lanes x 4 floats)
-constexpr int TY = 16;       // output rows per CTA
-constexpr int NT = 256;      // threads per CTA
+constexpr int TX = 64;       // output columns per CTA (16 thread columns x 4 floats)
+constexpr int NT = 256;      // threads per CTA: 16 x 16
 constexpr int SW = TX + 8;   // smem row stride: tile column c in [-4, TX+4) lives at index c + 4
+#ifndef MAPSM_C3_NBUF
+#define MAPSM_C3_NBUF 4
+#endif
+#ifndef MAPSM_C3_RY1
+#define MAPSM_C3_RY1 4
+#endif
+#ifndef MAPSM_C3_MINB1
+#define MAPSM_C3_MINB1 2
+#endif
+#ifndef MAPSM_C3_RY2
+#define MAPSM_C3_RY2 2
+#endif
+#ifndef MAPSM_C3_MINB2
+#define MAPSM_C3_MINB2 2
+#endif
+constexpr int NBUF = MAPSM_C3_NBUF;   // plane ring depth (NBUF - 1 planes in flight)
+
+// rows per thread (register blocking in y) and CTAs per SM, per radius
+template <int R> struct Cfg;
+template <> struct Cfg<1> { static constexpr int RY = MAPSM_C3_RY1, MINB = MAPSM_C3_MINB1; };
+template <> struct Cfg<2> { static constexpr int RY = MAPSM_C3_RY2, MINB = MAPSM_C3_MINB2; };
 
 template <int R>
 struct Conv3Params {
@@ -47,9 +70,10 @@ struct Conv3Params {
     int64_t rpitch;    // row pitch (floats)
     int64_t planes, h, w;
     int tiles_x;
+    int64_t tiles;
     int nbands;
-    int64_t zbeg[3], zend[3], nchunks[3];
-    int64_t zc;        // planes per chunk
+    int64_t zbeg[3], zend[3];
+    int64_t units;     // plane-tiles over all bands (band-major, then tile, then z)
     int top_map, bot_map, mode;  // plane maps (ROWMAP_*), y/x boundary (ColMode)
     float wt[(2 * R + 1) * (2 * R + 1) * (2 * R + 1)];
 };
@@ -78,78 +102,86 @@ __device__ __forceinline__ int64_t plane_map(int64_t Z, int64_t planes, int top_
     return Z;  // ROWMAP_HALO
 }
 
+__device__ __forceinline__ void cp16(float* dst, const float* src, bool valid) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 16 : 0) : "memory");
+}
+__device__ __forceinline__ void cp4(float* dst, const float* src, bool valid) {
+    const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
+    asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 4 : 0) : "memory");
+}
+__device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
+template <int N>
+__device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
+
+// The tile's staging items (fixed for the CTA): in-plane source offsets of
+// the thread's 16-byte interior chunks and apron floats (-1 = zero cell,
+// -2 = partial vector at the right edge: per-element path).
 template <int R>
-struct Stage {
+struct Items {
+    static constexpr int TY = 16 * Cfg<R>::RY;
     static constexpr int ROWS = TY + 2 * R;
-    static constexpr int NV = ROWS * (TX / 4);   // float4 items (interior columns)
-    static constexpr int NE = ROWS * 2 * R;      // scalar items (apron columns)
+    static constexpr int NV = ROWS * (TX / 4);
+    static constexpr int NE = ROWS * 2 * R;
     static constexpr int KV = (NV + NT - 1) / NT;
     static constexpr int KE = (NE + NT - 1) / NT;
-    float4 v[KV];
-    float e[KE];
+    int64_t voff[KV];
+    int64_t eoff[KE];
 };
 
 template <int R>
-__device__ __forceinline__ void stage_load(const Conv3Params<R>& p, Stage<R>& st, int64_t Z, int64_t x0, int64_t y0) {
-    const int64_t zp = plane_map(Z, p.planes, p.top_map, p.bot_map);
-    const float* plane = p.in + zp * p.ppitch;
+__device__ __forceinline__ void items_init(const Conv3Params<R>& p, Items<R>& it, int64_t x0, int64_t y0) {
 #pragma unroll
-    for (int k = 0; k < Stage<R>::KV; ++k) {
+    for (int k = 0; k < Items<R>::KV; ++k) {
         const int idx = threadIdx.x + k * NT;
-        float4 val = make_float4(0.f, 0.f, 0.f, 0.f);
-        if (idx < Stage<R>::NV) {
-            const int row = idx / (TX / 4), vq = idx % (TX / 4);
-            const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
-            const int64_t x = x0 + 4 * vq;
-            if (y >= 0) {
-                const float* rp = plane + y * p.rpitch;
-                if (x + 3 < p.w) {
-                    val = __ldg(reinterpret_cast<const float4*>(rp + x));
-                } else {
-                    float t[4];
-#pragma unroll
-                    for (int i = 0; i < 4; ++i) {
-                        const int64_t xx = axis_map(x + i, p.w, p.mode);
-                        t[i] = xx >= 0 ? __ldg(rp + xx) : 0.f;
-                    }
-                    val = make_float4(t[0], t[1], t[2], t[3]);
-                }
-            }
-        }
-        st.v[k] = val;
+        const int row = idx / (TX / 4), vq = idx % (TX / 4);
+        const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
+        const int64_t x = x0 + 4 * vq;
+        it.voff[k] = (idx >= Items<R>::NV || y < 0) ? -1 : (x + 3 < p.w ? y * p.rpitch + x : -2);
     }
 #pragma unroll
-    for (int k = 0; k < Stage<R>::KE; ++k) {
+    for (int k = 0; k < Items<R>::KE; ++k) {
         const int idx = threadIdx.x + k * NT;
-        float val = 0.f;
-        if (idx < Stage<R>::NE) {
-            const int row = idx / (2 * R), q = idx % (2 * R);
-            const int c = q < R ? q - R : TX + (q - R);
-            const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
-            const int64_t x = axis_map(x0 + c, p.w, p.mode);
-            if (y >= 0 && x >= 0) val = __ldg(plane + y * p.rpitch + x);
-        }
-        st.e[k] = val;
+        const int row = idx / (2 * R), q = idx % (2 * R);
+        const int c = q < R ? q - R : TX + (q - R);
+        const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
+        const int64_t x = axis_map(x0 + c, p.w, p.mode);
+        it.eoff[k] = (idx >= Items<R>::NE || y < 0 || x < 0) ? -1 : y * p.rpitch + x;
     }
 }
 
+// Issue the cp.async copies of input plane Z's tile into buffer `sm`.
 template <int R>
-__device__ __forceinline__ void stage_store(float* sm, const Stage<R>& st) {
+__device__ __forceinline__ void stage_issue(const Conv3Params<R>& p, const Items<R>& it, float* sm, int64_t Z,
+                                            int64_t x0, int64_t y0) {
+    const float* plane = p.in + plane_map(Z, p.planes, p.top_map, p.bot_map) * p.ppitch;
 #pragma unroll
-    for (int k = 0; k < Stage<R>::KV; ++k) {
+    for (int k = 0; k < Items<R>::KV; ++k) {
         const int idx = threadIdx.x + k * NT;
-        if (idx < Stage<R>::NV) {
+        if (idx < Items<R>::NV) {
             const int row = idx / (TX / 4), vq = idx % (TX / 4);
-            *reinterpret_cast<float4*>(sm + row * SW + 4 + 4 * vq) = st.v[k];
+            float* dst = sm + row * SW + 4 + 4 * vq;
+            const int64_t off = it.voff[k];
+            if (off != -2) {
+                cp16(dst, plane + (off >= 0 ? off : 0), off >= 0);
+            } else {  // right edge: per element
+                const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
+#pragma unroll
+                for (int i = 0; i < 4; ++i) {
+                    const int64_t x = axis_map(x0 + 4 * vq + i, p.w, p.mode);
+                    cp4(dst + i, plane + (x >= 0 ? y * p.rpitch + x : 0), x >= 0);
+                }
+            }
         }
     }
 #pragma unroll
-    for (int k = 0; k < Stage<R>::KE; ++k) {
+    for (int k = 0; k < Items<R>::KE; ++k) {
         const int idx = threadIdx.x + k * NT;
-        if (idx < Stage<R>::NE) {
+        if (idx < Items<R>::NE) {
             const int row = idx / (2 * R), q = idx % (2 * R);
             const int c = q < R ? q - R : TX + (q - R);
-            sm[row * SW + 4 + c] = st.e[k];
+            const int64_t off = it.eoff[k];
+            cp4(sm + row * SW + 4 + c, plane + (off >= 0 ? off : 0), off >= 0);
         }
     }
 }
@@ -165,94 +197,133 @@ __device__ __forceinline__ void store_out(const Conv3Params<R>& p, int64_t z, in
     }
 }
 
-// One input plane (step j of the chunk, J = j mod K compile-time): every live
-// accumulator slot takes its 9 (R=1) / 25 (R=2) taps of this plane.
+// One input plane (chunk step j, J = j mod K compile-time): every live
+// accumulator slot takes this plane's taps.  Window rows t = 0..RY+2R-1 of
+// the thread (tile rows ly*RY + t) are read once each; row t is tap row
+// dy = t - R - i of the thread's output row i.  For a fixed accumulator the
+// taps arrive in (dy, dx) order (t increasing), planes in dz order.
 template <int R, int J>
-__device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const float* sm, float (&acc)[2 * R + 1][4],
-                                              int lx, int ly) {
+__device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const float* sm,
+                                              float (&acc)[2 * R + 1][Cfg<R>::RY][4], int lx, int ly) {
     constexpr int K = 2 * R + 1;
+    constexpr int RY = Cfg<R>::RY;
 #pragma unroll
-    for (int dy = -R; dy <= R; ++dy) {
-        const float* row = sm + (ly + R + dy) * SW + 4 * lx;   // index 4*lx = tile column 4*lx - 4
+    for (int t = 0; t < RY + 2 * R; ++t) {
+        const float* row = sm + (ly * RY + t) * SW + 4 * lx;   // index 4*lx = tile column 4*lx - 4
         const float4 q0 = *reinterpret_cast<const float4*>(row);
         const float4 q1 = *reinterpret_cast<const float4*>(row + 4);
         const float4 q2 = *reinterpret_cast<const float4*>(row + 8);
         const float a[12] = {q0.x, q0.y, q0.z, q0.w, q1.x, q1.y, q1.z, q1.w, q2.x, q2.y, q2.z, q2.w};
 #pragma unroll
-        for (int dz = -R; dz <= R; ++dz) {
-            // this plane is tap plane dz of output oz = j - R - dz: slot (J - R - dz) mod K
-            const int slot = ((J - R - dz) % K + K) % K;
+        for (int i = 0; i < RY; ++i) {
+            const int dy = t - R - i;
+            if (dy < -R || dy > R) continue;
 #pragma unroll
-            for (int dx = -R; dx <= R; ++dx) {
-                const float wv = p.wt[((dz + R) * K + (dy + R)) * K + (dx + R)];
+            for (int dz = -R; dz <= R; ++dz) {
+                const int slot = ((J - R - dz) % K + K) % K;
 #pragma unroll
-                for (int i = 0; i < 4; ++i) acc[slot][i] = __fmaf_rn(wv, a[i + dx + 4], acc[slot][i]);
+                for (int dx = -R; dx <= R; ++dx) {
+                    const float wv = p.wt[((dz + R) * K + (dy + R)) * K + (dx + R)];
+#pragma unroll
+                    for (int e = 0; e < 4; ++e) acc[slot][i][e] = __fmaf_rn(wv, a[e + dx + 4], acc[slot][i][e]);
+                }
             }
         }
     }
 }
 
 template <int R, int J>
-__device__ __forceinline__ bool chunk_step(const Conv3Params<R>& p, float* sm, Stage<R>& st, float (&acc)[2 * R + 1][4],
-                                           int64_t j, int64_t nsteps, int64_t zs, int64_t zlen, int64_t x0, int64_t y0,
-                                           int lx, int ly) {
+__device__ __forceinline__ bool chunk_step(const Conv3Params<R>& p, const Items<R>& it, float* smbase,
+                                           float (&acc)[2 * R + 1][Cfg<R>::RY][4], int64_t j, int64_t nsteps,
+                                           int64_t zs, int64_t zlen, int64_t x0, int64_t y0, int lx, int ly) {
     constexpr int K = 2 * R + 1;
+    constexpr int RY = Cfg<R>::RY;
+    constexpr int BUF = Items<R>::ROWS * SW;
     if (j >= nsteps) return false;
-    __syncthreads();              // previous plane's readers are done
-    stage_store<R>(sm, st);
-    __syncthreads();
-    if (j + 1 < nsteps) stage_load<R>(p, st, zs - R + j + 1, x0, y0);   // next plane in flight
-    compute_plane<R, J>(p, sm, acc, lx, ly);
+    __syncthreads();   // every thread finished plane j-1: its ring slot may be refilled
+    if (j + NBUF - 1 < nsteps) stage_issue<R>(p, it, smbase + ((j + NBUF - 1) % NBUF) * BUF, zs - R + j + NBUF - 1, x0, y0);
+    cp_commit();       // (possibly empty group: keeps the group count uniform)
+    cp_wait<NBUF - 1>();   // plane j has landed (for this thread's copies)
+    __syncthreads();   // ... and for everybody's
+    compute_plane<R, J>(p, smbase + (j % NBUF) * BUF, acc, lx, ly);
     // output oz = j - 2R is complete (its dz = +R plane was this one)
     constexpr int done_slot = ((J - 2 * R) % K + K) % K;
     const int64_t oz = j - 2 * R;
-    if (oz >= 0 && oz < zlen) store_out<R>(p, zs + oz, y0 + ly, x0 + 4 * lx, acc[done_slot]);
+    if (oz >= 0 && oz < zlen) {
 #pragma unroll
-    for (int i = 0; i < 4; ++i) acc[done_slot][i] = 0.0f;
+        for (int i = 0; i < RY; ++i) store_out<R>(p, zs + oz, y0 + ly * RY + i, x0 + 4 * lx, acc[done_slot][i]);
+    }
+#pragma unroll
+    for (int i = 0; i < RY; ++i)
+#pragma unroll
+        for (int e = 0; e < 4; ++e) acc[done_slot][i][e] = 0.0f;
     return true;
 }
 
 template <int R, int... Js>
-__device__ __forceinline__ void run_chunk(const Conv3Params<R>& p, float* sm, int64_t zs, int64_t ze, int64_t x0,
+__device__ __forceinline__ void run_chunk(const Conv3Params<R>& p, float* smbase, int64_t zs, int64_t ze, int64_t x0,
                                           int64_t y0, int lx, int ly) {
     constexpr int K = 2 * R + 1;
-    float acc[K][4];
+    constexpr int RY = Cfg<R>::RY;
+    constexpr int BUF = Items<R>::ROWS * SW;
+    float acc[K][RY][4];
 #pragma unroll
     for (int s = 0; s < K; ++s)
 #pragma unroll
-        for (int i = 0; i < 4; ++i) acc[s][i] = 0.0f;
-    Stage<R> st;
+        for (int i = 0; i < RY; ++i)
+#pragma unroll
+            for (int e = 0; e < 4; ++e) acc[s][i][e] = 0.0f;
+    Items<R> it;
+    items_init<R>(p, it, x0, y0);
     const int64_t zlen = ze - zs;
     const int64_t nsteps = zlen + 2 * R;   // input planes zs-R .. ze+R-1
-    stage_load<R>(p, st, zs - R, x0, y0);
+    // prologue: planes 0 .. NBUF-2 in flight
+#pragma unroll
+    for (int q = 0; q < NBUF - 1; ++q) {
+        if (q < nsteps) stage_issue<R>(p, it, smbase + q * BUF, zs - R + q, x0, y0);
+        cp_commit();
+    }
     for (int64_t j = 0; j < nsteps; j += K) {
         bool go = true;
         // unrolled K steps: J = 0..K-1 are compile-time slot phases
-        ((go = go && chunk_step<R, Js>(p, sm, st, acc, j + Js, nsteps, zs, zlen, x0, y0, lx, ly)), ...);
+        ((go = go && chunk_step<R, Js>(p, it, smbase, acc, j + Js, nsteps, zs, zlen, x0, y0, lx, ly)), ...);
+    }
+    cp_wait<0>();
+}
+
+template <int R>
+__global__ void __launch_bounds__(NT, Cfg<R>::MINB) conv3d_kernel(const __grid_constant__ Conv3Params<R> p) {
+    extern __shared__ __align__(16) float smbase[];
+    constexpr int TY = Items<R>::TY;
+    const int lx = threadIdx.x % (TX / 4), ly = threadIdx.x / (TX / 4);
+    // Balanced split: CTA c of the (persistent, one-wave) grid owns plane-tiles
+    // [c*U/P, (c+1)*U/P) and walks them as runs of consecutive planes of one tile.
+    const int64_t P = gridDim.x;
+    int64_t u = p.units * (int64_t)blockIdx.x / P;
+    const int64_t uend = p.units * ((int64_t)blockIdx.x + 1) / P;
+    while (u < uend) {
+        int64_t v = u;
+        int b = 0;
+        while (b < p.nbands && v >= p.tiles * (p.zend[b] - p.zbeg[b])) v -= p.tiles * (p.zend[b] - p.zbeg[b]), ++b;
+        const int64_t nz = p.zend[b] - p.zbeg[b];
+        const int64_t tile = v / nz, z = v % nz;
+        const int64_t len = (nz - z) < (uend - u) ? (nz - z) : (uend - u);
+        const int64_t x0 = (tile % p.tiles_x) * TX;
+        const int64_t y0 = (tile / p.tiles_x) * TY;
+        const int64_t zs = p.zbeg[b] + z;
+        if constexpr (R == 1)
+            run_chunk<R, 0, 1, 2>(p, smbase, zs, zs + len, x0, y0, lx, ly);
+        else
+            run_chunk<R, 0, 1, 2, 3, 4>(p, smbase, zs, zs + len, x0, y0, lx, ly);
+        u += len;
+        __syncthreads();   // the next run refills the ring from slot 0
     }
 }
 
 template <int R>
-__global__ void __launch_bounds__(NT) conv3d_kernel(const __grid_constant__ Conv3Params<R> p) {
-    __shared__ __align__(16) float sm[(TY + 2 * R) * SW];
-    const int tile = blockIdx.x;
-    const int64_t x0 = (int64_t)(tile % p.tiles_x) * TX;
-    const int64_t y0 = (int64_t)(tile / p.tiles_x) * TY;
-    int64_t c = blockIdx.y;
-    int b = 0;
-    while (b < p.nbands && c >= p.nchunks[b]) c -= p.nchunks[b++];
-    if (b >= p.nbands) return;
-    const int64_t zs = p.zbeg[b] + c * p.zc;
-    const int64_t ze = zs + p.zc < p.zend[b] ? zs + p.zc : p.zend[b];
-    const int lx = threadIdx.x % (TX / 4), ly = threadIdx.x / (TX / 4);
-    if constexpr (R == 1)
-        run_chunk<R, 0, 1, 2>(p, sm, zs, ze, x0, y0, lx, ly);
-    else
-        run_chunk<R, 0, 1, 2, 3, 4>(p, sm, zs, ze, x0, y0, lx, ly);
-}
-
-template <int R>
 cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* weights, int num_sms, cudaStream_t s) {
+    constexpr int TY = Items<R>::TY;
+    constexpr size_t smem = (size_t)NBUF * Items<R>::ROWS * SW * sizeof(float);
     Conv3Params<R> p;
     p.in = static_cast<const float*>(g.in);
     p.out = static_cast<float*>(g.out);
@@ -263,6 +334,7 @@ cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* w
     p.w = g.w;
     p.tiles_x = (int)((g.w + TX - 1) / TX);
     const int64_t tiles = (int64_t)p.tiles_x * ((g.plane_rows + TY - 1) / TY);
+    p.tiles = tiles;
     p.top_map = g.top_map;
     p.bot_map = g.bot_map;
     p.mode = g.col_mode;
@@ -271,22 +343,20 @@ cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* w
     int64_t total = 0;
     for (int b = 0; b < bands.nbands; ++b) total += bands.end[b] - bands.begin[b];
     if (total <= 0 || tiles <= 0) return cudaSuccess;
-    // enough CTAs to keep every SM busy (~6 resident per SM), chunks >= 2K planes
-    const int64_t want = (int64_t)num_sms * 6;
-    int64_t chunks = (want + tiles - 1) / tiles;
-    int64_t zc = (total + chunks - 1) / chunks;
-    if (zc < 2 * K) zc = 2 * K;
-    p.zc = zc;
+    cudaError_t e = cudaFuncSetAttribute(conv3d_kernel<R>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem);
+    if (e != cudaSuccess) return e;   // (per device; cheap, so set on every launch)
+    // one wave of MINB CTAs per SM (persistent), each with an equal share of
+    // the plane-tiles; a share ends in at most a few runs (2R halo planes each)
     p.nbands = bands.nbands;
-    int64_t ny = 0;
+    p.units = 0;
     for (int b = 0; b < bands.nbands; ++b) {
         p.zbeg[b] = bands.begin[b];
-        p.zend[b] = bands.end[b];
-        p.nchunks[b] = bands.end[b] > bands.begin[b] ? (bands.end[b] - bands.begin[b] + zc - 1) / zc : 0;
-        ny += p.nchunks[b];
+        p.zend[b] = bands.end[b] > bands.begin[b] ? bands.end[b] : bands.begin[b];
+        p.units += tiles * (p.zend[b] - p.zbeg[b]);
     }
-    if (tiles > 0x7fffffff || ny > 65535) return cudaErrorInvalidConfiguration;
-    conv3d_kernel<R><<<dim3((unsigned)tiles, (unsigned)ny), NT, 0, s>>>(p);
+    int64_t ctas = (int64_t)num_sms * Cfg<R>::MINB;
+    if (ctas > p.units) ctas = p.units;
+    conv3d_kernel<R><<<(unsigned)ctas, NT, smem, s>>>(p);
     return cudaGetLastError();
 }
 

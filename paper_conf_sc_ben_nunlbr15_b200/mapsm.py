@@ -35,9 +35,13 @@ EXPORTED = [
     "mapsm_get_info", "mapsm_set_option", "mapsm_get_timing", "mapsm_grid_stream", "mapsm_status_string",
     "mapsm_last_error", "mapsm_version", "mapsm_locmon_create", "mapsm_locmon_destroy", "mapsm_locmon_output",
     "mapsm_locmon_query", "mapsm_locmon_copied", "mapsm_task_histogram", "mapsm_gather_async",
-    "mapsm_grid_create_3d",
+    "mapsm_grid_create_3d", "mapsm_matrix_create", "mapsm_matrix_destroy", "mapsm_matrix_bind",
+    "mapsm_invoke_unmodified", "mapsm_matrix_sync", "mapsm_matrix_gather", "mapsm_routine_sgemm",
+    "mapsm_routine_saxpy",
 ]
 MAX_DIMS = 3
+MAX_PARAMS = 8
+PAT_BLOCK2D, PAT_BLOCK2D_T, PAT_OUT_SI, PAT_INOUT_SI = 0, 1, 2, 3
 
 
 class MapsmError(RuntimeError):
@@ -69,6 +73,15 @@ class mapsm_box(ctypes.Structure):
 class mapsm_copy_op(ctypes.Structure):
     _fields_ = [("src", ctypes.c_int), ("dst", ctypes.c_int), ("box", mapsm_box)]
 
+
+class mapsm_segment(ctypes.Structure):
+    _fields_ = [("row0", ctypes.c_int64), ("rows", ctypes.c_int64), ("cols", ctypes.c_int64), ("ld", ctypes.c_int64),
+                ("ptr", ctypes.c_void_p)]
+
+
+# int routine(void* context, int slab, int device, void* stream, const mapsm_segment*, int, const float*, int)
+ROUTINE = ctypes.CFUNCTYPE(ctypes.c_int, ctypes.c_void_p, ctypes.c_int, ctypes.c_int, ctypes.c_void_p,
+                           ctypes.POINTER(mapsm_segment), ctypes.c_int, ctypes.POINTER(ctypes.c_float), ctypes.c_int)
 
 _lib = None
 
@@ -112,6 +125,12 @@ def lib() -> ctypes.CDLL:
         "mapsm_task_histogram": [vp, ci, vp, ci, P(i64)],
         "mapsm_gather_async": [vp, vp, i64, ci],
         "mapsm_grid_create_3d": [vp, i64, i64, i64, ci, P(vp)],
+        "mapsm_matrix_create": [vp, i64, i64, P(vp)],
+        "mapsm_matrix_destroy": [vp],
+        "mapsm_matrix_bind": [vp, vp, i64],
+        "mapsm_invoke_unmodified": [vp, i64, vp, vp, ci, P(vp), P(ci), P(ctypes.c_float), ci, P(i64)],
+        "mapsm_matrix_sync": [vp],
+        "mapsm_matrix_gather": [vp, vp, i64, ci],
     }
     for name, args in sig.items():
         f = getattr(L, name)
@@ -319,6 +338,53 @@ def mapsm_locmon_copied(m: int, datum: int, ops) -> None:
     for i, (src, dst, b) in enumerate(ops):
         arr[i].src, arr[i].dst, arr[i].box = src, dst, _box(b)
     _check(lib().mapsm_locmon_copied(m, datum, n, arr), "mapsm_locmon_copied")
+
+
+# Unmodified routines (NEXT-4): fp32 matrix datums and InvokeUnmodified.
+
+def mapsm_matrix_create(ctx: int, rows: int, cols: int) -> int:
+    out = ctypes.c_void_p()
+    _check(lib().mapsm_matrix_create(ctx, rows, cols, ctypes.byref(out)), "mapsm_matrix_create")
+    return out.value
+
+
+def mapsm_matrix_destroy(m: int) -> None:
+    _check(lib().mapsm_matrix_destroy(m), "mapsm_matrix_destroy")
+
+
+def mapsm_matrix_bind(m: int, buf, ld: int | None = None) -> None:
+    _check(lib().mapsm_matrix_bind(m, _ptr(buf), ld or _pitch(buf, 0) // 4), "mapsm_matrix_bind")
+
+
+def mapsm_matrix_sync(m: int) -> None:
+    _check(lib().mapsm_matrix_sync(m), "mapsm_matrix_sync")
+
+
+def mapsm_matrix_gather(m: int, buf, ld: int | None = None, root: int = 0) -> None:
+    p = None if buf is None else _ptr(buf)
+    _check(lib().mapsm_matrix_gather(m, p, ld or (0 if buf is None else _pitch(buf, 0) // 4), root),
+           "mapsm_matrix_gather")
+
+
+def routine_ptr(routine) -> int:
+    """'sgemm' / 'saxpy' (built-in cuBLAS wrappers), a ROUTINE callback, or an address."""
+    if isinstance(routine, str):
+        return ctypes.cast(getattr(lib(), f"mapsm_routine_{routine}"), ctypes.c_void_p).value
+    if isinstance(routine, ROUTINE):
+        return ctypes.cast(routine, ctypes.c_void_p).value
+    return int(routine)
+
+
+def mapsm_invoke_unmodified(ctx: int, task_rows: int, routine, params, patterns, scalars=(), context=None) -> int:
+    """Run `routine` per slab on the segments the patterns imply; returns bytes moved."""
+    n = len(params)
+    P = (ctypes.c_void_p * n)(*params)
+    pats = (ctypes.c_int * n)(*patterns)
+    sc = (ctypes.c_float * max(1, len(scalars)))(*scalars)
+    moved = ctypes.c_int64()
+    _check(lib().mapsm_invoke_unmodified(ctx, task_rows, routine_ptr(routine), context, n, P, pats, sc,
+                                         len(scalars), ctypes.byref(moved)), "mapsm_invoke_unmodified")
+    return moved.value
 
 
 def mapsm_grid_destroy(grid: int) -> None:

@@ -53,3 +53,32 @@ def cone_eval(op, gen, h, w, r, n, boundary, ys, ye, xs, xe, weights=None):
     oy = ys - y0 if (cut_t or cut_b) else ys
     ox = xs - x0 if (cut_l or cut_r) else xs
     return patch[oy:oy + (ye - ys), ox:ox + (xe - xs)]
+
+
+def cone_eval3d(vol_rows, d, h, w, r, n, boundary, zr, yr, xr, weights):
+    """Window(3D) light cone: the oracle's generation-n values of the block
+    zr x yr x xr ((start, end) per axis) of a d x h x w volume, evaluated on
+    the cut-out patch as cone_eval does in 2-D.  vol_rows(z, y0, nrows) ->
+    generated rows [y0, y0+nrows) of plane z (shape (nrows, w))."""
+    R = n * r
+    axes = [_axis(zr[0], zr[1], R, d, boundary), _axis(yr[0], yr[1], R, h, boundary),
+            _axis(xr[0], xr[1], R, w, boundary)]
+    (zidx, zm, z_start), (yidx, ym, y_start), (xidx, xm, x_start) = axes
+    patch = np.stack([rows_from(lambda y0, nr, z=int(z): vol_rows(z, y0, nr), yidx)[:, xidx] for z in zidx])
+    origin = [z_start, y_start, x_start]
+    modes = [zm, ym, xm]
+    sides = (zm[0], zm[1], ym[0], ym[1], xm[0], xm[1])
+    for _ in range(n):
+        patch = oracle.conv3d(patch, weights, 1, sides=sides)
+        sl = []
+        for a, m in enumerate(modes):
+            lo = r if m[2] else 0
+            hi = r if m[3] else 0
+            sl.append(slice(lo, patch.shape[a] - hi))
+            origin[a] += lo
+        patch = patch[tuple(sl)]
+    out = []
+    for a, (m, rng) in enumerate(zip(modes, (zr, yr, xr))):
+        o = rng[0] - origin[a] if (m[2] or m[3]) else rng[0]
+        out.append(slice(o, o + rng[1] - rng[0]))
+    return patch[tuple(out)]

@@ -34,6 +34,39 @@ __global__ void k_ur(float* out, float s, const __grid_constant__ Wt wt) {
     float t = 0; for (int c = 0; c < CH; ++c) t += a[c];
     out[blockIdx.x * blockDim.x + threadIdx.x] = t;
 }
+// FFMA2 (fma.rn.f32x2, sm_100a): two fp32 FMAs per lane per instruction.
+// rr: all operands register pairs; bc: the weight a broadcast scalar (UR).
+__global__ void k_f2rr(float* out, float s) {
+    unsigned long long a[CH], x[CH], w[CH];
+    for (int c = 0; c < CH; ++c) {
+        float2 fa = make_float2(threadIdx.x + c, c), fx = make_float2(s * c + threadIdx.x, s), fw = make_float2(s + c * 0.001f, s);
+        a[c] = *reinterpret_cast<unsigned long long*>(&fa); x[c] = *reinterpret_cast<unsigned long long*>(&fx);
+        w[c] = *reinterpret_cast<unsigned long long*>(&fw);
+    }
+#pragma unroll 1
+    for (int it = 0; it < ITERS; ++it)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) asm volatile("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(a[c]) : "l"(x[c]), "l"(w[c]));
+    float t = 0; for (int c = 0; c < CH; ++c) { float2 f = *reinterpret_cast<float2*>(&a[c]); t += f.x + f.y; }
+    out[blockIdx.x * blockDim.x + threadIdx.x] = t;
+}
+__global__ void k_f2bc(float* out, float s, const __grid_constant__ Wt wt) {
+    unsigned long long a[CH], x[CH];
+    for (int c = 0; c < CH; ++c) {
+        float2 fa = make_float2(threadIdx.x + c, c), fx = make_float2(s * c + threadIdx.x, s);
+        a[c] = *reinterpret_cast<unsigned long long*>(&fa); x[c] = *reinterpret_cast<unsigned long long*>(&fx);
+    }
+#pragma unroll 1
+    for (int it = 0; it < ITERS; ++it)
+#pragma unroll
+        for (int c = 0; c < CH; ++c) {
+            float2 wv = make_float2(wt.w[c], wt.w[c]);
+            unsigned long long W = *reinterpret_cast<unsigned long long*>(&wv);
+            asm volatile("fma.rn.f32x2 %0, %1, %2, %0;" : "+l"(a[c]) : "l"(x[c]), "l"(W));
+        }
+    float t = 0; for (int c = 0; c < CH; ++c) { float2 f = *reinterpret_cast<float2*>(&a[c]); t += f.x + f.y; }
+    out[blockIdx.x * blockDim.x + threadIdx.x] = t;
+}
 int main() {
     int sms, clk; cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, 0); cudaDeviceGetAttribute(&clk, cudaDevAttrClockRate, 0);
     float* out; cudaMalloc(&out, sms * 512 * 4 * 4);
@@ -48,6 +81,8 @@ int main() {
     };
     run("rrr", [&] { k_rrr<<<sms, 512>>>(out, 1.0001f); });
     run("imm", [&] { k_imm<<<sms, 512>>>(out, 1.0001f); });
+    run("f2rr", [&] { k_f2rr<<<sms, 512>>>(out, 1.0001f); });   // x2: each instruction is 2 FMAs per lane
+    run("f2bc", [&] { k_f2bc<<<sms, 512>>>(out, 1.0001f, wt); });
     run("ur", [&] { k_ur<<<sms, 512>>>(out, 1.0001f, wt); });
     return 0;
 }
