@@ -65,6 +65,11 @@ WORKLOADS = {
                     scaling="strong", bcell=8.0,
                     label="fp32 5x5x5 Window(3D) convolution 512x512x512 CLAMP, 20 iterations per step (SURVEY "
                           "§8(f) NEXT-2; FMA-bound; not a BASELINE config)"),
+    "sgemm8k": dict(op="sgemm", w=8192, h=8192, r=0, b="none", n=10, seed=0x5EED0008, wseed=None,
+                    scaling="weak", bcell=0.0,
+                    label="chain of fp32 8192x8192 matrix multiplications C = A B through InvokeUnmodified "
+                          "(cuBLAS SGEMM wrapper, Block2D / Block2D-T / SI patterns; the paper's 8K chain, "
+                          "P:L491-508; SURVEY §8(f) NEXT-4), 10 multiplications per step"),
     "hist8k": dict(op="histogram", w=8192, h=8192, r=0, b="no_checks", n=1, seed=0x5EED0006, wseed=None,
                    scaling="strong", bcell=1.0,
                    label="256-bin histogram of an 8192x8192 u8 image, uniform pixels (seed 0x5EED0006), one "
@@ -73,6 +78,8 @@ WORKLOADS = {
 
 
 def metric_of(wl):
+    if wl["op"] == "sgemm":
+        return "fp32 matrix-multiplication FLOP/s (unmodified cuBLAS routine)", "FLOP/s"
     if wl["op"] == "life":
         return "Game of Life cell-updates/s", "cell-updates/s"
     if wl["op"] == "conv":
@@ -149,6 +156,19 @@ def _oracle_sample(wl):
     import oracle
 
     w = wl["w"]
+    if wl["op"] == "sgemm":
+        from oracle import blas
+        import numpy as np
+
+        rows = 512
+        rng = np.random.default_rng(wl["seed"])
+        a = (rng.random((rows, w), dtype=np.float32) - 0.5)
+        bm = (rng.random((w, w), dtype=np.float32) - 0.5)
+
+        def run_mm(k):
+            for _ in range(k):
+                blas.sgemm(a, bm)
+        return run_mm, 2.0 * rows * w * w, f"{rows} x {w} @ {w} x {w} float64 products"
     if wl["op"] == "life":
         rows = 512
         g0 = mi.life_u8(wl["seed"], w, rows)
@@ -174,6 +194,8 @@ def _oracle_sample(wl):
 def _oracle_threads(wl):
     import oracle
 
+    if wl["op"] == "sgemm":
+        return os.cpu_count()  # numpy's BLAS threads
     return 1 if wl["op"] == "histogram" else oracle.num_threads()  # the histogram oracle is sequential
 
 
@@ -192,6 +214,144 @@ def cpu_baseline(wl, budget_s=12.0):
     return {"value": units * n / dt, "unit": unit, "cores": _oracle_threads(wl), "kind": "oracle",
             "sample": f"{what} of the same {wl['op']} workload ({wl['b']} boundary on the sample), {n} iterations, "
                       f"{dt:.1f} s wall (oracle/oracle.c)"}
+
+
+def run_sgemm(args, wl, rank, world, local_rank):
+    """NEXT-4 measurement: a chain of C = A B (m = 8192 rows per GPU, weak)
+    through mapsm_invoke_unmodified with the cuBLAS SGEMM wrapper; A, B
+    resident (the Location Monitor moves nothing after the first call)."""
+    import numpy as np
+    import torch
+    import torch.distributed as dist
+
+    from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
+
+    torch.cuda.set_device(local_rank)
+    dev = torch.device("cuda", local_rank)
+    if world > 1:
+        dist.init_process_group("nccl", device_id=dev)
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
+    uid = None
+    if world > 1:
+        obj = [M.mapsm_nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        uid = obj[0]
+    ctx = M.mapsm_ctx_create(rank, world, local_rank, uid, stream.cuda_stream)
+    k = n = wl["w"]
+    m = wl["h"] * world
+    chain = wl["n"]
+    g = torch.Generator().manual_seed(wl["seed"])
+    hA = (torch.rand((m, k), generator=g) - 0.5).pin_memory()
+    hB = (torch.rand((k, n), generator=g) - 0.5).pin_memory()
+    hC = torch.empty((m, n), dtype=torch.float32).pin_memory()
+    A = M.mapsm_matrix_create(ctx, m, k)
+    B = M.mapsm_matrix_create(ctx, k, n)
+    C = M.mapsm_matrix_create(ctx, m, n)
+    M.mapsm_matrix_bind(A, hA)
+    M.mapsm_matrix_bind(B, hB)
+    pats = [M.PAT_BLOCK2D, M.PAT_BLOCK2D_T, M.PAT_OUT_SI]
+
+    def step():
+        moved = 0
+        for _ in range(chain):
+            moved += M.mapsm_invoke_unmodified(ctx, m, "sgemm", [A, B, C], pats, (1.0, 0.0))
+        return moved
+
+    def barrier():
+        if world > 1:
+            dist.barrier(device_ids=[local_rank])
+        torch.cuda.synchronize()
+
+    first_moved = M.mapsm_invoke_unmodified(ctx, m, "sgemm", [A, B, C], pats, (1.0, 0.0))
+    for _ in range(args.warmup):
+        step()
+    barrier()
+    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
+    sampler = ClockSampler(local_rank)
+    sampler.start()
+    total_ms, moved = 0.0, 0
+    barrier()
+    for _ in range(args.steps):
+        flush.zero_()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        moved += step()
+        e1.record(stream)
+        e1.synchronize()
+        total_ms += e0.elapsed_time(e1)
+    barrier()
+    clocks = sampler.stop()
+    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    total_ms = float(t.item())
+    flop_step = 2.0 * m * n * k * chain
+    value = flop_step * args.steps / (total_ms / 1e3)
+    # e2e: host matrices bound, chain, gather C to pinned host memory
+    e2e_ms = 0.0
+    for _ in range(args.e2e_steps):
+        barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        M.mapsm_matrix_bind(A, hA)
+        M.mapsm_matrix_bind(B, hB)
+        step()
+        M.mapsm_matrix_gather(C, hC if rank == 0 else None)
+        e1.record(stream)
+        e1.synchronize()
+        e2e_ms += e0.elapsed_time(e1)
+    te = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
+    if world > 1:
+        dist.all_reduce(te, op=dist.ReduceOp.MAX)
+    e2e_value = flop_step * args.e2e_steps / (float(te.item()) / 1e3)
+    for h in (A, B, C):
+        M.mapsm_matrix_destroy(h)
+    M.mapsm_ctx_destroy(ctx)
+    if rank == 0:
+        sm_mhz = clocks.get("sm_mhz") or 1965.0
+        peak = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
+        ach = value / world / 1e12
+        cb = None
+        if not args.no_cpu_baseline:
+            from oracle import blas
+
+            rows = 512
+            a = hA[:rows].numpy()
+            b = hB.numpy()
+            t0 = time.perf_counter()
+            reps = 0
+            while time.perf_counter() - t0 < 8.0 or reps == 0:
+                blas.sgemm(a, b)
+                reps += 1
+            dt = time.perf_counter() - t0
+            cb = {"value": 2.0 * rows * n * k * reps / dt, "unit": "FLOP/s", "cores": os.cpu_count(),
+                  "kind": "oracle", "sample": f"{rows} x {k} @ {k} x {n} in float64 (oracle/blas.py, numpy), "
+                                              f"{reps} reps, {dt:.1f} s"}
+        line = {"metric": metric_of(wl)[0], "value": value, "unit": "FLOP/s", "n_gpus": world, "steps": args.steps,
+                "warmup": args.warmup, "ms_per_step": total_ms / args.steps, "higher_is_better": True,
+                "scaling": "weak", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+                "config": {"workload": wl["label"], "m": m, "n": n, "k": k, "multiplications_per_step": chain,
+                           "parallelism": f"row-slab x{world}",
+                           "l2": "L2 flushed between steps (256 MiB write); 768 MiB of operands per GPU"},
+                "e2e": {"value": e2e_value, "unit": "FLOP/s", "h2d_bytes_per_step": 4 * (m * k + k * n) * world,
+                        "d2h_bytes_per_step": 4 * m * n,
+                        "how": "mapsm_matrix_bind(A, B pinned host) + chain + mapsm_matrix_gather(C -> pinned host)"},
+                "gpu_launches": 0,
+                "gpu_launches_note": "the kernels are cuBLAS's (an unmodified library routine by design, P:L405)",
+                "moved_bytes": {"first_call": int(first_moved), "timed_region": int(moved)},
+                "roofline": {"bound": "fma", "kernel": "cuBLAS SGEMM (fp32 CUDA-core FMA, no TF32)", "achieved": ach,
+                             "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
+                             "peak_source": "148 SMs x 128 FP32 lanes x 2 flop x sampled SM clock (nominal)"},
+                "clocks": clocks, "cpu_baseline": cb,
+                "paper_context": "Table 4 P:L503-508: single-GPU 8K multiplication 245-366 ms on GTX 780/Titan "
+                                 "Black/GTX 980 (CUBLAS over MAPS-Multi 248.62 ms on GTX 980)"}
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        dist.barrier(device_ids=[local_rank])
+        dist.destroy_process_group()
 
 
 def run_reference(args, wl, rank, world):
@@ -220,7 +380,7 @@ def run_reference(args, wl, rank, world):
     line = {"impl": "reference", "metric": metric, "value": value, "unit": unit,
             "n_gpus": args.gpus, "steps": args.steps, "warmup": args.warmup, "ms_per_step": dt * 1e3 / args.steps,
             "higher_is_better": True, "scaling": wl["scaling"], "vs_baseline": None,
-            "dtype": "f32" if wl["op"] == "conv" else "u8", "data": "synthetic",
+            "dtype": "f32" if wl["op"] in ("conv", "sgemm") else "u8", "data": "synthetic",
             "config": {"workload": wl["label"]}, "cpu_baseline": cb,
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
     print(json.dumps(line), flush=True)
@@ -249,6 +409,9 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     if args.impl == "reference":
         run_reference(args, wl, rank, world)
+        return
+    if wl["op"] == "sgemm":
+        run_sgemm(args, wl, rank, world, local_rank)
         return
 
     import torch

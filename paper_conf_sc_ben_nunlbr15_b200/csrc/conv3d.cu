@@ -55,7 +55,8 @@ constexpr int SW = TX + 8;   // smem row stride: tile column c in [-4, TX+4) liv
 #ifndef MAPSM_C3_MINB2
 #define MAPSM_C3_MINB2 2
 #endif
-constexpr int NBUF = MAPSM_C3_NBUF;   // plane ring depth (NBUF - 1 planes in flight)
+constexpr int NBUF = MAPSM_C3_NBUF;
+typedef unsigned long long Acc2;   // a pair of fp32 accumulators (see fma_pair)   // plane ring depth (NBUF - 1 planes in flight)
 
 // rows per thread (register blocking in y) and CTAs per SM, per radius
 template <int R> struct Cfg;
@@ -72,10 +73,13 @@ struct Conv3Params {
     int tiles_x;
     int64_t tiles;
     int nbands;
-    int64_t zbeg[3], zend[3];
-    int64_t units;     // plane-tiles over all bands (band-major, then tile, then z)
+    int64_t zbeg[3], zend[3], zc[3];
+    int64_t units;     // plane-tiles over all bands (band-major, then z-block of zc planes, then tile, then z)
     int top_map, bot_map, mode;  // plane maps (ROWMAP_*), y/x boundary (ColMode)
     float wt[(2 * R + 1) * (2 * R + 1) * (2 * R + 1)];
+    // weight pairs for fma_pair, aligned so each loads as one 64-bit uniform
+    // register pair: wp[((dz+R)(2R+1) + dy+R) 2R + dx+R-1] = (W[..][dx-1], W[..][dx]), dx in [1-R, R]
+    float2 wp[(2 * R + 1) * (2 * R + 1) * 2 * R];
 };
 
 // Index along an axis of n cells under the in-plane boundary; -1 = zero cell.
@@ -89,10 +93,10 @@ __device__ __forceinline__ int64_t axis_map(int64_t i, int64_t n, int mode) {
     return -1;
 }
 
-// Slab-local plane index an input plane Z reads (halo planes live at -R..-1
-// and planes..planes+R-1 of the buffer).
-__device__ __forceinline__ int64_t plane_map(int64_t Z, int64_t planes, int top_map, int bot_map) {
-    if (Z >= 0 && Z < planes) return Z;
+// Slab-local plane index an input plane Z outside [0, planes) reads (halo
+// planes live at -R..-1 and planes..planes+R-1 of the buffer).  Out of line:
+// the hot loop only tests the range.
+__device__ __noinline__ int64_t plane_map_edge(int64_t Z, int64_t planes, int top_map, int bot_map) {
     const int m = Z < 0 ? top_map : bot_map;
     if (m == ROWMAP_WRAP) {
         int64_t q = Z % planes;
@@ -110,6 +114,10 @@ __device__ __forceinline__ void cp4(float* dst, const float* src, bool valid) {
     const unsigned d = (unsigned)__cvta_generic_to_shared(dst);
     asm volatile("cp.async.ca.shared.global [%0], [%1], 4, %2;\n" ::"r"(d), "l"(src), "r"(valid ? 4 : 0) : "memory");
 }
+__device__ __forceinline__ int64_t plane_map(int64_t Z, int64_t planes, int top_map, int bot_map) {
+    return (Z >= 0 && Z < planes) ? Z : plane_map_edge(Z, planes, top_map, bot_map);
+}
+
 __device__ __forceinline__ void cp_commit() { asm volatile("cp.async.commit_group;\n" ::: "memory"); }
 template <int N>
 __device__ __forceinline__ void cp_wait() { asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory"); }
@@ -150,6 +158,17 @@ __device__ __forceinline__ void items_init(const Conv3Params<R>& p, Items<R>& it
     }
 }
 
+// A 16-byte chunk that crosses the right edge of the plane (or lies past it):
+// four 4-byte copies with the x boundary resolved per element.
+__device__ __noinline__ void stage_partial(const float* plane, float* dst, int64_t yy, int64_t x, int64_t h, int64_t w,
+                                           int64_t rpitch, int mode) {
+    const int64_t y = axis_map(yy, h, mode);
+    for (int i = 0; i < 4; ++i) {
+        const int64_t xx = axis_map(x + i, w, mode);
+        cp4(dst + i, plane + (xx >= 0 && y >= 0 ? y * rpitch + xx : 0), xx >= 0 && y >= 0);
+    }
+}
+
 // Issue the cp.async copies of input plane Z's tile into buffer `sm`.
 template <int R>
 __device__ __forceinline__ void stage_issue(const Conv3Params<R>& p, const Items<R>& it, float* sm, int64_t Z,
@@ -162,16 +181,10 @@ __device__ __forceinline__ void stage_issue(const Conv3Params<R>& p, const Items
             const int row = idx / (TX / 4), vq = idx % (TX / 4);
             float* dst = sm + row * SW + 4 + 4 * vq;
             const int64_t off = it.voff[k];
-            if (off != -2) {
+            if (off != -2)
                 cp16(dst, plane + (off >= 0 ? off : 0), off >= 0);
-            } else {  // right edge: per element
-                const int64_t y = axis_map(y0 - R + row, p.h, p.mode);
-#pragma unroll
-                for (int i = 0; i < 4; ++i) {
-                    const int64_t x = axis_map(x0 + 4 * vq + i, p.w, p.mode);
-                    cp4(dst + i, plane + (x >= 0 ? y * p.rpitch + x : 0), x >= 0);
-                }
-            }
+            else  // right edge: per element, out of line
+                stage_partial(plane, dst, y0 - R + row, x0 + 4 * vq, p.h, p.w, p.rpitch, p.mode);
         }
     }
 #pragma unroll
@@ -187,14 +200,41 @@ __device__ __forceinline__ void stage_issue(const Conv3Params<R>& p, const Items
 }
 
 template <int R>
-__device__ __forceinline__ void store_out(const Conv3Params<R>& p, int64_t z, int64_t y, int64_t x, const float* a) {
+__device__ __forceinline__ void store_out(const Conv3Params<R>& p, int64_t z, int64_t y, int64_t x, const Acc2* acc2) {
     if (y >= p.h || x >= p.w) return;
+    const float2 p0 = *reinterpret_cast<const float2*>(&acc2[0]), p1 = *reinterpret_cast<const float2*>(&acc2[1]);
+    const float a[4] = {p0.y, p0.x, p1.y, p1.x};   // (hi, lo) = (out 2j, out 2j+1)
     float* op = p.out + z * p.ppitch + y * p.rpitch + x;
     if (x + 3 < p.w) {
         *reinterpret_cast<float4*>(op) = make_float4(a[0], a[1], a[2], a[3]);
     } else {
         for (int i = 0; i < 4 && x + i < p.w; ++i) op[i] = a[i];
     }
+}
+
+// Accumulators in pairs: Acc2 of outputs (x0+2j, x0+2j+1) holds
+// lo = out(x0+2j+1), hi = out(x0+2j), so that one FFMA2 with the input value
+// broadcast (R.F32) and the consecutive weights (W[dx-1], W[dx]) as a
+// uniform-register pair (UR.F32x2) advances both outputs by their own tap:
+// out(2j) by dx, out(2j+1) by dx-1 (each half is an IEEE fma, RN-even — the
+// oracle's fmaf).  The first and last value of a pair's window feed only one
+// of the two outputs: a scalar FFMA on that half.  2R FFMA2 + 2 FFMA per
+// pair and tap row instead of 2(2R+1) FFMA (the kernel is issue-bound, ncu:
+// issue slots 72% busy, not_selected the top stall).
+__device__ __forceinline__ void fma_pair(Acc2& acc, float v, const float2& wv) {
+    asm("{\n\t.reg .b64 x;\n\tmov.b64 x, {%1, %1};\n\tfma.rn.f32x2 %0, x, %2, %0;\n\t}"
+        : "+l"(acc)
+        : "f"(v), "l"(*reinterpret_cast<const unsigned long long*>(&wv)));
+}
+__device__ __forceinline__ void fma_lo(Acc2& acc, float w, float v) {
+    asm("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 l, %1, %2, l;\n\tmov.b64 %0, {l, h};\n\t}"
+        : "+l"(acc)
+        : "f"(w), "f"(v));
+}
+__device__ __forceinline__ void fma_hi(Acc2& acc, float w, float v) {
+    asm("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 h, %1, %2, h;\n\tmov.b64 %0, {l, h};\n\t}"
+        : "+l"(acc)
+        : "f"(w), "f"(v));
 }
 
 // One input plane (chunk step j, J = j mod K compile-time): every live
@@ -204,7 +244,7 @@ __device__ __forceinline__ void store_out(const Conv3Params<R>& p, int64_t z, in
 // taps arrive in (dy, dx) order (t increasing), planes in dz order.
 template <int R, int J>
 __device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const float* sm,
-                                              float (&acc)[2 * R + 1][Cfg<R>::RY][4], int lx, int ly) {
+                                              Acc2 (&acc)[2 * R + 1][Cfg<R>::RY][2], int lx, int ly) {
     constexpr int K = 2 * R + 1;
     constexpr int RY = Cfg<R>::RY;
 #pragma unroll
@@ -221,11 +261,15 @@ __device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const flo
 #pragma unroll
             for (int dz = -R; dz <= R; ++dz) {
                 const int slot = ((J - R - dz) % K + K) % K;
+                const float2* wq = p.wp + ((dz + R) * K + (dy + R)) * 2 * R + R - 1;   // wq[dx] = (W[dx-1], W[dx])
 #pragma unroll
-                for (int dx = -R; dx <= R; ++dx) {
-                    const float wv = p.wt[((dz + R) * K + (dy + R)) * K + (dx + R)];
+                for (int jp = 0; jp < 2; ++jp) {
+                    // window values a[m], m = 4 + 2jp + dx (dx of out(2jp)); in m order
+                    fma_hi(acc[slot][i][jp], wq[1 - R].x, a[4 + 2 * jp - R]);          // out(2jp) only, dx = -R
 #pragma unroll
-                    for (int e = 0; e < 4; ++e) acc[slot][i][e] = __fmaf_rn(wv, a[e + dx + 4], acc[slot][i][e]);
+                    for (int dx = -R + 1; dx <= R; ++dx)
+                        fma_pair(acc[slot][i][jp], a[4 + 2 * jp + dx], wq[dx]);
+                    fma_lo(acc[slot][i][jp], wq[R].y, a[5 + 2 * jp + R]);              // out(2jp+1) only, dx' = R
                 }
             }
         }
@@ -234,7 +278,7 @@ __device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const flo
 
 template <int R, int J>
 __device__ __forceinline__ bool chunk_step(const Conv3Params<R>& p, const Items<R>& it, float* smbase,
-                                           float (&acc)[2 * R + 1][Cfg<R>::RY][4], int64_t j, int64_t nsteps,
+                                           Acc2 (&acc)[2 * R + 1][Cfg<R>::RY][2], int64_t j, int64_t nsteps,
                                            int64_t zs, int64_t zlen, int64_t x0, int64_t y0, int lx, int ly) {
     constexpr int K = 2 * R + 1;
     constexpr int RY = Cfg<R>::RY;
@@ -254,9 +298,7 @@ __device__ __forceinline__ bool chunk_step(const Conv3Params<R>& p, const Items<
         for (int i = 0; i < RY; ++i) store_out<R>(p, zs + oz, y0 + ly * RY + i, x0 + 4 * lx, acc[done_slot][i]);
     }
 #pragma unroll
-    for (int i = 0; i < RY; ++i)
-#pragma unroll
-        for (int e = 0; e < 4; ++e) acc[done_slot][i][e] = 0.0f;
+    for (int i = 0; i < RY; ++i) acc[done_slot][i][0] = acc[done_slot][i][1] = 0ull;   // +0.0f pairs
     return true;
 }
 
@@ -266,13 +308,11 @@ __device__ __forceinline__ void run_chunk(const Conv3Params<R>& p, float* smbase
     constexpr int K = 2 * R + 1;
     constexpr int RY = Cfg<R>::RY;
     constexpr int BUF = Items<R>::ROWS * SW;
-    float acc[K][RY][4];
+    Acc2 acc[K][RY][2];
 #pragma unroll
     for (int s = 0; s < K; ++s)
 #pragma unroll
-        for (int i = 0; i < RY; ++i)
-#pragma unroll
-            for (int e = 0; e < 4; ++e) acc[s][i][e] = 0.0f;
+        for (int i = 0; i < RY; ++i) acc[s][i][0] = acc[s][i][1] = 0ull;
     Items<R> it;
     items_init<R>(p, it, x0, y0);
     const int64_t zlen = ze - zs;
@@ -297,7 +337,10 @@ __global__ void __launch_bounds__(NT, Cfg<R>::MINB) conv3d_kernel(const __grid_c
     constexpr int TY = Items<R>::TY;
     const int lx = threadIdx.x % (TX / 4), ly = threadIdx.x / (TX / 4);
     // Balanced split: CTA c of the (persistent, one-wave) grid owns plane-tiles
-    // [c*U/P, (c+1)*U/P) and walks them as runs of consecutive planes of one tile.
+    // [c*U/P, (c+1)*U/P) and walks them as runs of consecutive planes of one
+    // tile.  Units are ordered z-block-major (zc planes, ~P/tiles blocks), so
+    // the CTAs running at the same time hold neighbouring tiles of the same
+    // planes and the tiles' shared apron sectors hit in L2.
     const int64_t P = gridDim.x;
     int64_t u = p.units * (int64_t)blockIdx.x / P;
     const int64_t uend = p.units * ((int64_t)blockIdx.x + 1) / P;
@@ -306,8 +349,12 @@ __global__ void __launch_bounds__(NT, Cfg<R>::MINB) conv3d_kernel(const __grid_c
         int b = 0;
         while (b < p.nbands && v >= p.tiles * (p.zend[b] - p.zbeg[b])) v -= p.tiles * (p.zend[b] - p.zbeg[b]), ++b;
         const int64_t nz = p.zend[b] - p.zbeg[b];
-        const int64_t tile = v / nz, z = v % nz;
-        const int64_t len = (nz - z) < (uend - u) ? (nz - z) : (uend - u);
+        const int64_t zb = v / (p.tiles * p.zc[b]);
+        const int64_t rem = v - zb * p.tiles * p.zc[b];
+        const int64_t blen = (nz - zb * p.zc[b]) < p.zc[b] ? (nz - zb * p.zc[b]) : p.zc[b];
+        const int64_t tile = rem / blen, zin = rem % blen;
+        const int64_t z = zb * p.zc[b] + zin;
+        const int64_t len = (blen - zin) < (uend - u) ? (blen - zin) : (uend - u);
         const int64_t x0 = (tile % p.tiles_x) * TX;
         const int64_t y0 = (tile / p.tiles_x) * TY;
         const int64_t zs = p.zbeg[b] + z;
@@ -340,6 +387,9 @@ cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* w
     p.mode = g.col_mode;
     constexpr int K = 2 * R + 1;
     for (int i = 0; i < K * K * K; ++i) p.wt[i] = weights[i];
+    for (int zy = 0; zy < K * K; ++zy)
+        for (int dx = 1 - R; dx <= R; ++dx)
+            p.wp[zy * 2 * R + dx + R - 1] = make_float2(weights[zy * K + dx + R - 1], weights[zy * K + dx + R]);
     int64_t total = 0;
     for (int b = 0; b < bands.nbands; ++b) total += bands.end[b] - bands.begin[b];
     if (total <= 0 || tiles <= 0) return cudaSuccess;
@@ -354,8 +404,26 @@ cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* w
         p.zend[b] = bands.end[b] > bands.begin[b] ? bands.end[b] : bands.begin[b];
         p.units += tiles * (p.zend[b] - p.zbeg[b]);
     }
-    int64_t ctas = (int64_t)num_sms * Cfg<R>::MINB;
+    // One run (a z-block of one tile) per CTA where the shape allows: the CTAs
+    // of a z-block then march through the same planes in step, and the x/y
+    // apron sectors a tile shares with its neighbours are read once from DRAM
+    // (measured: a balanced split with runs starting at unrelated planes read
+    // 1.7x the algorithmic bytes).  The grid is the largest multiple of the
+    // tile count that fits in one wave, else one wave of balanced runs.
+    const int64_t slots = (int64_t)num_sms * Cfg<R>::MINB;
+    int64_t nzb = slots / tiles;
+    int64_t ctas;
+    if (nzb >= 1 && bands.nbands == 1) {
+        ctas = tiles * nzb;
+    } else {
+        ctas = slots;
+        nzb = (slots + tiles - 1) / tiles;
+    }
     if (ctas > p.units) ctas = p.units;
+    for (int b = 0; b < bands.nbands; ++b) {
+        const int64_t nz = p.zend[b] - p.zbeg[b];
+        p.zc[b] = nz > 0 ? (nz + nzb - 1) / nzb : 1;
+    }
     conv3d_kernel<R><<<(unsigned)ctas, NT, smem, s>>>(p);
     return cudaGetLastError();
 }
