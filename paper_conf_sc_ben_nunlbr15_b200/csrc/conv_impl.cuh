@@ -33,10 +33,10 @@ namespace conv_detail {
 #define MAPSM_CONV_BIG_CTAS 1
 #endif
 #ifndef MAPSM_CONV_BIG_NC
-#define MAPSM_CONV_BIG_NC 8
+#define MAPSM_CONV_BIG_NC 7
 #endif
 constexpr int kConvBigCtas = MAPSM_CONV_BIG_CTAS;  // CTAs per SM for r >= 3
-constexpr int kConvBigNC = MAPSM_CONV_BIG_NC;      // consumer warps per CTA for r >= 3 (8 or 16)
+constexpr int kConvBigNC = MAPSM_CONV_BIG_NC;      // consumer warps per CTA for r >= 3
 #ifndef MAPSM_CONV_BIG_EPL
 #define MAPSM_CONV_BIG_EPL 4
 #endif
@@ -260,7 +260,43 @@ template <int R>
 struct ConvTmaParams {
     tma::RowStream s;
     float wt[(2 * R + 1) * (2 * R + 1)];
+    // weight pairs for the FFMA2 path: wp[d * 2R + m - 1] = (W[d][m-1], W[d][m]),
+    // m = 1..2R, 8-byte aligned so each is one 64-bit uniform-register pair
+    float2 wp[(2 * R + 1) * 2 * R];
 };
+
+// FFMA2 (fma.rn.f32x2) pair accumulation, radius >= kConvPairMinR.
+// Acc2 of outputs (2j, 2j+1) of a lane holds hi = out(2j), lo = out(2j+1).
+// Window value m of the pair (element 2j - R + m, m = 0..2R+1) feeds out(2j)
+// with tap W[m] (m <= 2R) and out(2j+1) with tap W[m-1] (m >= 1): one FFMA2
+// with the value broadcast and the pair (W[m-1], W[m]) as a 64-bit uniform
+// register does both for m = 1..2R; m = 0 and m = 2R+1 feed a single half
+// (scalar FFMA).  Each half is an IEEE fma, RN-even, and each output still
+// receives its taps in increasing dx — the oracle's fmaf chain exactly
+// (reading c11).  2R FFMA2 + 2 FFMA per pair and tap row instead of
+// 2(2R+1) FFMA: the r >= 3 kernels are FFMA-issue-bound.
+#ifndef MAPSM_CONV_PAIR_MINR
+#define MAPSM_CONV_PAIR_MINR 3
+#endif
+constexpr int kConvPairMinR = MAPSM_CONV_PAIR_MINR;
+typedef unsigned long long Acc2;
+__device__ __forceinline__ void fma_pair(Acc2& acc, float v, const float2& wv) {
+    asm("{\n\t.reg .b64 x;\n\tmov.b64 x, {%1, %1};\n\tfma.rn.f32x2 %0, x, %2, %0;\n\t}"
+        : "+l"(acc)
+        : "f"(v), "l"(*reinterpret_cast<const unsigned long long*>(&wv)));
+}
+__device__ __forceinline__ void fma_lo(Acc2& acc, float w, float v) {
+    asm("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 l, %1, %2, l;\n\tmov.b64 %0, {l, h};\n\t}"
+        : "+l"(acc)
+        : "f"(w), "f"(v));
+}
+__device__ __forceinline__ void fma_hi(Acc2& acc, float w, float v) {
+    asm("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 h, %1, %2, h;\n\tmov.b64 %0, {l, h};\n\t}"
+        : "+l"(acc)
+        : "f"(w), "f"(v));
+}
+__device__ __forceinline__ float acc_hi(Acc2 a) { return __uint_as_float((unsigned)(a >> 32)); }
+__device__ __forceinline__ float acc_lo(Acc2 a) { return __uint_as_float((unsigned)a); }
 
 template <int EPL>
 struct VecF;
@@ -307,7 +343,10 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
     }
     {
     const int t = warp * 32 + lane;
-    float acc[K][EPL];
+    constexpr bool PAIR = R >= kConvPairMinR;
+    static_assert(EPL % 2 == 0, "pairs of outputs");
+    float acc[PAIR ? 1 : K][EPL];
+    Acc2 acc2[PAIR ? K : 1][EPL / 2];
     while (tma::seg_next<NC, EPL>(p, it, sg)) {
         tma::consume_align<NS>(full, empty, ring, lane);
         uint32_t ph = ring.phase;  // segment starts at stage 0
@@ -358,25 +397,64 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                 }
             }
             // v[q + e] = element t*EPL + q + e - R  ->  buf[4 - R + q + e]
+            // Tap row d of output o = j - d lives in slot (k - d) mod K (== o mod K, NS % K == 0).
+            if constexpr (PAIR) {
+                // Window value m outermost, then tap row d and pair jp: the 2R+1 x EPL/2
+                // accumulator chains of this input row are independent, so consecutive
+                // FFMA2s never wait on each other; each chain still takes m (= its dx)
+                // in increasing order.
+#pragma unroll
+                for (int m = 0; m <= K; ++m) {
+#pragma unroll
+                    for (int d = 0; d < K; ++d) {
+                        const int o = j - d;
+                        const int slot = ((k - d) % K + K) % K;
+                        if (check && !(o >= 0 && o < n_out)) continue;
+#pragma unroll
+                        for (int jp = 0; jp < EPL / 2; ++jp) {
+                            const float v = buf[4 - R + 2 * jp + m];
+                            Acc2& a = acc2[slot][jp];
+                            if (m == 0) {
+                                if (d == 0) a = 0ull;   // (+0.0f, +0.0f): output o starts here
+                                fma_hi(a, pp.wt[d * K], v);
+                            } else if (m == K) {
+                                fma_lo(a, pp.wt[d * K + K - 1], v);
+                            } else {
+                                fma_pair(a, v, pp.wp[d * (K - 1) + m - 1]);
+                            }
+                        }
+                    }
+                }
+            }
 #pragma unroll
             for (int d = 0; d < K; ++d) {
                 const int o = j - d;
-                const int slot = ((k - d) % K + K) % K;  // == o mod K since NS % K == 0
+                const int slot = ((k - d) % K + K) % K;
                 if (!check || (o >= 0 && o < n_out)) {
+                    float res[EPL];
+                    if constexpr (PAIR) {
 #pragma unroll
-                    for (int q = 0; q < EPL; ++q) {
-                        float a = (d == 0) ? 0.f : acc[slot][q];
+                        for (int jp = 0; jp < EPL / 2; ++jp) {
+                            res[2 * jp] = acc_hi(acc2[slot][jp]);
+                            res[2 * jp + 1] = acc_lo(acc2[slot][jp]);
+                        }
+                    } else {
 #pragma unroll
-                        for (int e = 0; e < K; ++e) a = __fmaf_rn(pp.wt[d * K + e], buf[4 - R + q + e], a);
-                        acc[slot][q] = a;
+                        for (int q = 0; q < EPL; ++q) {
+                            float a = (d == 0) ? 0.f : acc[slot][q];
+#pragma unroll
+                            for (int e = 0; e < K; ++e) a = __fmaf_rn(pp.wt[d * K + e], buf[4 - R + q + e], a);
+                            acc[slot][q] = a;
+                            res[q] = a;
+                        }
                     }
                     if (d == K - 1 && active) {
                         using OT = typename VecF<EPL>::T;
                         OT ov;
                         if constexpr (EPL == 4)
-                            ov = make_float4(acc[slot][0], acc[slot][1], acc[slot][2], acc[slot][3]);
+                            ov = make_float4(res[0], res[1], res[2], res[3]);
                         else
-                            ov = make_float2(acc[slot][0], acc[slot][1]);
+                            ov = make_float2(res[0], res[1]);
                         *reinterpret_cast<OT*>(out0 + (int64_t)o * p.pitch) = ov;
                         if constexpr (FUSED) {  // boundary rows also go to the neighbours' halos
                             const int64_t yo = sg.ys + o;
@@ -444,6 +522,8 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     p.top_map = g.top_map;
     p.bot_map = g.bot_map;
     for (int j = 0; j < K * K; ++j) pp.wt[j] = weights[j];
+    for (int d = 0; d < K; ++d)
+        for (int m = 1; m < K; ++m) pp.wp[d * (K - 1) + m - 1] = make_float2(weights[d * K + m - 1], weights[d * K + m]);
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
     static int ctas_per_sm = 0;
     if (ctas_per_sm == 0) {
@@ -471,6 +551,18 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     return cudaGetLastError();
 }
 
+// The FMA-bound radii (r >= 3) are compiled one column mode per translation
+// unit (conv_r<R>_cm<CM>.cu) so their large unrolled kernels build in
+// parallel; conv_r<R>.cu declares them extern.
+#define MAPSM_CONV_BIG_INST(KW, R, NS, CM)                                                                        \
+    KW template cudaError_t conv_detail::launch_conv_tma_t<R, 2, NS, CM, conv_detail::kConvBigEPL>(               \
+        const StencilGeom&, const RowBands&, const float*, int, cudaStream_t, const FusedLink*);                 \
+    KW template cudaError_t                                                                                      \
+    conv_detail::launch_conv_tma_t<R, conv_detail::kConvBigNC, NS, CM, conv_detail::kConvBigEPL>(                \
+        const StencilGeom&, const RowBands&, const float*, int, cudaStream_t, const FusedLink*);
+#define MAPSM_CONV_BIG_INST_ALL(KW, R, NS) \
+    MAPSM_CONV_BIG_INST(KW, R, NS, COL_WRAP) MAPSM_CONV_BIG_INST(KW, R, NS, COL_CLAMP) MAPSM_CONV_BIG_INST(KW, R, NS, COL_ZERO)
+
 template <int R, int NS>
 cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                             cudaStream_t s, const FusedLink* link) {
@@ -484,12 +576,19 @@ cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float
             default: return launch_conv_tma_t<R, NC, NS, COL_ZERO, EPL>(g, b, weights, num_sms, s, link);
         }
     };
-    if constexpr (R <= 2 || kConvBigNC == 16) {
+    if constexpr (R <= 2) {
         if (nvec > 8 * 32) return go(std::integral_constant<int, 16>());
+        if (nvec > 4 * 32) return go(std::integral_constant<int, 8>());
+        if (nvec > 2 * 32) return go(std::integral_constant<int, 4>());
+        return go(std::integral_constant<int, 2>());
+    } else {
+        // FMA-bound radii: kConvBigNC consumer warps + the producer warp.  7
+        // keeps the CTA at 8 warps = 2 per SM sub-partition, so ptxas may give
+        // each thread 255 registers (9 warps put 3 on one sub-partition and
+        // cap it at 168: the FFMA2 kernel then spills).  Narrow rows: 2.
+        if (nvec > (kConvBigNC / 2) * 32) return go(std::integral_constant<int, kConvBigNC>());
+        return go(std::integral_constant<int, 2>());
     }
-    if (nvec > 4 * 32) return go(std::integral_constant<int, 8>());
-    if (nvec > 2 * 32) return go(std::integral_constant<int, 4>());
-    return go(std::integral_constant<int, 2>());
 }
 
 template <int R, int PF>
@@ -554,13 +653,17 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
 }  // namespace conv_detail
 
 template <int R>
+constexpr int kConvNS = R == 1 ? 12 : R == 2 ? 10 : R == 3 ? 14 : 9;  // ring stages: multiples of 2R+1
+
+template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                                cudaStream_t s, const FusedLink* link) {
-    constexpr int kNS = R == 1 ? 12 : R == 2 ? 10 : R == 3 ? 14 : 9;  // multiples of 2R+1
+    constexpr int kNS = kConvNS<R>;
     constexpr int kPF = R <= 2 ? 2 : 1;
 #ifndef MAPSM_CONV_REGS
-    if (g.w % 4 == 0 && g.w >= 4 && g.pitch % 16 == 0)
+    if (g.w % 4 == 0 && g.w >= 4 && g.pitch % 16 == 0) {
         return conv_detail::launch_conv_tma<R, kNS>(g, b, weights, num_sms, s, link);
+    }
 #endif
     if (link || b.nbands > 2) return cudaErrorInvalidValue;  // fused exchange needs the TMA kernel
     return conv_detail::launch_conv_t<R, kPF>(g, b, weights, num_sms, s);
