@@ -57,6 +57,10 @@ WORKLOADS = {
                   scaling="weak", bcell=8.0,
                   label="fp32 9x9 (r=4) window stencil, 32768 wide x 4096 rows per GPU, ZERO, 100 iterations per "
                         "step (BASELINE configs[4], weak scaling)"),
+    "conv9sq": dict(op="conv", w=32768, h=32768, r=4, b="zero", n=100, seed=0x5EED0005, wseed=0x5EED0055,
+                    scaling="weak", bcell=8.0,
+                    label="fp32 9x9 (r=4) window stencil, 32768x32768 per GPU, ZERO, 100 iterations per step "
+                          "(BASELINE configs[4], SURVEY 8(d) alternative reading: 32768^2 per GPU)"),
     "conv3d": dict(op="conv", w=512, h=512, d=512, r=1, b="zero", n=100, seed=0x5EED0007, wseed=0x5EED0077,
                    scaling="strong", bcell=8.0,
                    label="fp32 3x3x3 Window(3D) convolution 512x512x512 ZERO, 100 iterations per step (SURVEY "
