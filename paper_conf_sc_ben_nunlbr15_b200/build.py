@@ -66,11 +66,19 @@ def build(force: bool = False, verbose: bool = False, out: str | None = None, cs
     nvcc = os.environ.get("NVCC", "nvcc")
     incs = ["-I", INCLUDE, "-I", src_dir, "-I", _nccl_include()]
     srcs = sorted(glob.glob(os.path.join(src_dir, "*.cu")) + glob.glob(os.path.join(src_dir, "*.cpp")))
+    # incremental: a translation unit recompiles when it is newer than its
+    # object or any shared header / build flag source changed
+    hdr_t = max(os.path.getmtime(p) for p in
+                glob.glob(os.path.join(src_dir, "*.h")) + glob.glob(os.path.join(src_dir, "*.cuh"))
+                + [os.path.join(INCLUDE, "mapsm.h"), __file__])
     objs, cmds = [], []
     for src in srcs:
         obj = os.path.join(obj_dir, os.path.basename(src) + ".o")
-        cmds.append([nvcc, *ARCH, *NVFLAGS, *(extra or []), *incs, "-c", src, "-o", obj])
         objs.append(obj)
+        if (not force and os.path.exists(obj)
+                and os.path.getmtime(obj) > max(os.path.getmtime(src), hdr_t)):
+            continue
+        cmds.append([nvcc, *ARCH, *NVFLAGS, *(extra or []), *incs, "-c", src, "-o", obj])
     # translation units compile in parallel (the conv radii are the slow ones)
     from concurrent.futures import ThreadPoolExecutor
 
