@@ -253,7 +253,10 @@ mapsm_status mapsm_gather(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, i
  * processes: per-slab shared-memory bins, device-side sum across local slabs,
  * ncclAllReduce across processes) written to bins[0..255] (host or device
  * memory, 64-bit counts) on every process.  nbins must be 256; the grid's op
- * must be HISTOGRAM (else ESTATE).  Collective; synchronises.              */
+ * must be HISTOGRAM (else ESTATE).  Collective.  Host `bins`: returns with
+ * the counts written (synchronises).  Device `bins`: stream-ordered on the
+ * ctx stream, like mapsm_iterate — complete after mapsm_sync or any later
+ * synchronisation of that stream.                                          */
 mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
 
 /* Chained task: a Reductive (Static) histogram task
@@ -273,7 +276,8 @@ mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
  *              v >= 1 -> 255 (v * 256 is exact in fp32; DESIGN.md h4).
  * `moved_bytes` (may be NULL) receives the bytes this process received for
  * the task.  EINVAL: target_slabs out of range.  ESTATE: grid not bound.
- * Collective; synchronises.                                                  */
+ * Collective; synchronisation as mapsm_histogram (host bins: synchronises;
+ * device bins: stream-ordered).                                              */
 mapsm_status mapsm_task_histogram(mapsm_grid grid, int target_slabs, uint64_t* bins, int nbins,
                                   int64_t* moved_bytes);
 

@@ -1402,6 +1402,14 @@ extern "C" mapsm_status mapsm_task_histogram(mapsm_grid g, int target_slabs, uin
     }
     TRY(aggregate_bins(g, parts, owner, bins));
     if (moved_bytes) *moved_bytes = moved;
+    // Device-memory bins: stream-ordered like mapsm_iterate (complete on the
+    // grid's stream; mapsm_sync surfaces async errors).  Host bins: the call
+    // returns with the counts in place (the paper's Gather-then-read).
+    int bdev = -1;
+    if (is_device_ptr(bins, &bdev)) {
+        CK(cudaGetLastError());
+        return MAPSM_OK;
+    }
     return check_async(g);
 }
 
