@@ -128,6 +128,12 @@ class ClockSampler:
     def stop(self):
         if self.proc is None:
             return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        # a timed region shorter than nvidia-smi's start-up (the histogram's
+        # ~0.3 ms) has no sample yet: take the first one right after it
+        late = not self.lines
+        t_end = time.time() + 3.0
+        while not self.lines and time.time() < t_end:
+            time.sleep(0.01)
         self.proc.terminate()
         try:
             self.proc.wait(timeout=5)
@@ -148,8 +154,11 @@ class ClockSampler:
             for nm, v in zip(names, parts[2:6]):
                 if v.lower().startswith("active"):
                     reasons.add(nm)
-        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
-                "reasons": sorted(reasons), "samples": len(sm)}
+        out = {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
+               "reasons": sorted(reasons), "samples": len(sm)}
+        if late and sm:
+            out["note"] = "timed region shorter than the sampling start-up; sampled just after it"
+        return out
 
 
 # ------------------------------------------------------------------ oracle leg

@@ -94,6 +94,7 @@ struct Slab {
     cudaGraphExec_t graph_tb[2] = {nullptr, nullptr};  // deep-halo passes (K generations each)
     int64_t graph_tb_passes = 0;
     unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
+    unsigned long long* hist_acc = nullptr;  // 256 counts + CTA ticket, zero between single-launch histograms
     unsigned int* gbar = nullptr;        // grid-barrier word of the persistent Life kernel
     // fused peer-memory exchange (MAPSM_OPT_EXCHANGE = P2P): my mailbox and
     // the neighbours' buffers / mailboxes (same process, or CUDA IPC)
@@ -298,6 +299,7 @@ static void free_slab(Slab& s) {
         if (s.base[b]) cudaFree(s.base[b]);
     if (s.staging) cudaFree(s.staging);
     if (s.hist) cudaFree(s.hist);
+    if (s.hist_acc) cudaFree(s.hist_acc);
     if (s.gbar) cudaFree(s.gbar);
     if (s.mailbox) cudaFree(s.mailbox);
     for (void* q : s.ipc_opened) cudaIpcCloseMemHandle(q);
@@ -368,7 +370,9 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
         CK(cudaMalloc(&s.mailbox, kMailboxBytes));
         CK(cudaMemset(s.mailbox, 0, kMailboxBytes));
         CK(cudaMalloc(&s.hist, 256 * sizeof(unsigned long long)));  // histogram / chained-task partials
-        g->device_bytes += 256 * sizeof(unsigned long long);
+        CK(cudaMalloc(&s.hist_acc, 257 * sizeof(unsigned long long)));
+        CK(cudaMemset(s.hist_acc, 0, 257 * sizeof(unsigned long long)));
+        g->device_bytes += 513 * sizeof(unsigned long long);
         for (int b = 0; b < nbuf; ++b) {
             cudaError_t e = cudaMalloc(&s.base[b], bytes);
             if (e != cudaSuccess) {
@@ -1379,6 +1383,28 @@ extern "C" mapsm_status mapsm_task_histogram(mapsm_grid g, int target_slabs, uin
         NK(g_nccl.groupEnd());
     }
     for (int j = 0; j < T; ++j) g->lm.copied(0, ops[j]);
+
+    // One slab in one process, u8 image on its own partition: a single launch
+    // whose last CTA writes the bins (device bins on the slab's device: in
+    // place; otherwise into s.hist, then one copy).
+    if (same && G == 1 && c->world == 1 && g->op == MAPSM_OP_HISTOGRAM && g->slabs.size() == 1) {
+        Slab& s = g->slabs[0];
+        CK(cudaSetDevice(s.device));
+        int bdev = -1;
+        const bool dev_bins = is_device_ptr(bins, &bdev) && bdev == s.device;
+        CK(launch_histogram_final(reinterpret_cast<const uint8_t*>(row_ptr(g, s, g->cur, 0)), g->pitch, g->w,
+                                  s.plan.rows, s.hist_acc,
+                                  dev_bins ? reinterpret_cast<unsigned long long*>(bins) : s.hist, s.num_sms,
+                                  s.main));
+        g->launches++;
+        if (moved_bytes) *moved_bytes = moved;
+        if (dev_bins) {
+            CK(cudaGetLastError());
+            return MAPSM_OK;
+        }
+        CK(cudaMemcpyAsync(bins, s.hist, 256 * sizeof(unsigned long long), cudaMemcpyDefault, s.main));
+        return check_async(g);
+    }
 
     // The Reductive-Static task itself, per local target slab, then aggregation.
     std::vector<const unsigned long long*> parts;

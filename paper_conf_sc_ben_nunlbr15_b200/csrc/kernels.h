@@ -89,6 +89,13 @@ cudaError_t launch_conv_wide(const StencilGeom& g, const RowBands& b, int r, con
 // (zeroed here; 64-bit counts); and the sum of g partial histograms.
 cudaError_t launch_histogram(const uint8_t* img, int64_t pitch, int64_t w, int64_t rows, unsigned long long* out,
                              int num_sms, cudaStream_t s);
+// Single-launch variant (one slab, one process): CTAs commit into `acc`
+// (256 counts + a CTA ticket at acc[256], all zero on entry and left zero on
+// exit); the last CTA to commit moves the counts to final_out[256] and
+// re-zeroes acc.  No memset, no copy.
+cudaError_t launch_histogram_final(const uint8_t* img, int64_t pitch, int64_t w, int64_t rows,
+                                   unsigned long long* acc, unsigned long long* final_out, int num_sms,
+                                   cudaStream_t s);
 // Chained histogram tasks over stencil grids (api.cpp mapsm_task_histogram):
 // Life (bit-packed rows; bins 0 = dead, 1 = alive) and fp32 (bin =
 // floor(v * 256) clamped).  `out` is zeroed here.
