@@ -483,7 +483,7 @@ def main():
 
     def step():
         if op == "histogram":
-            M.mapsm_histogram(grid.handle, d_bins)
+            M.mapsm_histogram(grid.handle, d_bins, sync=False)
         else:
             grid.iterate(n)
 
@@ -652,7 +652,7 @@ def main():
             e0 = torch.cuda.Event(enable_timing=True)
             e1 = torch.cuda.Event(enable_timing=True)
             e0.record(stream)
-            M.mapsm_task_histogram(grid.handle, 0, d_b)
+            M.mapsm_task_histogram(grid.handle, 0, d_b, sync=False)
             e1.record(stream)
             e1.synchronize()
             c_ms += e0.elapsed_time(e1)

@@ -116,6 +116,41 @@ typedef struct {
 mapsm_status mapsm_plan_query(int64_t h, int g, int radius, mapsm_boundary boundary, int rank,
                               mapsm_slab_plan* out);
 
+/* The messages of the multi-process data plane, as the runtime issues them
+ * (pure host arithmetic; the NCCL exchange and gather iterate exactly these
+ * lists, so the CPU tests can replay them over another transport).
+ * A message moves `rows` whole rows of `pitch` bytes between a slab buffer
+ * laid out as [halo rows | owned rows | halo rows] and the peer:            */
+typedef enum { MAPSM_MSG_SEND = 0, MAPSM_MSG_RECV = 1 } mapsm_msg_kind;
+typedef struct {
+    int kind;            /* mapsm_msg_kind */
+    int peer;            /* the other slab (global rank) */
+    int64_t row;         /* first slab-local row (owned row 0 = 0; top halo rows are < 0,
+                          * bottom halo rows >= rows) */
+    int64_t rows;        /* rows in the message */
+    int64_t offset;      /* byte offset of `row` from the buffer's allocation base
+                          * = (row + halo) * pitch; 0 for a gather receive (staging) */
+    int64_t bytes;       /* rows * pitch */
+    int64_t global_row;  /* global row index (mod h) of the message's first row */
+} mapsm_msg;
+/* Halo exchange of one pass of slab `rank` (Alg 1's P2P copies; "two-line
+ * boundary exchanges per iteration"): `depth` rows per message (r per
+ * generation, or K*r with deep halos), buffers with `halo` >= depth rows per
+ * side.  Order (the contract, inside one ncclGroupStart/End): send-up (rows
+ * [0, depth) to up), send-down (rows [rows-depth, rows) to down), recv-bottom
+ * (rows [rows, rows+depth) from down), recv-top (rows [-depth, 0) from up);
+ * messages of a global edge under CLAMP/ZERO (and all at g == 1) are absent.
+ * Pair-wise issue order matching makes g == 2 WRAP (up == down) correct.
+ * ENOMEM (with *n_msgs set) if max_msgs is too small (4 always suffices);
+ * EINVAL as mapsm_plan_query, or depth > a slab's rows.                      */
+mapsm_status mapsm_exchange_plan(int64_t h, int g, int radius, mapsm_boundary boundary, int rank, int64_t depth,
+                                 int64_t halo, int64_t pitch, mapsm_msg* out, int max_msgs, int* n_msgs);
+/* Gather (Table 2) to `root`: a non-root slab sends its owned rows
+ * (one SEND); the root receives every other slab in slab order (g-1 RECVs,
+ * offset 0 = into staging) and places message k at global_row = y0_k.       */
+mapsm_status mapsm_gather_plan(int64_t h, int g, int radius, mapsm_boundary boundary, int rank, int root,
+                               int64_t halo, int64_t pitch, mapsm_msg* out, int max_msgs, int* n_msgs);
+
 /* ------------------------------------------------- segment location monitor
  * Alg 2 (§4.4): tracks, per datum, `lastOutput` (the segments the
  * last task wrote, per location, and whether they are partials that still
@@ -253,10 +288,11 @@ mapsm_status mapsm_gather(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes, i
  * processes: per-slab shared-memory bins, device-side sum across local slabs,
  * ncclAllReduce across processes) written to bins[0..255] (host or device
  * memory, 64-bit counts) on every process.  nbins must be 256; the grid's op
- * must be HISTOGRAM (else ESTATE).  Collective.  Host `bins`: returns with
- * the counts written (synchronises).  Device `bins`: stream-ordered on the
- * ctx stream, like mapsm_iterate — complete after mapsm_sync or any later
- * synchronisation of that stream.                                          */
+ * must be HISTOGRAM (else ESTATE).  Collective.  Host, pinned or MANAGED
+ * `bins` (host-readable memory): returns with the counts written
+ * (synchronises).  Device-memory `bins` (cudaMalloc): stream-ordered on the
+ * grid's stream (mapsm_grid_stream), like mapsm_iterate — complete after
+ * mapsm_sync or any later synchronisation of that stream.                  */
 mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
 
 /* Chained task: a Reductive (Static) histogram task
@@ -276,8 +312,8 @@ mapsm_status mapsm_histogram(mapsm_grid grid, uint64_t* bins, int nbins);
  *              v >= 1 -> 255 (v * 256 is exact in fp32; DESIGN.md h4).
  * `moved_bytes` (may be NULL) receives the bytes this process received for
  * the task.  EINVAL: target_slabs out of range.  ESTATE: grid not bound.
- * Collective; synchronisation as mapsm_histogram (host bins: synchronises;
- * device bins: stream-ordered).                                              */
+ * Collective; synchronisation as mapsm_histogram (host / managed bins:
+ * synchronises; device-memory bins: stream-ordered).                         */
 mapsm_status mapsm_task_histogram(mapsm_grid grid, int target_slabs, uint64_t* bins, int nbins,
                                   int64_t* moved_bytes);
 
@@ -442,6 +478,35 @@ mapsm_status mapsm_get_timing(mapsm_grid grid, double* bulk_ms, int64_t* bulk_la
 
 /* The compute stream of local slab `local_index` (a cudaStream_t).           */
 mapsm_status mapsm_grid_stream(mapsm_grid grid, int local_index, void** stream);
+
+/* Launch geometry of the last compute kernel launched for local slab
+ * `local_index` (which = 0: the bulk / whole-slab launch, 1: the boundary-row
+ * launch of Alg 1's exchange step), as the launcher issued it — so
+ * tests can check that the kernel configuration they drive is the one the
+ * bench times (e.g. rows per CTA >= 2 ring trips).  Pure host bookkeeping;
+ * recorded at enqueue / graph-capture time.  Kernel ids: */
+typedef enum {
+    MAPSM_KERNEL_NONE = 0, MAPSM_KERNEL_LIFE_TMA = 1, MAPSM_KERNEL_LIFE_REG = 2, MAPSM_KERNEL_LIFE_ANYW = 3,
+    MAPSM_KERNEL_LIFE_PERSIST = 4, MAPSM_KERNEL_LIFE_TB = 5, MAPSM_KERNEL_CONV_TMA = 6, MAPSM_KERNEL_CONV_REG = 7,
+    MAPSM_KERNEL_CONV_GENERIC = 8, MAPSM_KERNEL_CONV_WIDE = 9, MAPSM_KERNEL_CONV3D = 10,
+    MAPSM_KERNEL_LIFE_TB_PERSIST = 11
+} mapsm_kernel;
+typedef struct {
+    int kernel;              /* mapsm_kernel */
+    int threads;             /* threads per CTA */
+    int smem_bytes;          /* dynamic shared memory per CTA */
+    int ring_stages;         /* NS of the row ring (0: no ring) */
+    int rows_per_stage;      /* input rows per ring stage */
+    int consumer_warps;      /* consumer warps per CTA (ring kernels) */
+    int gens_per_launch;     /* generations one launch advances */
+    int64_t ctas;            /* CTAs launched */
+    int64_t strips;          /* column strips per row (ring kernels) */
+    /* ring kernels: over the CTAs that have work, the output rows of the
+     * CTA's LONGEST (strip, row-run) segment (min and max over CTAs), the
+     * CTA's total output rows (min), and the segment count over all CTAs   */
+    int64_t min_cta_seg_rows, max_cta_seg_rows, min_cta_rows, segments;
+} mapsm_launch_info;
+mapsm_status mapsm_launch_query(mapsm_grid grid, int local_index, int which, mapsm_launch_info* out);
 
 const char* mapsm_status_string(mapsm_status s);
 const char* mapsm_last_error(void);

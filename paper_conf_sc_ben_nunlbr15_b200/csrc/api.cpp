@@ -22,6 +22,8 @@
 #include <cstdint>
 #include <cstdio>
 #include <cstring>
+#include <algorithm>
+#include <array>
 #include <string>
 #include <vector>
 
@@ -109,6 +111,7 @@ struct Slab {
     int64_t staging_bytes = 0;
     std::vector<TimingPair> t_bulk, t_bnd;
     size_t t_bulk_used = 0, t_bnd_used = 0;
+    LaunchRec rec_bulk, rec_bnd;   // last launches (mapsm_launch_query)
 };
 
 enum GridState { ST_CREATED = 0, ST_WINDOW = 1, ST_OP = 2, ST_BOUND = 3 };
@@ -402,7 +405,12 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
         for (auto& t : g->slabs) same += t.device == s.device;
         if (same > 1) s.num_sms = s.num_sms / same > 0 ? s.num_sms / same : 1;
     }
-    CK(cudaDeviceSynchronize());
+    // the memsets above ran on each device's legacy stream, which the
+    // non-blocking slab streams do not wait for: finish them on every device
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaDeviceSynchronize());
+    }
     g->p2p_linked = false;
     return MAPSM_OK;
 }
@@ -468,23 +476,45 @@ extern "C" mapsm_status mapsm_grid_slab(mapsm_grid g, int i, int64_t* y0, int64_
 
 // ------------------------------------------------------------ halo exchange
 
+// Both exchange modes iterate the ordered message list of plan.cpp
+// (exchange_messages, exported as mapsm_exchange_plan): NCCL issues it
+// verbatim; local mode resolves every receive to the sending slab's matching
+// send (the j-th receive from peer P takes P's j-th send to me — NCCL's
+// pair-wise in-order matching) and performs it as a peer copy.
+static int slab_messages(const mapsm_grid_s* g, const Slab& s, int64_t depth, mapsm_msg* out) {
+    return exchange_messages(s.plan, g->units(), depth, g->halo, g->pitch, out);
+}
+
 // Local mode: slab i pulls its halos of buffer b from its neighbours with
 // device/peer copies on its side stream, after the neighbours' ev_b.
 static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events, int64_t depth) {
-    const int64_t bytes = depth * g->pitch;
-    for (auto& s : g->slabs) {
+    const int G = (int)g->slabs.size();
+    std::vector<std::array<mapsm_msg, 4>> msgs(G);
+    std::vector<int> nm(G);
+    for (int k = 0; k < G; ++k) nm[k] = slab_messages(g, g->slabs[k], depth, msgs[k].data());
+    for (int k = 0; k < G; ++k) {
+        Slab& s = g->slabs[k];
         CK(cudaSetDevice(s.device));
-        if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
-            Slab& u = g->slabs[s.plan.up];
+        int nth_from[2] = {0, 0};  // receives so far from each of (at most) two peers
+        int peers[2] = {-1, -1};
+        for (int i = 0; i < nm[k]; ++i) {
+            const mapsm_msg& m = msgs[k][i];
+            if (m.kind != MAPSM_MSG_RECV) continue;
+            int slot = (peers[0] == m.peer || peers[0] < 0) ? 0 : 1;
+            peers[slot] = m.peer;
+            const int j = nth_from[slot]++;
+            // the j-th send of slab m.peer addressed to slab k
+            const mapsm_msg* src = nullptr;
+            int seen = 0;
+            for (int q = 0; q < nm[m.peer] && !src; ++q) {
+                const mapsm_msg& t = msgs[m.peer][q];
+                if (t.kind == MAPSM_MSG_SEND && t.peer == k && seen++ == j) src = &t;
+            }
+            if (!src || src->bytes != m.bytes)
+                return fail(MAPSM_ESTATE, "exchange plan: slab %d receive %d has no matching send", k, i);
+            Slab& u = g->slabs[m.peer];
             if (wait_events) CK(cudaStreamWaitEvent(s.side, u.ev_b, 0));
-            CK(cudaMemcpyAsync(row_ptr(g, s, b, -depth), row_ptr(g, u, b, u.plan.rows - depth), bytes,
-                               cudaMemcpyDefault, s.side));
-            g->exchanges++;
-        }
-        if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
-            Slab& d = g->slabs[s.plan.down];
-            if (wait_events) CK(cudaStreamWaitEvent(s.side, d.ev_b, 0));
-            CK(cudaMemcpyAsync(row_ptr(g, s, b, s.plan.rows), row_ptr(g, d, b, 0), bytes, cudaMemcpyDefault,
+            CK(cudaMemcpyAsync(s.base[b] + m.offset, u.base[b] + src->offset, (size_t)m.bytes, cudaMemcpyDefault,
                                s.side));
             g->exchanges++;
         }
@@ -493,22 +523,20 @@ static mapsm_status exchange_local(mapsm_grid_s* g, int b, bool wait_events, int
     return MAPSM_OK;
 }
 
-// NCCL mode: one group per iteration, issued on the side stream in the fixed
-// order send-up, send-down, recv-bottom (from down), recv-top (from up): with
-// g == 2 under WRAP both neighbours are the same peer, and this order makes
-// the peer's first recv (its bottom halo) match my first send (my top rows).
+// NCCL mode: one group per pass, issued on the side stream in the list's
+// order (send-up, send-down, recv-bottom, recv-top; see plan.cpp).
 static mapsm_status exchange_nccl(mapsm_grid_s* g, int b, int64_t depth) {
     Slab& s = g->slabs[0];
-    const size_t bytes = (size_t)depth * (size_t)g->pitch;
+    mapsm_msg msgs[4];
+    const int n = slab_messages(g, s, depth, msgs);
     NK(g_nccl.groupStart());
-    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.send(row_ptr(g, s, b, 0), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
-    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.send(row_ptr(g, s, b, s.plan.rows - depth), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
-    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.recv(row_ptr(g, s, b, s.plan.rows), bytes, ncclUint8, s.plan.down, g->ctx->comm, s.side));
-    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE)
-        NK(g_nccl.recv(row_ptr(g, s, b, -depth), bytes, ncclUint8, s.plan.up, g->ctx->comm, s.side));
+    for (int i = 0; i < n; ++i) {
+        const mapsm_msg& m = msgs[i];
+        if (m.kind == MAPSM_MSG_SEND)
+            NK(g_nccl.send(s.base[b] + m.offset, (size_t)m.bytes, ncclUint8, m.peer, g->ctx->comm, s.side));
+        else
+            NK(g_nccl.recv(s.base[b] + m.offset, (size_t)m.bytes, ncclUint8, m.peer, g->ctx->comm, s.side));
+    }
     NK(g_nccl.groupEnd());
     g->exchanges += s.plan.n_recv;
     return MAPSM_OK;
@@ -529,6 +557,7 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
     geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
     geom.plane_rows = g->d ? g->h : 0;
     geom.rpitch = g->rpitch;
+    geom.rec = bulk ? &s.rec_bulk : &s.rec_bnd;
     TimingPair* tp = nullptr;
     if (g->opt_timing && &s == &g->slabs[0]) {
         auto& vec = bulk ? s.t_bulk : s.t_bnd;
@@ -890,6 +919,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
             geom.top_map = rowmap_of(s.plan.top_kind);
             geom.bot_map = rowmap_of(s.plan.bottom_kind);
             geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+            geom.rec = &s.rec_bulk;
             cudaError_t e = launch_life_persistent(geom, k, s.gbar, s.num_sms, s.main);
             if (e != cudaSuccess) return fail(MAPSM_ECUDA, "persistent Life launch: %s", cudaGetErrorString(e));
             g->launches++;
@@ -962,6 +992,22 @@ extern "C" mapsm_status mapsm_sync(mapsm_grid g) {
 }
 
 // ------------------------------------------------------------- bind / read
+
+// Device memory only (not managed): results written here are stream-ordered;
+// managed and host memory are host-readable, so calls writing there return
+// with the data in place.
+static bool is_device_only_ptr(const void* p, int* dev) {
+    cudaPointerAttributes a;
+    if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+        cudaGetLastError();
+        return false;
+    }
+    if (a.type == cudaMemoryTypeDevice) {
+        *dev = a.device;
+        return true;
+    }
+    return false;
+}
 
 static bool is_device_ptr(const void* p, int* dev) {
     cudaPointerAttributes a;
@@ -1121,35 +1167,39 @@ static mapsm_status gather_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, int r
     CK(cudaSetDevice(s.device));
     if (!async) TRY(check_async(g));
     const int64_t slab_bytes_row = g->pitch;
+    // the gather list of plan.cpp (mapsm_gather_plan): non-root ranks send
+    // their owned rows; the root receives every other slab in slab order
+    std::vector<mapsm_msg> msgs(c->world > 1 ? c->world - 1 : 1);
+    int nmsg = 0;
+    TRY(mapsm_gather_plan(g->units(), c->g, g->r, g->boundary, c->rank, root, g->halo, g->pitch, msgs.data(),
+                          (int)msgs.size(), &nmsg));
     if (c->rank != root) {
-        NK(g_nccl.send(row_ptr(g, s, g->cur, 0), (size_t)(s.plan.rows * slab_bytes_row), ncclUint8, root, c->comm,
-                       s.main));
+        for (int i = 0; i < nmsg; ++i)
+            NK(g_nccl.send(s.base[g->cur] + msgs[i].offset, (size_t)msgs[i].bytes, ncclUint8, msgs[i].peer, c->comm,
+                           s.main));
         return async ? MAPSM_OK : check_async(g);
     }
     int pdev = -1;
     const bool on_dev = is_device_ptr(ptr, &pdev) && pdev == s.device;
-    // Root: receive each slab into a temporary buffer, then unpack / copy out.
+    // Root: its own rows, then each received slab via a temporary buffer.
     mapsm_slab_plan pk;
     compute_plan(g->units(), c->g, g->r, g->boundary, 0, &pk);
     const int64_t max_rows = pk.rows;  // slab 0 is never shorter than any other
     char* tmp = nullptr;
     CK(cudaMallocAsync(reinterpret_cast<void**>(&tmp), (size_t)(max_rows * slab_bytes_row), s.main));
-    mapsm_status st = MAPSM_OK;
-    for (int k = 0; k < c->world && st == MAPSM_OK; ++k) {
-        compute_plan(g->units(), c->g, g->r, g->boundary, k, &pk);
-        char* dst = static_cast<char*>(ptr) + pk.y0 * g->rows_per_unit() * pitch;
-        if (k == root) {
-            st = read_slab(g, s, dst, pitch, on_dev);
-            continue;
-        }
-        ncclResult_t r = g_nccl.recv(tmp, (size_t)(pk.rows * slab_bytes_row), ncclUint8, k, c->comm, s.main);
+    mapsm_status st = read_slab(g, s, static_cast<char*>(ptr) + s.plan.y0 * g->rows_per_unit() * pitch, pitch, on_dev);
+    for (int i = 0; i < nmsg && st == MAPSM_OK; ++i) {
+        const mapsm_msg& m = msgs[i];
+        char* dst = static_cast<char*>(ptr) + m.global_row * g->rows_per_unit() * pitch;
+        ncclResult_t r = g_nccl.recv(tmp + m.offset, (size_t)m.bytes, ncclUint8, m.peer, c->comm, s.main);
         if (r != ncclSuccess) {
-            st = fail(MAPSM_ENCCL, "gather recv from %d: %s", k, g_nccl.errStr(r));
+            st = fail(MAPSM_ENCCL, "gather recv from %d: %s", m.peer, g_nccl.errStr(r));
             break;
         }
         // Reuse read_slab's copy-out path on a view of the received rows.
         Slab view = s;
-        view.plan = pk;
+        view.plan.y0 = m.global_row;
+        view.plan.rows = m.rows;
         view.base[g->cur] = tmp - g->halo * g->pitch;
         view.staging = s.staging;
         view.staging_bytes = s.staging_bytes;
@@ -1391,7 +1441,7 @@ extern "C" mapsm_status mapsm_task_histogram(mapsm_grid g, int target_slabs, uin
         Slab& s = g->slabs[0];
         CK(cudaSetDevice(s.device));
         int bdev = -1;
-        const bool dev_bins = is_device_ptr(bins, &bdev) && bdev == s.device;
+        const bool dev_bins = is_device_only_ptr(bins, &bdev) && bdev == s.device;
         CK(launch_histogram_final(reinterpret_cast<const uint8_t*>(row_ptr(g, s, g->cur, 0)), g->pitch, g->w,
                                   s.plan.rows, s.hist_acc,
                                   dev_bins ? reinterpret_cast<unsigned long long*>(bins) : s.hist, s.num_sms,
@@ -1432,7 +1482,7 @@ extern "C" mapsm_status mapsm_task_histogram(mapsm_grid g, int target_slabs, uin
     // grid's stream; mapsm_sync surfaces async errors).  Host bins: the call
     // returns with the counts in place (the paper's Gather-then-read).
     int bdev = -1;
-    if (is_device_ptr(bins, &bdev)) {
+    if (is_device_only_ptr(bins, &bdev)) {
         CK(cudaGetLastError());
         return MAPSM_OK;
     }
@@ -1557,6 +1607,53 @@ extern "C" mapsm_status mapsm_grid_stream(mapsm_grid g, int i, void** stream) {
     if (!g || !stream) return fail(MAPSM_EINVAL, "NULL argument");
     if (i < 0 || i >= (int)g->slabs.size()) return fail(MAPSM_EINVAL, "local slab %d out of range", i);
     *stream = g->slabs[i].main;
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_launch_query(mapsm_grid g, int i, int which, mapsm_launch_info* o) {
+    if (!g || !o) return fail(MAPSM_EINVAL, "NULL argument");
+    if (i < 0 || i >= (int)g->slabs.size()) return fail(MAPSM_EINVAL, "local slab %d out of range", i);
+    if (which != 0 && which != 1) return fail(MAPSM_EINVAL, "which must be 0 (bulk) or 1 (boundary)");
+    const LaunchRec& r = which == 0 ? g->slabs[i].rec_bulk : g->slabs[i].rec_bnd;
+    memset(o, 0, sizeof *o);
+    o->kernel = r.kernel;
+    o->threads = r.threads;
+    o->smem_bytes = r.smem;
+    o->ring_stages = r.ring_stages;
+    o->rows_per_stage = r.rows_per_stage;
+    o->consumer_warps = r.consumer_warps;
+    o->gens_per_launch = r.gens;
+    o->ctas = r.ctas;
+    o->strips = r.nstrips;
+    if (r.ring_stages > 0) {
+        // the (strip, row) split of tma_rows.cuh seg_iter / seg_next, per CTA
+        int64_t mn = INT64_MAX, mx = 0, mtot = INT64_MAX, nseg = 0;
+        for (int b = 0; b < r.nbands; ++b) {
+            const int64_t C = r.cta_begin[b + 1] - r.cta_begin[b];
+            const int64_t nr = r.end[b] - r.begin[b];
+            const int64_t T = r.nstrips * nr;
+            for (int64_t c = 0; c < C; ++c) {
+                int64_t pos = c * T / C;
+                const int64_t hi = (c + 1) * T / C;
+                if (pos >= hi) continue;
+                int64_t longest = 0;
+                mtot = std::min(mtot, hi - pos);
+                while (pos < hi) {
+                    const int64_t r0 = pos % nr;
+                    const int64_t r1 = (nr - r0 < hi - pos) ? nr : r0 + (hi - pos);
+                    longest = std::max(longest, r1 - r0);
+                    pos += r1 - r0;
+                    ++nseg;
+                }
+                mn = std::min(mn, longest);
+                mx = std::max(mx, longest);
+            }
+        }
+        o->min_cta_seg_rows = nseg ? mn : 0;
+        o->max_cta_seg_rows = mx;
+        o->min_cta_rows = nseg ? mtot : 0;
+        o->segments = nseg;
+    }
     return MAPSM_OK;
 }
 

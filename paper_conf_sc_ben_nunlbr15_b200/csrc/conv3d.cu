@@ -424,6 +424,13 @@ cudaError_t launch_t(const StencilGeom& g, const RowBands& bands, const float* w
         const int64_t nz = p.zend[b] - p.zbeg[b];
         p.zc[b] = nz > 0 ? (nz + nzb - 1) / nzb : 1;
     }
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_CONV3D;
+        g.rec->ctas = ctas;
+        g.rec->threads = NT;
+        g.rec->smem = smem;
+    }
     conv3d_kernel<R><<<(unsigned)ctas, NT, smem, s>>>(p);
     return cudaGetLastError();
 }

@@ -543,6 +543,7 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     }
     tma_set_link(p, link, R);
     const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems, link != nullptr);
+    tma_record(g.rec, LK_CONV_TMA, p, ctas, (NC + 1) * 32, smem, NS, 1, NC);
     if (ctas == 0) return cudaSuccess;
     if (link)
         conv_tma_kernel<R, NC, NS, CM, EPL, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(pp);

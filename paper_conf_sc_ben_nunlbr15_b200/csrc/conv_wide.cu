@@ -151,6 +151,12 @@ cudaError_t launch(const StencilGeom& g, const RowBands& b, const float* weights
         tiles += p.tiles_x * p.tiles_y[i];
     }
     if (tiles == 0) return cudaSuccess;
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_CONV_WIDE;
+        g.rec->ctas = tiles;
+        g.rec->threads = kThreads;
+    }
     conv_wide_kernel<R><<<(unsigned)tiles, kThreads, 0, s>>>(p);
     return cudaGetLastError();
 }

@@ -17,6 +17,28 @@ enum RowMap : int {
 // Column boundary == the grid's boundary (columns are never split).
 enum ColMode : int { COL_WRAP = 0, COL_CLAMP = 1, COL_ZERO = 2 };
 
+// What a launcher actually launched (mapsm_launch_query): the kernel, its
+// grid, and for the row-streaming ring kernels the band table the CTAs split
+// (tma_rows.cuh seg_iter), so the host can report rows per CTA segment.
+enum LaunchKernel : int {
+    LK_NONE = 0, LK_LIFE_TMA = 1, LK_LIFE_REG = 2, LK_LIFE_ANYW = 3, LK_LIFE_PERSIST = 4, LK_LIFE_TB = 5,
+    LK_CONV_TMA = 6, LK_CONV_REG = 7, LK_CONV_GENERIC = 8, LK_CONV_WIDE = 9, LK_CONV3D = 10,
+    LK_LIFE_TB_PERSIST = 11
+};
+struct LaunchRec {
+    int kernel = LK_NONE;
+    int64_t ctas = 0;
+    int threads = 0, smem = 0;
+    int ring_stages = 0;     // NS of the shared-memory ring (0: no ring)
+    int rows_per_stage = 0;  // input rows per ring stage
+    int consumer_warps = 0;
+    int64_t nstrips = 0;     // column strips of a row
+    int nbands = 0;
+    int64_t begin[3] = {0, 0, 0}, end[3] = {0, 0, 0};
+    int64_t cta_begin[4] = {0, 0, 0, 0};
+    int gens = 1;            // generations per launch
+};
+
 // One stencil launch over a slab.  `in`/`out` point at owned row 0 of the
 // input/output slab buffers; halo rows live at rows -r..-1 and rows..rows+r-1.
 struct StencilGeom {
@@ -29,6 +51,7 @@ struct StencilGeom {
     // Window(3D) grids: `rows` counts planes, `pitch` is the plane pitch, and a
     // plane holds plane_rows rows of rpitch bytes (0 for 2-D grids)
     int64_t plane_rows = 0, rpitch = 0;
+    LaunchRec* rec = nullptr;  // filled by the launcher when non-null
 };
 
 // Output-row bands computed by one launch (1 band = all rows or interior;

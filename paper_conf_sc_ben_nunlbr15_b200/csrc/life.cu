@@ -505,6 +505,7 @@ cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_s
     }
     tma_set_link(p, link, 1);
     const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems, link != nullptr);
+    tma_record(g.rec, LK_LIFE_TMA, p, ctas, (NC + 1) * 32, smem, NS, 1, NC);
     if (ctas == 0) return cudaSuccess;
     if (link)
         life_tma_kernel<NC, NS, CM, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(p);
@@ -560,7 +561,7 @@ __global__ void life_anyw_kernel(const __grid_constant__ LifeParams p, int tail_
             const uint32_t first = __ldg(row);
             const uint32_t lastw = __ldg(row + last);
             // cell left of bit 0 of word m, and right of the word's last cell
-            uint32_t lbit, rbit;
+            uint32_t lbit;
             if (m > 0) {
                 lbit = __ldg(row + m - 1) >> 31;
             } else {

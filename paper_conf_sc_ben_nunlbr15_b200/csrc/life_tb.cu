@@ -333,7 +333,7 @@ __global__ void __maxnreg__(MAPSM_TB_REGS) life_tb_kernel(const __grid_constant_
 }
 
 template <int K, int CM>
-cudaError_t launch_tb_t(const TbParams& P0, const RowBands& b, int nc, int num_sms, cudaStream_t s) {
+cudaError_t launch_tb_t(const TbParams& P0, const RowBands& b, int nc, int num_sms, cudaStream_t s, LaunchRec* rec) {
     TbParams P = P0;
     const int smem = kNS * rows_per_stage(K) * (int)(P.strip * 4 + 32) + 2 * kNS * 8;
     auto kfn = life_tb_kernel<K, kNS, CM>;
@@ -357,6 +357,7 @@ cudaError_t launch_tb_t(const TbParams& P0, const RowBands& b, int nc, int num_s
         occ_smem[nc] = smem;
     }
     const int64_t ctas = tma_plan_grid(P.s, b, num_sms, occ[nc], (int)P.strip);
+    tma_record(rec, LK_LIFE_TB, P.s, ctas, (nc + 1) * 32, smem, kNS, rows_per_stage(K), nc, K);
     if (ctas == 0) return cudaSuccess;
     kfn<<<(unsigned)ctas, (nc + 1) * 32, smem, s>>>(P);
     cudaError_t e = cudaGetLastError();
@@ -371,11 +372,12 @@ cudaError_t launch_tb_t(const TbParams& P0, const RowBands& b, int nc, int num_s
 }
 
 template <int K>
-cudaError_t launch_tb_k(const TbParams& P, const RowBands& b, int col_mode, int nc, int num_sms, cudaStream_t s) {
+cudaError_t launch_tb_k(const TbParams& P, const RowBands& b, int col_mode, int nc, int num_sms, cudaStream_t s,
+                        LaunchRec* rec) {
     switch (col_mode) {
-        case COL_WRAP: return launch_tb_t<K, COL_WRAP>(P, b, nc, num_sms, s);
-        case COL_CLAMP: return launch_tb_t<K, COL_CLAMP>(P, b, nc, num_sms, s);
-        default: return launch_tb_t<K, COL_ZERO>(P, b, nc, num_sms, s);
+        case COL_WRAP: return launch_tb_t<K, COL_WRAP>(P, b, nc, num_sms, s, rec);
+        case COL_CLAMP: return launch_tb_t<K, COL_CLAMP>(P, b, nc, num_sms, s, rec);
+        default: return launch_tb_t<K, COL_ZERO>(P, b, nc, num_sms, s, rec);
     }
 }
 
@@ -406,11 +408,11 @@ cudaError_t launch_life_tb(const StencilGeom& g, const RowBands& b, int k, int z
     P.zero_bot = zero_bot;
     const int nc = (int)((P.strip + kOut - 1) / kOut);
     switch (k) {
-        case 2: return launch_tb_k<2>(P, b, g.col_mode, nc, num_sms, s);
-        case 3: return launch_tb_k<3>(P, b, g.col_mode, nc, num_sms, s);
-        case 4: return launch_tb_k<4>(P, b, g.col_mode, nc, num_sms, s);
-        case 6: return launch_tb_k<6>(P, b, g.col_mode, nc, num_sms, s);
-        default: return launch_tb_k<8>(P, b, g.col_mode, nc, num_sms, s);
+        case 2: return launch_tb_k<2>(P, b, g.col_mode, nc, num_sms, s, g.rec);
+        case 3: return launch_tb_k<3>(P, b, g.col_mode, nc, num_sms, s, g.rec);
+        case 4: return launch_tb_k<4>(P, b, g.col_mode, nc, num_sms, s, g.rec);
+        case 6: return launch_tb_k<6>(P, b, g.col_mode, nc, num_sms, s, g.rec);
+        default: return launch_tb_k<8>(P, b, g.col_mode, nc, num_sms, s, g.rec);
     }
 }
 

@@ -56,7 +56,83 @@ mapsm_status compute_plan(int64_t h, int g, int r, mapsm_boundary b, int rank, m
     return MAPSM_OK;
 }
 
+// The halo exchange of one pass (Alg 1's P2P copies, "two-line
+// boundary exchanges per iteration") as an ordered message list, for one
+// slab buffer laid out as [halo rows | rows owned rows | halo rows] at
+// `pitch` bytes per row.  The ISSUE ORDER is part of the contract: send-up
+// (my first `depth` rows to up), send-down (my last `depth` rows to down),
+// recv-bottom (from down into my bottom halo), recv-top (from up into my top
+// halo).  Point-to-point messages between one pair of ranks match in issue
+// order, so with g == 2 under WRAP (up == down) the peer's first receive (its
+// bottom halo) takes my first send (my top rows) — which is exactly the row
+// that follows its last row on the torus.
+int exchange_messages(const mapsm_slab_plan& p, int64_t h, int64_t depth, int64_t halo, int64_t pitch,
+                      mapsm_msg* out) {
+    int n = 0;
+    auto modh = [h](int64_t v) { int64_t m = v % h; return m < 0 ? m + h : m; };
+    auto put = [&](int kind, int peer, int64_t row) {
+        mapsm_msg m;
+        m.kind = kind;
+        m.peer = peer;
+        m.row = row;
+        m.rows = depth;
+        m.offset = (row + halo) * pitch;
+        m.bytes = depth * pitch;
+        m.global_row = modh(p.y0 + row);
+        out[n++] = m;
+    };
+    const bool top = p.top_kind == MAPSM_HALO_EXCHANGE, bot = p.bottom_kind == MAPSM_HALO_EXCHANGE;
+    if (depth <= 0) return 0;
+    if (top) put(MAPSM_MSG_SEND, p.up, 0);
+    if (bot) put(MAPSM_MSG_SEND, p.down, p.rows - depth);
+    if (bot) put(MAPSM_MSG_RECV, p.down, p.rows);
+    if (top) put(MAPSM_MSG_RECV, p.up, -depth);
+    return n;
+}
+
 }  // namespace mapsm
+
+extern "C" mapsm_status mapsm_exchange_plan(int64_t h, int g, int radius, mapsm_boundary boundary, int rank,
+                                            int64_t depth, int64_t halo, int64_t pitch, mapsm_msg* out,
+                                            int max_msgs, int* n_msgs) {
+    if (!out || !n_msgs || pitch < 1 || depth < 0 || halo < depth) return MAPSM_EINVAL;
+    mapsm_slab_plan p;
+    mapsm_status st = mapsm::compute_plan(h, g, radius, boundary, rank, &p);
+    if (st != MAPSM_OK) return st;
+    if (g > 1 && depth > h / g) return MAPSM_EINVAL;  // every halo row must belong to the neighbour
+    mapsm_msg tmp[4];
+    const int n = mapsm::exchange_messages(p, h, depth, halo, pitch, tmp);
+    *n_msgs = n;
+    if (n > max_msgs) return MAPSM_ENOMEM;
+    for (int i = 0; i < n; ++i) out[i] = tmp[i];
+    return MAPSM_OK;
+}
+
+extern "C" mapsm_status mapsm_gather_plan(int64_t h, int g, int radius, mapsm_boundary boundary, int rank, int root,
+                                          int64_t halo, int64_t pitch, mapsm_msg* out, int max_msgs, int* n_msgs) {
+    if (!out || !n_msgs || pitch < 1 || halo < 0 || root < 0 || root >= g) return MAPSM_EINVAL;
+    mapsm_slab_plan p;
+    mapsm_status st = mapsm::compute_plan(h, g, radius, boundary, rank, &p);
+    if (st != MAPSM_OK) return st;
+    int n = 0;
+    const int need = rank == root ? g - 1 : 1;
+    *n_msgs = need;
+    if (need > max_msgs) return MAPSM_ENOMEM;
+    if (rank != root) {
+        // my owned rows [0, rows) to the root
+        out[n++] = mapsm_msg{MAPSM_MSG_SEND, root, 0, p.rows, halo * pitch, p.rows * pitch, p.y0};
+    } else {
+        // the root receives every other slab, in slab order, into a staging
+        // buffer (offset 0) and places it at global row y0_k
+        for (int k = 0; k < g; ++k) {
+            if (k == root) continue;
+            mapsm_slab_plan q;
+            mapsm::compute_plan(h, g, radius, boundary, k, &q);
+            out[n++] = mapsm_msg{MAPSM_MSG_RECV, k, 0, q.rows, 0, q.rows * pitch, q.y0};
+        }
+    }
+    return MAPSM_OK;
+}
 
 extern "C" mapsm_status mapsm_plan_query(int64_t h, int g, int radius, mapsm_boundary boundary, int rank,
                                          mapsm_slab_plan* out) {

@@ -13,6 +13,9 @@
 
 namespace mapsm {
 mapsm_status compute_plan(int64_t h, int g, int r, mapsm_boundary b, int rank, mapsm_slab_plan* out);
+// The ordered halo-exchange messages of one pass (plan.cpp; <= 4); returns the count.
+int exchange_messages(const mapsm_slab_plan& p, int64_t h, int64_t depth, int64_t halo, int64_t pitch,
+                      mapsm_msg* out);
 
 // Records a thread-local error message (mapsm_last_error) and returns s.
 mapsm_status fail(mapsm_status s, const char* fmt, ...);

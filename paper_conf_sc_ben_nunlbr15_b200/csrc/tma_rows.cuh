@@ -170,9 +170,12 @@ __device__ __forceinline__ unsigned int ld_acquire_sys(const unsigned int* p) {
 
 // Producer side: before the TMA load of a halo row, wait for its delivery.
 // Bounded spin: a protocol failure traps (kernel error) instead of hanging.
+// The counters and the target (gen * r * nstrips) are taken mod 2^32; the
+// comparison is wrap-safe because a counter is never more than one
+// generation's deliveries (r * nstrips << 2^31) away from the target.
 __device__ __forceinline__ void wait_delivery(const unsigned int* counter, unsigned int target) {
     unsigned int spins = 0;
-    while (ld_acquire_sys(counter) < target) {
+    while ((int)(ld_acquire_sys(counter) - target) < 0) {
         __nanosleep(64);
         if (++spins > (1u << 26)) __trap();  // ~seconds: the neighbour never delivered
     }
@@ -377,6 +380,27 @@ inline int64_t tma_plan_grid(tma::RowStream& p, const RowBands& b, int num_sms, 
     }
     for (int i = b.nbands; i < tma::kMaxBands; ++i) p.cta_begin[i + 1] = (int)total;
     return total;
+}
+
+// Host side: describe a ring-kernel launch for mapsm_launch_query.
+inline void tma_record(LaunchRec* rec, int kernel, const tma::RowStream& p, int64_t ctas, int threads, int smem,
+                       int ns, int rows_per_stage, int consumer_warps, int gens = 1) {
+    if (!rec) return;
+    rec->kernel = kernel;
+    rec->ctas = ctas;
+    rec->threads = threads;
+    rec->smem = smem;
+    rec->ring_stages = ns;
+    rec->rows_per_stage = rows_per_stage;
+    rec->consumer_warps = consumer_warps;
+    rec->nstrips = p.nstrips;
+    rec->nbands = p.nbands;
+    for (int i = 0; i < 3; ++i) {
+        rec->begin[i] = p.begin[i];
+        rec->end[i] = p.end[i];
+    }
+    for (int i = 0; i < 4; ++i) rec->cta_begin[i] = p.cta_begin[i];
+    rec->gens = gens;
 }
 
 }  // namespace mapsm

@@ -37,8 +37,15 @@ EXPORTED = [
     "mapsm_locmon_query", "mapsm_locmon_copied", "mapsm_task_histogram", "mapsm_gather_async",
     "mapsm_grid_create_3d", "mapsm_matrix_create", "mapsm_matrix_destroy", "mapsm_matrix_bind",
     "mapsm_invoke_unmodified", "mapsm_matrix_sync", "mapsm_matrix_gather", "mapsm_routine_sgemm",
-    "mapsm_routine_saxpy",
+    "mapsm_routine_saxpy", "mapsm_launch_query", "mapsm_exchange_plan", "mapsm_gather_plan",
 ]
+MSG_SEND, MSG_RECV = 0, 1
+(KERNEL_NONE, KERNEL_LIFE_TMA, KERNEL_LIFE_REG, KERNEL_LIFE_ANYW, KERNEL_LIFE_PERSIST, KERNEL_LIFE_TB,
+ KERNEL_CONV_TMA, KERNEL_CONV_REG, KERNEL_CONV_GENERIC, KERNEL_CONV_WIDE, KERNEL_CONV3D,
+ KERNEL_LIFE_TB_PERSIST) = range(12)
+KERNEL_NAMES = {0: "none", 1: "life_tma_kernel", 2: "life_step_kernel", 3: "life_anyw_kernel",
+                4: "life_persist_kernel", 5: "life_tb_kernel", 6: "conv_tma_kernel", 7: "conv_step_kernel",
+                8: "conv_generic_kernel", 9: "conv_wide_kernel", 10: "conv3d_kernel", 11: "life_tb_persist_kernel"}
 MAX_DIMS = 3
 MAX_PARAMS = 8
 PAT_BLOCK2D, PAT_BLOCK2D_T, PAT_OUT_SI, PAT_INOUT_SI = 0, 1, 2, 3
@@ -64,6 +71,19 @@ class mapsm_grid_info(ctypes.Structure):
                 ("launches", ctypes.c_int64), ("exchanges", ctypes.c_int64), ("device_bytes", ctypes.c_int64),
                 ("used_graphs", ctypes.c_int), ("gens_per_pass", ctypes.c_int), ("halo_rows", ctypes.c_int64),
                 ("d", ctypes.c_int64)]
+
+
+class mapsm_msg(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int), ("peer", ctypes.c_int), ("row", ctypes.c_int64), ("rows", ctypes.c_int64),
+                ("offset", ctypes.c_int64), ("bytes", ctypes.c_int64), ("global_row", ctypes.c_int64)]
+
+
+class mapsm_launch_info(ctypes.Structure):
+    _fields_ = [("kernel", ctypes.c_int), ("threads", ctypes.c_int), ("smem_bytes", ctypes.c_int),
+                ("ring_stages", ctypes.c_int), ("rows_per_stage", ctypes.c_int), ("consumer_warps", ctypes.c_int),
+                ("gens_per_launch", ctypes.c_int), ("ctas", ctypes.c_int64), ("strips", ctypes.c_int64),
+                ("min_cta_seg_rows", ctypes.c_int64), ("max_cta_seg_rows", ctypes.c_int64),
+                ("min_cta_rows", ctypes.c_int64), ("segments", ctypes.c_int64)]
 
 
 class mapsm_box(ctypes.Structure):
@@ -98,6 +118,8 @@ def lib() -> ctypes.CDLL:
     P = ctypes.POINTER
     sig = {
         "mapsm_plan_query": [i64, ci, ci, ci, ci, P(mapsm_slab_plan)],
+        "mapsm_exchange_plan": [i64, ci, ci, ci, ci, i64, i64, i64, P(mapsm_msg), ci, P(ci)],
+        "mapsm_gather_plan": [i64, ci, ci, ci, ci, ci, i64, i64, P(mapsm_msg), ci, P(ci)],
         "mapsm_ctx_create": [ci, ci, ci, vp, vp, P(vp)],
         "mapsm_ctx_create_local": [ci, P(ci), P(vp)],
         "mapsm_ctx_destroy": [vp],
@@ -117,6 +139,7 @@ def lib() -> ctypes.CDLL:
         "mapsm_set_option": [vp, ci, i64],
         "mapsm_get_timing": [vp, P(ctypes.c_double), P(i64), P(ctypes.c_double), P(i64)],
         "mapsm_grid_stream": [vp, ci, P(vp)],
+        "mapsm_launch_query": [vp, ci, ci, P(mapsm_launch_info)],
         "mapsm_locmon_create": [ci, P(vp)],
         "mapsm_locmon_destroy": [vp],
         "mapsm_locmon_output": [vp, ci, ci, P(ci), P(mapsm_box), ci],
@@ -177,6 +200,27 @@ def mapsm_plan_query(h: int, g: int, radius: int, boundary: int, rank: int) -> m
     p = mapsm_slab_plan()
     _check(lib().mapsm_plan_query(h, g, radius, boundary, rank, ctypes.byref(p)), "mapsm_plan_query")
     return p
+
+
+def mapsm_exchange_plan(h: int, g: int, radius: int, boundary: int, rank: int, depth: int, halo: int,
+                        pitch: int) -> list[mapsm_msg]:
+    """The ordered halo-exchange messages of slab `rank` for one pass."""
+    out = (mapsm_msg * 4)()
+    n = ctypes.c_int()
+    _check(lib().mapsm_exchange_plan(h, g, radius, boundary, rank, depth, halo, pitch, out, 4, ctypes.byref(n)),
+           "mapsm_exchange_plan")
+    return [out[i] for i in range(n.value)]
+
+
+def mapsm_gather_plan(h: int, g: int, radius: int, boundary: int, rank: int, root: int, halo: int,
+                      pitch: int) -> list[mapsm_msg]:
+    """The gather-to-root messages of slab `rank`."""
+    cap = max(1, g)
+    out = (mapsm_msg * cap)()
+    n = ctypes.c_int()
+    _check(lib().mapsm_gather_plan(h, g, radius, boundary, rank, root, halo, pitch, out, cap, ctypes.byref(n)),
+           "mapsm_gather_plan")
+    return [out[i] for i in range(n.value)]
 
 
 def mapsm_nccl_unique_id() -> bytes:
@@ -265,21 +309,33 @@ def mapsm_read(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
     _check(lib().mapsm_read(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read")
 
 
-def mapsm_histogram(grid: int, bins=None) -> np.ndarray:
+def _is_cuda_tensor(buf) -> bool:
+    return bool(getattr(buf, "is_cuda", False))
+
+
+def mapsm_histogram(grid: int, bins=None, sync: bool = True) -> np.ndarray:
     """Reductive-Static aggregate: 256 uint64 counts (into `bins` if given:
-    a numpy array or a torch tensor, host or device)."""
+    a numpy array or a torch tensor, host or device).  For a device tensor
+    the C call is stream-ordered on the grid's stream; with sync=True (the
+    default) this wrapper waits for it (mapsm_sync) so the counts can be read
+    on any stream; sync=False leaves them pending (read after mapsm_sync)."""
     out = np.zeros(256, dtype=np.uint64) if bins is None else bins
     _check(lib().mapsm_histogram(grid, _ptr(out), 256), "mapsm_histogram")
+    if sync and _is_cuda_tensor(out):
+        mapsm_sync(grid)
     return out
 
 
-def mapsm_task_histogram(grid: int, target_slabs: int = 0, bins=None) -> tuple[np.ndarray, int]:
+def mapsm_task_histogram(grid: int, target_slabs: int = 0, bins=None, sync: bool = True) -> tuple[np.ndarray, int]:
     """Chained Reductive-Static task over the grid's current generation with
-    its own partition (0 = the grid's); returns (bins, bytes moved here)."""
+    its own partition (0 = the grid's); returns (bins, bytes moved here).
+    Device-tensor bins: as mapsm_histogram (sync=False leaves them pending)."""
     out = np.zeros(256, dtype=np.uint64) if bins is None else bins
     moved = ctypes.c_int64()
     _check(lib().mapsm_task_histogram(grid, target_slabs, _ptr(out), 256, ctypes.byref(moved)),
            "mapsm_task_histogram")
+    if sync and _is_cuda_tensor(out):
+        mapsm_sync(grid)
     return out, moved.value
 
 
@@ -415,6 +471,13 @@ def mapsm_grid_stream(grid: int, local_index: int = 0) -> int:
     return out.value or 0
 
 
+def mapsm_launch_query(grid: int, local_index: int = 0, which: int = 0) -> mapsm_launch_info:
+    """Geometry of the last bulk (which=0) or boundary (which=1) launch."""
+    out = mapsm_launch_info()
+    _check(lib().mapsm_launch_query(grid, local_index, which, ctypes.byref(out)), "mapsm_launch_query")
+    return out
+
+
 def mapsm_version() -> str:
     return lib().mapsm_version().decode()
 
@@ -498,6 +561,9 @@ class Grid:
 
     def info(self) -> mapsm_grid_info:
         return mapsm_get_info(self.handle)
+
+    def launch(self, which: int = 0, local_index: int = 0) -> mapsm_launch_info:
+        return mapsm_launch_query(self.handle, local_index, which)
 
     def set_option(self, opt: int, value: int):
         mapsm_set_option(self.handle, opt, value)
