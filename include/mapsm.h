@@ -425,10 +425,16 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         exchange exposure; results are then WRONG for g > 1)
  *   MAPSM_OPT_TIMING      1 = record CUDA events around every compute kernel
  *                         (forces direct launches); read with mapsm_get_timing
- *   MAPSM_OPT_PERSISTENT  1 (default) Life slabs without exchanged halos whose
- *                         double buffer fits in L2 (<= 64 MiB) run up to 1024
- *                         generations per cooperative launch (grid barrier
- *                         between generations); 0 = one launch per generation
+ *   MAPSM_OPT_PERSISTENT  1 (default) Life slabs without exchanged halos
+ *                         (one slab): if the double-buffered slab fits in the
+ *                         SMs' shared memory (w % 128 == 0; e.g. 8192^2), ONE
+ *                         cooperative launch runs all n generations SMEM-
+ *                         resident, K generations between neighbour-only halo
+ *                         exchanges between SMs; else, if it fits in L2
+ *                         (<= 64 MiB), up to 1024 generations per cooperative
+ *                         launch with a grid barrier between generations;
+ *                         2 = the grid-barrier kernel only; 0 = one launch per
+ *                         generation
  *   MAPSM_OPT_EXCHANGE    MAPSM_EXCHANGE_COPY (default): boundary-row kernel,
  *                         then NCCL send/recv (multi-process) or peer
  *                         cudaMemcpyAsync (single process) on a side stream,

@@ -98,6 +98,9 @@ struct Slab {
     unsigned long long* hist = nullptr;  // 256 partial counts (histogram op)
     unsigned long long* hist_acc = nullptr;  // 256 counts + CTA ticket, zero between single-launch histograms
     unsigned int* gbar = nullptr;        // grid-barrier word of the persistent Life kernel
+    uint32_t* rxbuf = nullptr;           // SMEM-resident Life: halo exchange slots
+    unsigned int* rflags = nullptr;      // ... and per-CTA pass counters
+    int64_t rxbytes = 0;
     // fused peer-memory exchange (MAPSM_OPT_EXCHANGE = P2P): my mailbox and
     // the neighbours' buffers / mailboxes (same process, or CUDA IPC)
     void* mailbox = nullptr;
@@ -133,6 +136,7 @@ struct mapsm_grid_s {
     int cur = 0;                    // buffer holding the current generation
     int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
     bool opt_graphs = true, opt_no_exchange = false, opt_timing = false, opt_persistent = true;
+    int opt_persistent_mode = 1;  // 1: SMEM-resident kernel when the slab fits, 2: grid-barrier kernel only
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
     int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
     int64_t halo = 0;           // halo rows allocated above/below each slab (r, or K*r with deep halos)
@@ -304,6 +308,8 @@ static void free_slab(Slab& s) {
     if (s.hist) cudaFree(s.hist);
     if (s.hist_acc) cudaFree(s.hist_acc);
     if (s.gbar) cudaFree(s.gbar);
+    if (s.rxbuf) cudaFree(s.rxbuf);
+    if (s.rflags) cudaFree(s.rflags);
     if (s.mailbox) cudaFree(s.mailbox);
     for (void* q : s.ipc_opened) cudaIpcCloseMemHandle(q);
     for (int b = 0; b < 2; ++b) {
@@ -900,34 +906,62 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
         if (n == 0) return MAPSM_OK;
     }
     if (n > 0) g->deep_valid = false;  // per-generation steps exchange only r rows
-    // L2-resident Life slabs with no exchanged halos: persistent kernel, up to
-    // kPersistChunk generations per cooperative launch.
-    if (g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 && g->tb_k <= 1 &&
-        !has_exchange(g->slabs[0]) && g->w % 64 == 0 && 2 * g->slabs[0].plan.alloc_rows * g->pitch <= (64ll << 20)) {
+    // Life slabs with no exchanged halos (one slab): if the double-buffered
+    // slab fits in the SMs' shared memory, ONE cooperative launch of the
+    // SMEM-resident temporally blocked kernel runs all n generations
+    // (life_resident.cu); else, if it fits in L2, the grid-barrier persistent
+    // kernel, up to kPersistChunk generations per launch.
+    const bool one_slab = g->op == MAPSM_OP_LIFE && g->opt_persistent && !g->opt_timing && g->slabs.size() == 1 &&
+                          g->tb_k <= 1 && !has_exchange(g->slabs[0]) && g->w % 64 == 0;
+    if (one_slab) {
         Slab& s = g->slabs[0];
         CK(cudaSetDevice(s.device));
-        if (!s.gbar) CK(cudaMalloc(&s.gbar, sizeof(unsigned int)));
-        const int64_t kPersistChunk = 1024;
-        for (int64_t done = 0; done < n;) {
-            const int64_t k = (n - done < kPersistChunk) ? n - done : kPersistChunk;
-            StencilGeom geom;
-            geom.in = row_ptr(g, s, g->cur, 0);
-            geom.out = row_ptr(g, s, g->cur ^ 1, 0);
-            geom.pitch = g->pitch;
-            geom.rows = s.plan.rows;
-            geom.w = g->w;
-            geom.top_map = rowmap_of(s.plan.top_kind);
-            geom.bot_map = rowmap_of(s.plan.bottom_kind);
-            geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
-            geom.rec = &s.rec_bulk;
-            cudaError_t e = launch_life_persistent(geom, k, s.gbar, s.num_sms, s.main);
-            if (e != cudaSuccess) return fail(MAPSM_ECUDA, "persistent Life launch: %s", cudaGetErrorString(e));
+        StencilGeom geom;
+        geom.in = row_ptr(g, s, g->cur, 0);
+        geom.out = row_ptr(g, s, g->cur ^ 1, 0);
+        geom.pitch = g->pitch;
+        geom.rows = s.plan.rows;
+        geom.w = g->w;
+        geom.top_map = rowmap_of(s.plan.top_kind);
+        geom.bot_map = rowmap_of(s.plan.bottom_kind);
+        geom.col_mode = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+        geom.rec = &s.rec_bulk;
+        int rctas = 0, rk = 0, rsmem = 0;
+        if (g->opt_persistent_mode != 2 && life_resident_plan(g->w, s.plan.rows, s.num_sms, &rctas, &rk, &rsmem)) {
+            const int64_t xb = life_resident_xbuf_bytes(g->w, rctas, rk);
+            if (s.rxbytes < xb) {
+                if (s.rxbuf) cudaFree(s.rxbuf);
+                if (s.rflags) cudaFree(s.rflags);
+                s.rxbuf = nullptr;
+                s.rflags = nullptr;
+                s.rxbytes = 0;
+                CK(cudaMalloc(&s.rxbuf, (size_t)xb));
+                CK(cudaMalloc(&s.rflags, sizeof(unsigned int) * (size_t)s.num_sms));
+                s.rxbytes = xb;
+            }
+            cudaError_t e = launch_life_resident(geom, n, rctas, rk, rsmem, s.rxbuf, s.rflags, s.main);
+            if (e != cudaSuccess) return fail(MAPSM_ECUDA, "resident Life launch: %s", cudaGetErrorString(e));
             g->launches++;
-            if (k & 1) g->cur ^= 1;
-            g->gen += k;
-            done += k;
+            g->cur ^= 1;  // generation n is in the other buffer, whatever the parity of n
+            g->gen += n;
+            return MAPSM_OK;
         }
-        return MAPSM_OK;
+        if (2 * s.plan.alloc_rows * g->pitch <= (64ll << 20)) {
+            if (!s.gbar) CK(cudaMalloc(&s.gbar, sizeof(unsigned int)));
+            const int64_t kPersistChunk = 1024;
+            for (int64_t done = 0; done < n;) {
+                const int64_t k = (n - done < kPersistChunk) ? n - done : kPersistChunk;
+                geom.in = row_ptr(g, s, g->cur, 0);
+                geom.out = row_ptr(g, s, g->cur ^ 1, 0);
+                cudaError_t e = launch_life_persistent(geom, k, s.gbar, s.num_sms, s.main);
+                if (e != cudaSuccess) return fail(MAPSM_ECUDA, "persistent Life launch: %s", cudaGetErrorString(e));
+                g->launches++;
+                if (k & 1) g->cur ^= 1;
+                g->gen += k;
+                done += k;
+            }
+            return MAPSM_OK;
+        }
     }
     // CUDA graphs for the single-stream-per-process modes (g == 1 and NCCL);
     // local multi-slab mode issues directly (it is the single-GPU test vehicle).
@@ -1537,7 +1571,11 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             g->opt_graph_iters = v;
             break;
         case MAPSM_OPT_NO_EXCHANGE: g->opt_no_exchange = v != 0; break;
-        case MAPSM_OPT_PERSISTENT: g->opt_persistent = v != 0; break;
+        case MAPSM_OPT_PERSISTENT:
+            if (v < 0 || v > 2) return fail(MAPSM_EINVAL, "persistent mode %lld (0, 1, 2)", (long long)v);
+            g->opt_persistent = v != 0;
+            g->opt_persistent_mode = v == 2 ? 2 : 1;
+            break;
         case MAPSM_OPT_EXCHANGE:
             if (v != MAPSM_EXCHANGE_COPY && v != MAPSM_EXCHANGE_P2P) return fail(MAPSM_EINVAL, "exchange mode %lld", (long long)v);
             if (g->state >= ST_BOUND && (v == MAPSM_EXCHANGE_P2P) != g->opt_p2p)

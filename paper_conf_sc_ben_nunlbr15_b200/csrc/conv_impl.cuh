@@ -622,6 +622,12 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
         }
         if (maxr <= 0) return cudaSuccess;
         dim3 grid((unsigned)((g.w + 127) / 128), (unsigned)(maxr < 4096 ? maxr : 4096), (unsigned)b.nbands);
+        if (g.rec) {
+            *g.rec = LaunchRec();
+            g.rec->kernel = LK_CONV_GENERIC;
+            g.rec->ctas = (int64_t)grid.x * grid.y * grid.z;
+            g.rec->threads = 128;
+        }
         conv_generic_kernel<R><<<grid, 128, 0, s>>>(p);
         return cudaGetLastError();
     }
@@ -647,6 +653,12 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
     }
     if (max_warps == 0) return cudaSuccess;
     dim3 grid((unsigned)((max_warps + kThreads / 32 - 1) / (kThreads / 32)), (unsigned)b.nbands);
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_CONV_REG;
+        g.rec->ctas = (int64_t)grid.x * grid.y;
+        g.rec->threads = kThreads;
+    }
     conv_step_kernel<R, PF><<<grid, kThreads, 0, s>>>(p);
     return cudaGetLastError();
 }

@@ -82,6 +82,16 @@ cudaError_t launch_life_step(const StencilGeom& g, const RowBands& b, int num_sm
 // of generation 0 / 1 (generation n ends in g.in if n is even, else g.out).
 // `bar` = one device word of barrier state.
 cudaError_t launch_life_persistent(const StencilGeom& g, int64_t n, unsigned int* bar, int num_sms, cudaStream_t s);
+// n generations of a whole slab (no exchanged halos) resident in SHARED
+// memory (life_resident.cu): one cooperative launch of `ctas` CTAs (one per
+// SM), K generations between neighbour-only halo exchanges through `xbuf`
+// (life_resident_xbuf_bytes) with `flags` (ctas words).  Generation n is
+// written to g.out (always, whatever the parity of n).  life_resident_plan:
+// false if the slab does not fit (w % 128, shared-memory capacity).
+bool life_resident_plan(int64_t w, int64_t rows, int num_sms, int* ctas, int* K, int* smem);
+int64_t life_resident_xbuf_bytes(int64_t w, int ctas, int K);
+cudaError_t launch_life_resident(const StencilGeom& g, int64_t n, int ctas, int K, int smem, uint32_t* xbuf,
+                                 unsigned int* flags, cudaStream_t s);
 // K generations of Life in ONE temporally blocked launch (life_tb.cu): reads
 // input rows [-K, rows+K) of g.in (halo rows must be valid to depth K; under
 // ROWMAP_CLAMP the rows outside are the MIRROR image), writes owned rows of

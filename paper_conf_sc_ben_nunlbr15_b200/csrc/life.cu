@@ -608,6 +608,12 @@ cudaError_t launch_life_anyw_t(const StencilGeom& g, const RowBands& b, cudaStre
     if (maxr <= 0) return cudaSuccess;
     const int tail = (int)(g.w - 32 * (p.nw - 1));
     dim3 grid((unsigned)((p.nw + 127) / 128), (unsigned)(maxr < 8192 ? maxr : 8192), (unsigned)b.nbands);
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_LIFE_ANYW;
+        g.rec->ctas = (int64_t)grid.x * grid.y * grid.z;
+        g.rec->threads = 128;
+    }
     life_anyw_kernel<CM><<<grid, 128, 0, s>>>(p, tail);
     return cudaGetLastError();
 }
@@ -701,6 +707,12 @@ cudaError_t launch_life_t(const StencilGeom& g, const RowBands& b, int num_sms, 
     }
     if (max_warps == 0) return cudaSuccess;
     dim3 grid((unsigned)((max_warps + kThreads / 32 - 1) / (kThreads / 32)), (unsigned)b.nbands);
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_LIFE_REG;
+        g.rec->ctas = (int64_t)grid.x * grid.y;
+        g.rec->threads = kThreads;
+    }
     life_step_kernel<V, P, CM><<<grid, kThreads, 0, s>>>(p);
     return cudaGetLastError();
 }
@@ -747,6 +759,13 @@ cudaError_t launch_life_persist_t(const StencilGeom& g, int64_t n, unsigned int*
     p.begin[1] = p.end[1] = p.nchunks[1] = 0;
     cudaError_t e = cudaMemsetAsync(bar, 0, sizeof(unsigned int), s);
     if (e != cudaSuccess) return e;
+    if (g.rec) {
+        *g.rec = LaunchRec();
+        g.rec->kernel = LK_LIFE_PERSIST;
+        g.rec->ctas = grid;
+        g.rec->threads = kPersistThreads;
+        g.rec->gens = (int)n;
+    }
     void* args[] = {(void*)&p, (void*)&n, (void*)&bar};
     return cudaLaunchCooperativeKernel((const void*)life_persist_kernel<V, P, CM>, dim3((unsigned)grid),
                                        dim3(kPersistThreads), args, 0, s);

@@ -19,8 +19,8 @@ def run(ctx, g0, n, b, steps=None, graphs=True, graph_iters=None, persistent=Tru
     with M.Grid(ctx, w, h, "life", 1, b) as g:
         if not graphs:
             g.set_option(M.OPT_GRAPHS, 0)
-        if not persistent:
-            g.set_option(M.OPT_PERSISTENT, 0)
+        if persistent is not True:
+            g.set_option(M.OPT_PERSISTENT, int(persistent))
         if graph_iters:
             g.set_option(M.OPT_GRAPH_ITERS, graph_iters)
         g.bind(g0)
@@ -49,7 +49,7 @@ def test_config0_closed_form(ctx):
 @pytest.mark.parametrize("shape", [(64, 1), (64, 2), (64, 3), (128, 130), (192, 77), (320, 64), (1024, 333),
                                    (4096, 257), (8192 + 64, 100)])
 @pytest.mark.parametrize("n", [0, 1, 2, 7])
-@pytest.mark.parametrize("persistent", [True, False])
+@pytest.mark.parametrize("persistent", [True, 2, False])
 def test_random_vs_oracle(ctx, b, shape, n, persistent):
     w, h = shape
     g0 = mi.life_u8(1000 + w + h, w, h)
@@ -108,11 +108,44 @@ def test_local_multislab_partition_invariance(local_ctx, g, b):
 
 
 def test_persistent_long_run_many_chunks(ctx):
-    """> 1024 generations: several persistent launches, odd total."""
+    """> 1024 generations on the grid-barrier persistent kernel (mode 2):
+    several launches, odd total."""
     g0 = mi.life_u8(77, 256, 96)
-    out, info = run(ctx, g0, 2051, "wrap")
+    out, info = run(ctx, g0, 2051, "wrap", persistent=2)
     assert np.array_equal(out, oracle.life(g0, 2051, "wrap"))
     assert info.launches == 3
+
+
+# ------------------------------------- SMEM-resident kernel (life_resident.cu)
+
+@pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
+@pytest.mark.parametrize("shape", [(128, 16), (256, 96), (1024, 333), (4096, 1000), (8192, 1200), (2048, 4096),
+                                   (128, 9)])
+@pytest.mark.parametrize("n", [1, 7, 8, 9, 33])
+def test_resident_vs_oracle(ctx, b, shape, n):
+    """One cooperative launch, all generations in shared memory, K generations
+    between neighbour exchanges: shapes from one CTA to all SMs with R == K
+    rows per CTA (4096x1000), ragged splits, n below / at / above K."""
+    w, h = shape
+    g0 = mi.life_u8(4000 + w + h, w, h)
+    with M.Grid(ctx, w, h, "life", 1, b) as g:
+        g.bind(g0)
+        g.iterate(n)
+        info, li = g.info(), g.launch()
+        out = g.gather()
+    assert li.kernel == M.KERNEL_LIFE_TB_PERSIST and info.launches == 1 and info.generation == n
+    assert np.array_equal(out, oracle.life(g0, n, b))
+
+
+def test_resident_split_calls_and_parity(ctx):
+    """Several iterate calls (odd and even n) keep the buffer parity right."""
+    g0 = mi.life_u8(17, 8192, 1024)
+    with M.Grid(ctx, 8192, 1024, "life", 1, "wrap") as g:
+        g.bind(g0)
+        for k in (3, 8, 1, 16, 5):
+            g.iterate(k)
+        out = g.gather()
+    assert np.array_equal(out, oracle.life(g0, 33, "wrap"))
 
 
 def test_local_multislab_min_height(local_ctx):

@@ -7,7 +7,9 @@
 #   bench[=ARGS]          python bench.py ARGS (default: the driver's default run)
 #   launches[=ARGS]       ncu launch list (gpu__time_duration) of bench.py ARGS
 #   ncu=REGEX[:ARGS]      ncu --set full of the first launch of kernels matching
-#                         REGEX while running tools/kbench.py ARGS
+#                         REGEX while running `python ARGS` (e.g.
+#                         ncu=conv_tma:tools/kbench.py,conv9,4 or
+#                         ncu=life_resident:bench.py,--workload,life8k,--steps,1)
 #   sanitize              compute-sanitizer memcheck/racecheck/synccheck of tools/sanitize_cases.py
 # ARGS use ',' for spaces (e.g. bench=--workload,conv9,--steps,5).
 set -u
@@ -27,9 +29,13 @@ for step in "$@"; do
       timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/${TAG}_smoke.log 2>&1
       echo "smoke rc=$?"; tail -2 gpurun_out/${TAG}_smoke.log ;;
     tests)
-      k=""; [ -n "$arg" ] && k="-k $arg"
-      timeout 3000 python -m pytest tests -m gpu -q --timeout 1200 $k > gpurun_out/${TAG}_pytest.log 2>&1
-      echo "pytest rc=$?"; tail -4 gpurun_out/${TAG}_pytest.log ;;
+      n=$(ls gpurun_out/${TAG}_pytest*.log 2>/dev/null | wc -l)
+      if [ -n "$arg" ]; then
+        timeout 3000 python -m pytest tests -m gpu -q --timeout 1200 -k "$arg" > gpurun_out/${TAG}_pytest$n.log 2>&1
+      else
+        timeout 3000 python -m pytest tests -m gpu -q --timeout 1200 > gpurun_out/${TAG}_pytest$n.log 2>&1
+      fi
+      echo "pytest$n rc=$?"; tail -4 gpurun_out/${TAG}_pytest$n.log ;;
     bench)
       n=$(ls gpurun_out/${TAG}_bench*.json 2>/dev/null | wc -l)
       timeout 900 python bench.py $arg > gpurun_out/${TAG}_bench$n.json 2> gpurun_out/${TAG}_bench$n.err
@@ -42,8 +48,8 @@ for step in "$@"; do
     ncu)
       re=${arg%%:*}; ka=""; [[ "$arg" == *:* ]] && ka=${arg#*:}
       n=$(ls gpurun_out/${TAG}_ncu*.ncu-rep 2>/dev/null | wc -l)
-      timeout 900 ncu --set full --clock-control none --import-source on -k regex:$re -s 2 -c 1 \
-        -o gpurun_out/${TAG}_ncu$n python tools/kbench.py $ka > gpurun_out/${TAG}_ncu$n.log 2>&1
+      timeout 900 ncu --set full --clock-control none --import-source on -k regex:$re -s ${NCU_SKIP:-2} -c 1 \
+        -o gpurun_out/${TAG}_ncu$n python $ka > gpurun_out/${TAG}_ncu$n.log 2>&1
       echo "ncu$n rc=$?"
       ncu -i gpurun_out/${TAG}_ncu$n.ncu-rep --page raw --csv > gpurun_out/${TAG}_ncu$n.raw.csv 2>/dev/null ;;
     sanitize)
