@@ -1,9 +1,13 @@
-"""bench.py — Game of Life cell-updates/s and % HBM roofline on 1..8 B200.
+"""bench.py — Game of Life cell-updates/s and % of roofline on 1..8 B200.
 
 Contract (driver): ``python bench.py --gpus N --steps K --warmup W`` (torchrun
 for N > 1) prints ONE JSON line on rank 0.  Default workload = BASELINE.json
-configs[2] at N=1 (``life64k``); ``--workload`` selects the other configs
-(``life8k``, ``conv5``, ``conv9``) and the §8(f) NEXT-1 histogram (``hist8k``).
+configs[2] at N=1 (``life64k``, the metric's configuration).  The same line
+carries, under ``configs``, every other BASELINE configuration measured under
+the same clock (``life8k`` = configs[1], ``conv5`` = configs[3], ``conv9`` =
+configs[4]), each with its own value, ms_per_step, clocks, roofline (its own
+dominant kernel and bound) and cpu_baseline.  ``--workload`` runs one
+workload alone (also the §8(f) NEXT items: ``hist8k``, ``conv3d``, ``sgemm8k``).
 
 * step      = one pass of the hot path over the resident grid: for the stencils
               one ``mapsm_iterate(grid, n)`` call (n generations: boundary rows,
@@ -16,14 +20,17 @@ configs[2] at N=1 (``life64k``); ``--workload`` selects the other configs
 * e2e       = the same metric through the public C ABI with pinned HOST buffers
               and the host<->device copies inside the timed region (mapsm_bind
               of the host rows, the step, mapsm_read / histogram to host).
-* roofline  = the dominant kernel vs the measured HBM copy bandwidth
-              (MEASURED_PEAKS.json hbm_gbs); algorithmic bytes: 0.25 B per Life
-              cell-update, 8 B per conv cell-update, 1 B per histogram pixel.
+* roofline  = the dominant kernel of the step (named from the library's launch
+              record, mapsm_launch_query) against its bound: HBM (measured copy
+              bandwidth, MEASURED_PEAKS.json hbm_gbs) for Life 65536^2 and the
+              5x5 conv; the ALU pipe for the L2/SMEM-resident 8192^2 Life; the
+              FP32 FMA pipe for the 9x9 conv.  achieved = algorithmic bytes (or
+              ops) per launch / the average launch duration over the timed
+              region (step time / launches per step, launch gaps included).
 * cpu_baseline = the CPU oracle (oracle/, OpenMP) timed on a bounded sample of
-              the same workload on rank 0 only.
-* deep_halo = (Life) the same workload on the deep-halo path (MAPSM_OPT_DEEP_HALO
-              = --deep-halo K, default 8: K generations per pass of the
-              temporally blocked kernel, K-row halos exchanged once per pass),
+              the same workload on rank 0 at N = 1.
+* deep_halo = (Life 65536^2) the deep-halo path (MAPSM_OPT_DEEP_HALO = K: K
+              generations per pass, K-row halos exchanged once per pass),
               reported separately with its ALU-pipe roofline.
 ``--impl reference`` times only the oracle (this tier's reference arm).
 """
@@ -47,9 +54,9 @@ WORKLOADS = {
                     label="Game of Life 65536x65536 WRAP, random p=0.5 (splitmix64 seed 0x5EED0003), "
                           "200 generations per step (BASELINE configs[2])"),
     "life8k": dict(op="life", w=8192, h=8192, r=1, b="wrap", n=1000, seed=0x5EED0002, wseed=None,
-                   scaling="strong", bcell=0.25,
+                   scaling="strong", bcell=0.25, single_gpu=True,
                    label="Game of Life 8192x8192 WRAP, random p=0.5 (seed 0x5EED0002), 1000 generations per step "
-                         "(BASELINE configs[1]; L2-resident)"),
+                         "(BASELINE configs[1], 1 B200; SMEM-resident)"),
     "conv5": dict(op="conv", w=16384, h=16384, r=2, b="clamp", n=500, seed=0x5EED0004, wseed=0x5EED0044,
                   scaling="strong", bcell=8.0,
                   label="fp32 5x5 window convolution 16384x16384 CLAMP, 500 iterations per step (BASELINE configs[3])"),
@@ -101,64 +108,76 @@ def load_peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks / throttle reasons sampled during the timed region."""
+    """nvidia-smi SM clocks / throttle reasons, sampled every 50 ms for the
+    whole run (started before any warm-up) with the host time of every
+    sample; ``region(t0, t1)`` summarises the samples taken inside one timed
+    region.  A region without a sample (shorter than the period) reports
+    sm_mhz = None (no off-region clock is substituted)."""
 
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
               "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+    NAMES = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
 
     def __init__(self, device_index: int):
         self.dev = device_index
         self.proc = None
-        self.lines = []
+        self.samples = []  # (host time, sm, smax, reasons)
 
     def start(self):
         try:
             self.proc = subprocess.Popen(["nvidia-smi", f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
-                                          "-lms", "100", "-i", str(self.dev)], stdout=subprocess.PIPE,
+                                          "-lms", "50", "-i", str(self.dev)], stdout=subprocess.PIPE,
                                          stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
         except Exception:
             self.proc = None
+        return self
 
     def _read(self):
         for line in self.proc.stdout:
-            self.lines.append(line.strip())
-
-    def stop(self):
-        if self.proc is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        # a timed region shorter than nvidia-smi's start-up (the histogram's
-        # ~0.3 ms) has no sample yet: take the first one right after it
-        late = not self.lines
-        t_end = time.time() + 3.0
-        while not self.lines and time.time() < t_end:
-            time.sleep(0.01)
-        self.proc.terminate()
-        try:
-            self.proc.wait(timeout=5)
-        except Exception:
-            self.proc.kill()
-        self.t.join(timeout=2)
-        sm, smax, reasons = [], [], set()
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        for ln in self.lines:
-            parts = [p.strip() for p in ln.split(",")]
+            now = time.time()
+            parts = [p.strip() for p in line.strip().split(",")]
             if len(parts) < 6:
                 continue
             try:
-                sm.append(float(parts[0]))
-                smax.append(float(parts[1]))
+                sm, smax = float(parts[0]), float(parts[1])
             except ValueError:
                 continue
-            for nm, v in zip(names, parts[2:6]):
-                if v.lower().startswith("active"):
-                    reasons.add(nm)
-        out = {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(smax) if smax else None,
-               "reasons": sorted(reasons), "samples": len(sm)}
-        if late and sm:
-            out["note"] = "timed region shorter than the sampling start-up; sampled just after it"
-        return out
+            reasons = {nm for nm, v in zip(self.NAMES, parts[2:6]) if v.lower().startswith("active")}
+            self.samples.append((now, sm, smax, reasons))
+
+    def region(self, t0, t1):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"], "samples": 0}
+        time.sleep(0.06)  # let the sample that closes the region arrive
+        inside = [s for s in list(self.samples) if t0 <= s[0] <= t1 + 0.055]
+        if not inside:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0,
+                    "note": f"no nvidia-smi sample inside the {1e3 * (t1 - t0):.0f} ms region (50 ms period)"}
+        reasons = set()
+        for s in inside:
+            reasons |= s[3]
+        return {"sm_mhz": statistics.median(s[1] for s in inside), "sm_max_mhz": max(s[2] for s in inside),
+                "reasons": sorted(reasons), "samples": len(inside)}
+
+    def stop(self):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+
+def sm_clock_for_peak(clocks):
+    """SM clock for a derived (ALU / FP32) peak: the region's median sample,
+    else MEASURED_PEAKS.json sm_max_mhz (stated in peak_source)."""
+    if clocks.get("sm_mhz"):
+        return float(clocks["sm_mhz"]), "the SM clock sampled during the timed region"
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    mhz = float(json.load(open(p)).get("sm_max_mhz", 1965.0)) if os.path.exists(p) else 1965.0
+    return mhz, "MEASURED_PEAKS.json sm_max_mhz (no clock sample inside the region)"
 
 
 # ------------------------------------------------------------------ oracle leg
@@ -212,7 +231,7 @@ def _oracle_threads(wl):
     return 1 if wl["op"] == "histogram" else oracle.num_threads()  # the histogram oracle is sequential
 
 
-def cpu_baseline(wl, budget_s=12.0):
+def cpu_baseline(wl, budget_s=8.0):
     """Time the oracle (as it stands) on a bounded sample of the workload."""
     run, units, what = _oracle_sample(wl)
     t0 = time.perf_counter()
@@ -281,10 +300,11 @@ def run_sgemm(args, wl, rank, world, local_rank):
         step()
     barrier()
     flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)
-    sampler = ClockSampler(local_rank)
-    sampler.start()
+    sampler = ClockSampler(local_rank).start()
+    time.sleep(0.3)
     total_ms, moved = 0.0, 0
     barrier()
+    t_region = time.time()
     for _ in range(args.steps):
         flush.zero_()
         e0 = torch.cuda.Event(enable_timing=True)
@@ -295,7 +315,8 @@ def run_sgemm(args, wl, rank, world, local_rank):
         e1.synchronize()
         total_ms += e0.elapsed_time(e1)
     barrier()
-    clocks = sampler.stop()
+    clocks = sampler.region(t_region, time.time())
+    sampler.stop()
     t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
     if world > 1:
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
@@ -324,7 +345,7 @@ def run_sgemm(args, wl, rank, world, local_rank):
         M.mapsm_matrix_destroy(h)
     M.mapsm_ctx_destroy(ctx)
     if rank == 0:
-        sm_mhz = clocks.get("sm_mhz") or 1965.0
+        sm_mhz, clk_src = sm_clock_for_peak(clocks)
         peak = 148 * 128 * 2 * sm_mhz * 1e6 / 1e12
         ach = value / world / 1e12
         cb = None
@@ -357,7 +378,7 @@ def run_sgemm(args, wl, rank, world, local_rank):
                 "moved_bytes": {"first_call": int(first_moved), "timed_region": int(moved)},
                 "roofline": {"bound": "fma", "kernel": "cuBLAS SGEMM (fp32 CUDA-core FMA, no TF32)", "achieved": ach,
                              "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
-                             "peak_source": "148 SMs x 128 FP32 lanes x 2 flop x sampled SM clock (nominal)"},
+                             "peak_source": f"148 SMs x 128 FP32 lanes x 2 flop x {sm_mhz:.0f} MHz ({clk_src})"},
                 "clocks": clocks, "cpu_baseline": cb,
                 "paper_context": "Table 4 P:L503-508: single-GPU 8K multiplication 245-366 ms on GTX 780/Titan "
                                  "Black/GTX 980 (CUBLAS over MAPS-Multi 248.62 ms on GTX 980)"}
@@ -401,6 +422,318 @@ def run_reference(args, wl, rank, world):
 
 # ------------------------------------------------------------------ GPU leg
 
+SUB_CONFIGS = ["life8k", "conv5", "conv9"]  # BASELINE configs[1], [3], [4] beside the headline configs[2]
+ALU_OPS_PER_WORD = 12  # Life: 2 funnel shifts + 2 LOP3 (3-cell row sum) + 8 LOP3 (rule) per 32-cell word
+
+
+class Env:
+    """Per-process GPU state shared by every measured workload."""
+
+    def __init__(self, args, rank, world, local_rank):
+        import torch
+        import torch.distributed as dist
+
+        from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
+
+        self.torch, self.dist, self.M = torch, dist, M
+        self.args, self.rank, self.world, self.local_rank = args, rank, world, local_rank
+        torch.cuda.set_device(local_rank)
+        self.dev = torch.device("cuda", local_rank)
+        if world > 1:
+            dist.init_process_group("nccl", device_id=self.dev)
+        # A dedicated (non-default) stream: libmapsm launches on it, and the CUDA
+        # events of the timed regions are recorded on it.
+        self.stream = torch.cuda.Stream(device=self.dev)
+        torch.cuda.set_stream(self.stream)
+        uid = None
+        if world > 1:
+            obj = [M.mapsm_nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            uid = obj[0]
+        self.ctx = M.mapsm_ctx_create(rank, world, local_rank, uid, self.stream.cuda_stream)
+        self.flush = torch.empty(256 << 20, dtype=torch.uint8, device=self.dev)  # > 126 MB L2
+        self.sampler = ClockSampler(local_rank).start()
+
+    def barrier(self):
+        if self.world > 1:
+            self.dist.barrier(device_ids=[self.local_rank])
+        self.torch.cuda.synchronize()
+
+    def max_over_ranks(self, x, dtype=None):
+        t = self.torch.tensor([x], dtype=dtype or self.torch.float64, device=self.dev)
+        if self.world > 1:
+            self.dist.all_reduce(t, op=self.dist.ReduceOp.MAX)
+        return t.item()
+
+    def sum_over_ranks(self, x):
+        t = self.torch.tensor([x], dtype=self.torch.int64, device=self.dev)
+        if self.world > 1:
+            self.dist.all_reduce(t, op=self.dist.ReduceOp.SUM)
+        return int(t.item())
+
+    def timed(self, fn, steps, flush=True):
+        """K steps, each bracketed by CUDA events on the library's stream, L2
+        flushed before each step outside the events; returns (sum ms, t0, t1)."""
+        torch = self.torch
+        total = 0.0
+        self.barrier()
+        t0 = time.time()
+        for _ in range(steps):
+            if flush:
+                self.flush.zero_()
+            e0 = torch.cuda.Event(enable_timing=True)
+            e1 = torch.cuda.Event(enable_timing=True)
+            e0.record(self.stream)
+            fn()
+            e1.record(self.stream)
+            e1.synchronize()
+            total += e0.elapsed_time(e1)
+        self.barrier()
+        return total, t0, time.time()
+
+    def close(self):
+        self.M.mapsm_ctx_destroy(self.ctx)
+        self.sampler.stop()
+        if self.world > 1:
+            self.dist.barrier(device_ids=[self.local_rank])
+            self.dist.destroy_process_group()
+
+
+def host_input(env, wl, rows, y0):
+    """Pinned host rows [y0, y0+rows) of the workload's synthetic input."""
+    import mapsm_inputs as mi
+
+    torch = env.torch
+    d = wl.get("d", 0)
+    w, h = wl["w"], wl["h"]
+    dt = torch.float32 if wl["op"] == "conv" else torch.uint8
+    t = torch.empty((rows, h, w) if d else (rows, w), dtype=dt, pin_memory=True)
+    if d:
+        t.numpy()[:] = mi.volume_f32(wl["seed"], w, h, rows, z0=y0)
+    elif wl["op"] == "life":
+        mi.life_u8(wl["seed"], w, rows, y0=y0, out=t.numpy())
+    elif wl["op"] == "conv":
+        mi.field_f32(wl["seed"], w, rows, y0=y0, out=t.numpy())
+    else:
+        mi.image_u8(wl["seed"], w, rows, y0=y0, out=t.numpy())
+    return t
+
+
+def roofline_of(env, name, wl, kernel, cells_launch, t_launch_s, clocks, launch_unit):
+    """The dominant kernel's roofline: algorithmic work of one launch over the
+    average launch duration in the timed region."""
+    peak_gbs, peak_src = load_peaks()
+    bcell = wl["bcell"]
+    hbm_ach = bcell * cells_launch / t_launch_s / 1e9
+    hbm = {"achieved": hbm_ach, "peak": peak_gbs, "unit": "GB/s", "frac": hbm_ach / peak_gbs,
+           "bytes_per_unit": bcell, "peak_source": peak_src}
+    traffic = None
+    tfile = os.path.join(ROOT, "profiles", "traffic.json")
+    if os.path.exists(tfile):
+        try:
+            traffic = json.load(open(tfile)).get(name)
+        except Exception:
+            traffic = None
+    base = {"kernel": kernel, "launch_unit": launch_unit, "ms_per_launch": t_launch_s * 1e3, "traffic": traffic}
+    mhz, clk_src = sm_clock_for_peak(clocks)
+    if wl["op"] == "life" and kernel in ("life_tb_persist_kernel", "life_persist_kernel", "life_tb_kernel"):
+        # L2 / SMEM resident (or temporally blocked): bound by the ALU pipe
+        ach = cells_launch * ALU_OPS_PER_WORD / 32 / t_launch_s / 1e12
+        peak = 148 * 64 * mhz * 1e6 / 1e12
+        return {"bound": "alu", **base, "achieved": ach, "peak": peak, "unit": "T ALU lane-ops/s", "frac": ach / peak,
+                "ops_per_unit": ALU_OPS_PER_WORD / 32,
+                "algorithmic_ops_per_launch": cells_launch * ALU_OPS_PER_WORD / 32,
+                "peak_source": f"148 SMs x 64 ALU lanes/clk x {mhz:.0f} MHz ({clk_src}; B200_PROFILING.md unit "
+                               "counts, LOP3/SHF issue measured with tools/pipebench.cu)",
+                "hbm_equivalent": {**hbm, "note": "working set resident in L2 / shared memory: the HBM "
+                                                  "fraction is not a bound (it can exceed 1)"}}
+    if wl["op"] == "conv":
+        fma_cell = (2 * wl["r"] + 1) ** (3 if wl.get("d") else 2)
+        if fma_cell / bcell > 5.7:  # above the FMA/HBM balance (37.2 TFMA/s / 6.5 TB/s): FP32-FMA bound
+            ach = 2.0 * fma_cell * cells_launch / t_launch_s / 1e12
+            peak = 148 * 128 * 2 * mhz * 1e6 / 1e12
+            return {"bound": "alu", **base, "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
+                    "flops_per_unit": 2.0 * fma_cell, "algorithmic_flops_per_launch": 2.0 * fma_cell * cells_launch,
+                    "peak_source": f"derived: 148 SM x 128 FP32 FMA/clk x 2 flop x {mhz:.0f} MHz ({clk_src}; "
+                                   "B200_PROFILING.md unit counts; FFMA2 issue measured with tools/pipebench3.cu)",
+                    "hbm": hbm, "note": f"FP32-FMA bound ({fma_cell / bcell:.2f} FMA/B > 5.7 balance)"}
+    return {"bound": "hbm", **base, "achieved": hbm_ach, "peak": peak_gbs, "unit": "GB/s",
+            "frac": hbm_ach / peak_gbs, "frac_vs_8TBps_spec": hbm_ach / 8000.0, "bytes_per_unit": bcell,
+            "algorithmic_bytes_per_launch": bcell * cells_launch, "peak_source": peak_src}
+
+
+def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=False):
+    """One workload: K timed steps + e2e (+ the headline's extras)."""
+    M, torch, args = env.M, env.torch, env.args
+    world, rank = env.world, env.rank
+    op = wl["op"]
+    w = wl["w"]
+    h = wl["h"] * (world if wl["scaling"] == "weak" else 1)
+    n = wl["n"]
+    d = wl.get("d", 0)
+    if op == "conv":
+        import mapsm_inputs as mi
+        W = mi.weights3d_f32(wl["wseed"], wl["r"]) if d else mi.weights_f32(wl["wseed"], wl["r"])
+    else:
+        W = None
+    grid = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, d=d)
+    cpu_ = w * (h if d else 1)             # cells per partition unit (row or plane)
+    cells_total = w * h * (d if d else 1)
+    if args.graph_iters:
+        grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
+    y0, rows = grid.local_rows()
+    h_in = host_input(env, {**wl, "h": h}, rows, y0)
+    h_out = torch.empty_like(h_in, pin_memory=True) if op != "histogram" else None
+    d_bins = torch.zeros(256, dtype=torch.int64, device=env.dev)
+    h_bins = torch.zeros(256, dtype=torch.int64, pin_memory=True)
+    grid.bind(h_in)
+    info0 = grid.info()
+
+    def step():
+        if op == "histogram":
+            M.mapsm_histogram(grid.handle, d_bins, sync=False)
+        else:
+            grid.iterate(n)
+
+    for _ in range(warmup):
+        step()
+    env.barrier()
+    if min_region_s > 0:  # sub-configurations: at least min_region_s of timed steps (clock samples)
+        one, _, _ = env.timed(step, 1)
+        one = env.max_over_ranks(one)
+        steps = max(steps, min(400, int(min_region_s * 1e3 / max(one, 1e-3)) + 1))
+    launches0 = grid.info().launches
+    total_ms, t0, t1 = env.timed(step, steps)
+    clocks = env.sampler.region(t0, t1)
+    launches = grid.info().launches - launches0
+    used_graphs = bool(grid.info().used_graphs)
+    total_ms = env.max_over_ranks(total_ms)
+    total_launches = env.sum_over_ranks(launches)
+    units_per_step = cells_total * n
+    value = units_per_step * steps / (total_ms / 1e3)
+    ms_per_step = total_ms / steps
+    li = grid.launch(0)
+    kernel = M.KERNEL_NAMES.get(li.kernel, "?") if op != "histogram" else "histogram_kernel"
+    slab_cells = rows * cpu_
+    # the unit of the roofline: one launch of the dominant kernel.  At N = 1
+    # every generation is one launch (or a whole persistent step is one);
+    # with exchanged halos a generation is boundary + interior launches + the
+    # exchange, and the generation is the unit.
+    per_process_launches = max(1, launches // steps)
+    if op == "histogram":
+        gens_per_launch, unit = 1, "one histogram call (one launch)"
+    elif li.gens_per_launch > 1 and per_process_launches == 1:
+        gens_per_launch, unit = n, f"one launch = {n} generations (SMEM-resident persistent kernel)"
+    elif per_process_launches == n:
+        gens_per_launch, unit = 1, "one launch = one generation"
+    else:
+        gens_per_launch, unit = 1, "one generation (boundary + interior launches + halo exchange)"
+    t_launch = (ms_per_step / 1e3) / (n / gens_per_launch)
+    roofline = roofline_of(env, name, wl, kernel, slab_cells * gens_per_launch, t_launch, clocks, unit)
+
+    exposure = None
+    if world > 1 and op != "histogram":  # halo-exchange exposure: the same steps without the exchange
+        grid.set_option(M.OPT_NO_EXCHANGE, 1)
+        grid.iterate(n)
+        ne_ms, _, _ = env.timed(step, 2, flush=False)
+        ne = env.max_over_ranks(ne_ms) / 2
+        grid.set_option(M.OPT_NO_EXCHANGE, 0)
+        exposure = {"ms_per_step_no_exchange": ne, "exposed_pct": 100.0 * (ms_per_step - ne) / ms_per_step}
+
+    # e2e: host buffers through the public API, copies inside the timed region
+    def e2e_step():
+        grid.bind(h_in)
+        if op == "histogram":
+            M.mapsm_histogram(grid.handle, h_bins)
+        else:
+            grid.iterate(n)
+            M.mapsm_read(grid.handle, h_out, grid._rp(h_out))
+
+    e2e_ms, _, _ = env.timed(e2e_step, e2e_steps, flush=False)
+    e2e_value = units_per_step * e2e_steps / (env.max_over_ranks(e2e_ms) / 1e3)
+    elem = 4 if op == "conv" else 1
+    h2d = cells_total * elem
+    d2h = 256 * 8 * world if op == "histogram" else cells_total * elem
+
+    chained = deep = None
+    if extras and op != "histogram":
+        # Chained task (SURVEY §8(f) NEXT-3): a Reductive-Static histogram of the
+        # current generation, data movement inferred by Alg 2 (0 bytes on the
+        # grid's own partition); whole call timed after an L2 flush.
+        d_b = torch.zeros(256, dtype=torch.int64, device=env.dev)
+        _, moved = M.mapsm_task_histogram(grid.handle, 0, d_b)
+        c_ms, _, _ = env.timed(lambda: M.mapsm_task_histogram(grid.handle, 0, d_b, sync=False), steps)
+        c_s = env.max_over_ranks(c_ms) / 1e3 / steps
+        peak_gbs, _ = load_peaks()
+        tb = 0.125 if op == "life" else 4.0
+        ach = tb * rows * cpu_ / c_s / 1e9
+        chained = {"task": "histogram of the current generation (mapsm_task_histogram, grid's own partition)",
+                   "moved_bytes": int(moved), "ms_per_call": c_s * 1e3, "cells_per_s": cells_total / c_s,
+                   "roofline": {"bound": "hbm", "kernel": "histogram_life_kernel" if op == "life"
+                                else "histogram_f32_kernel", "bytes_per_unit": tb, "achieved": ach,
+                                "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
+                                "note": "whole call timed (kernel + bins, one launch)"}}
+    grid.close()
+    if extras and op == "life" and args.deep_halo > 1:
+        # Deep halos (SURVEY §8(f) NEXT-2): K generations per pass, K-row halos
+        # once per pass — reported separately (not the per-iteration exchange
+        # of the north_star design; bound by the ALU pipe, not HBM).
+        K = args.deep_halo
+        dg = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], None, deep_halo=K)
+        dg.bind(h_in)
+        for _ in range(warmup):
+            dg.iterate(n)
+        dl0 = dg.info().launches
+        d_ms, dt0, dt1 = env.timed(lambda: dg.iterate(n), steps)
+        dclocks = env.sampler.region(dt0, dt1)
+        dinfo = dg.info()
+        dl = (dinfo.launches - dl0) // steps
+        dg.close()
+        d_ms = env.max_over_ranks(d_ms)
+        d_value = units_per_step * steps / (d_ms / 1e3)
+        passes = n // K
+        t_pass = (d_ms / steps / 1e3) / max(1, passes)
+        droof = roofline_of(env, name, wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
+                            f"one pass = {K} generations ({dl} launches per step)")
+        deep = {"generations_per_pass": int(dinfo.gens_per_pass), "halo_rows": int(dinfo.halo_rows),
+                "value": d_value, "unit": metric_of(wl)[1], "ms_per_step": d_ms / steps,
+                "vs_per_generation_path": d_value / value, "roofline": droof, "clocks": dclocks,
+                "hbm_bytes_per_cell_update": 0.25 / K}
+
+    metric, unit_name = metric_of(wl)
+    nbuf = 1 if op == "histogram" else 2
+    ws_mib = nbuf * (rows + 2 * wl["r"]) * info0.pitch_bytes / 2**20
+    dtype = {"life": "u32 bit-sliced (1 bit/cell)", "conv": "f32", "histogram": "u8 in, u32/u64 counts"}[op]
+    para = f"row-slab x{world}"
+    if world > 1:
+        para += " + NCCL allreduce of bins" if op == "histogram" else " + NCCL halo exchange"
+    line = {
+        "metric": metric, "value": value, "unit": unit_name, "n_gpus": world, "steps": steps,
+        "warmup": warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
+        "scaling": wl["scaling"], "vs_baseline": None, "dtype": dtype, "data": "synthetic",
+        "config": {"workload": wl["label"], "w": w, "h": h, **({"d": d} if d else {}),
+                   "iterations_per_step": n, "radius": wl["r"], "boundary": wl["b"], "parallelism": para,
+                   "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU working set "
+                         f"{ws_mib:.0f} MiB vs 126 MB L2", "cuda_graphs": used_graphs,
+                   "kernel": kernel, "launch": {"ctas": int(li.ctas), "threads": int(li.threads),
+                                                "smem_bytes": int(li.smem_bytes),
+                                                "ring_stages": int(li.ring_stages)}},
+        "e2e": {"value": e2e_value, "unit": unit_name, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "how": ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step" if op == "histogram"
+                        else "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")},
+        "gpu_launches": total_launches,
+        "roofline": roofline,
+        "clocks": clocks,
+    }
+    if exposure is not None:
+        line["halo_exposure"] = exposure
+    if deep is not None:
+        line["deep_halo"] = deep
+    if chained is not None:
+        line["chained_task"] = chained
+    return line
+
+
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -410,9 +743,10 @@ def main():
     ap.add_argument("--workload", default="life64k", choices=sorted(WORKLOADS))
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-configs", action="store_true", help="headline only (no BASELINE sub-configurations)")
     ap.add_argument("--graph-iters", type=int, default=0)
     ap.add_argument("--deep-halo", type=int, default=8,
-                    help="Life workloads: also measure the deep-halo path with K generations per pass "
+                    help="Life 65536^2: also measure the deep-halo path with K generations per pass "
                          "(reported under 'deep_halo'; 0/1 = skip)")
     args = ap.parse_args()
     wl = dict(WORKLOADS[args.workload])
@@ -427,345 +761,29 @@ def main():
         run_sgemm(args, wl, rank, world, local_rank)
         return
 
-    import torch
-    import torch.distributed as dist
-
-    import mapsm_inputs as mi
-    from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
-
-    torch.cuda.set_device(local_rank)
-    dev = torch.device("cuda", local_rank)
-    if world > 1:
-        dist.init_process_group("nccl", device_id=dev)
-    # A dedicated (non-default) stream: libmapsm launches on it, and the CUDA
-    # events of the timed region are recorded on it.
-    stream = torch.cuda.Stream(device=dev)
-    torch.cuda.set_stream(stream)
-    uid = None
-    if world > 1:
-        obj = [M.mapsm_nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        uid = obj[0]
-    ctx = M.mapsm_ctx_create(rank, world, local_rank, uid, stream.cuda_stream)
-
-    op = wl["op"]
-    w = wl["w"]
-    h = wl["h"] * (world if wl["scaling"] == "weak" else 1)
-    n = wl["n"]
-    d = wl.get("d", 0)   # Window(3D): partition units are planes of h rows
-    if op == "conv":
-        W = mi.weights3d_f32(wl["wseed"], wl["r"]) if d else mi.weights_f32(wl["wseed"], wl["r"])
-    else:
-        W = None
-    grid = M.Grid(ctx, w, h, op, wl["r"], wl["b"], W, d=d)
-    cpu_ = w * (h if d else 1)             # cells per partition unit (row or plane)
-    cells_total = w * h * (d if d else 1)
-    if args.graph_iters:
-        grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
-    y0, rows = grid.local_rows()
-    host_dtype = torch.float32 if op == "conv" else torch.uint8
-    # pinned host rows of this rank (input and result buffers for e2e)
-    h_in = torch.empty((rows, h, w) if d else (rows, w), dtype=host_dtype, pin_memory=True)
-    if d:
-        h_in.numpy()[:] = mi.volume_f32(wl["seed"], w, h, rows, z0=y0)
-    elif op == "life":
-        mi.life_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
-    elif op == "conv":
-        mi.field_f32(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
-    else:
-        mi.image_u8(wl["seed"], w, rows, y0=y0, out=h_in.numpy())
-    h_out = torch.empty_like(h_in, pin_memory=True) if op != "histogram" else None
-    d_bins = torch.zeros(256, dtype=torch.int64, device=dev)
-    h_bins = torch.zeros(256, dtype=torch.int64, pin_memory=True)
-    grid.bind(h_in)
-    info0 = grid.info()
-    flush = torch.empty(256 << 20, dtype=torch.uint8, device=dev)  # > 126 MB L2
-
-    def step():
-        if op == "histogram":
-            M.mapsm_histogram(grid.handle, d_bins, sync=False)
-        else:
-            grid.iterate(n)
-
-    def barrier():
-        if world > 1:
-            dist.barrier(device_ids=[local_rank])
-        torch.cuda.synchronize()
-
-    # warm-up (graph capture, NCCL connections, clocks)
-    for _ in range(args.warmup):
-        step()
-    barrier()
-
-    # timed region: K steps, L2 flushed between steps outside the events
-    sampler = ClockSampler(local_rank)
-    sampler.start()
-    launches0 = grid.info().launches
-    total_ms = 0.0
-    barrier()
-    for _ in range(args.steps):
-        flush.zero_()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        step()
-        e1.record(stream)
-        e1.synchronize()
-        total_ms += e0.elapsed_time(e1)
-    barrier()
-    clocks = sampler.stop()
-    launches = grid.info().launches - launches0
-    used_graphs = bool(grid.info().used_graphs)
-    t = torch.tensor([total_ms], dtype=torch.float64, device=dev)
-    tl = torch.tensor([launches], dtype=torch.int64, device=dev)
-    if world > 1:
-        dist.all_reduce(t, op=dist.ReduceOp.MAX)
-        dist.all_reduce(tl, op=dist.ReduceOp.SUM)
-    total_ms = float(t.item())
-    total_launches = int(tl.item())
-    units_per_step = cells_total * n
-    value = units_per_step * args.steps / (total_ms / 1e3)
-    ms_per_step = total_ms / args.steps
-
-    peak_gbs, peak_src = load_peaks()
-    bcell = wl["bcell"]
-    slab_cells = rows * cpu_
-    # achieved over the timed region: each stencil step is n back-to-back bulk
-    # launches (N == 1), the histogram step one launch (plus its aggregation)
-    bulk_launches_per_step = n if op != "histogram" else 1
-    per_launch_s = (total_ms / 1e3) / (args.steps * bulk_launches_per_step)
-    achieved_region = bcell * slab_cells / per_launch_s / 1e9
-    kernel = {"life": "life_tma_kernel", "conv": "conv3d_kernel" if d else "conv_tma_kernel",
-              "histogram": "histogram_kernel"}[op]
-    roofline = {"bound": "hbm", "peak": peak_gbs, "unit": "GB/s", "kernel": kernel,
-                "bytes_per_unit": bcell, "algorithmic_bytes_per_launch": bcell * slab_cells, "peak_source": peak_src}
-    per_kernel_s = None
-    if op != "histogram":
-        # CUDA events around every bulk launch on the launching stream
-        # (direct launches, same kernels and configuration) for one step
-        grid.set_option(M.OPT_TIMING, 1)
-        grid.iterate(n)
-        bulk_ms, bulk_n, bnd_ms, bnd_n = M.mapsm_get_timing(grid.handle)
-        grid.set_option(M.OPT_TIMING, 0)
-        bulk_rows = rows if bnd_n == 0 else rows - 2 * wl["r"]
-        per_kernel_s = (bulk_ms / 1e3) / max(1, bulk_n)
-        achieved_kernel = bcell * bulk_rows * cpu_ / per_kernel_s / 1e9
-        roofline["achieved_events_per_launch_GBps"] = achieved_kernel
-        roofline["kernel_ms_per_launch"] = per_kernel_s * 1e3
-        achieved = achieved_region if world == 1 else achieved_kernel
-    else:
-        achieved = achieved_region
-        roofline["note"] = ("whole step timed (memset + kernel + aggregation + bins copy); the 64 MiB image "
-                            "is re-read from HBM after each L2 flush")
-    roofline["achieved"] = achieved
-    roofline["frac"] = achieved / peak_gbs
-    roofline["frac_vs_8TBps_spec"] = achieved / 8000.0
-    roofline["traffic"] = None
-    tfile = os.path.join(ROOT, "profiles", "traffic.json")
-    if os.path.exists(tfile):
-        try:
-            roofline["traffic"] = json.load(open(tfile)).get(args.workload)
-        except Exception:
-            pass
-    if op == "conv":
-        fma_per_cell = (2 * wl["r"] + 1) ** (3 if d else 2)
-        sm_mhz = clocks.get("sm_mhz") or 1965.0
-        fma_peak = 148 * 128 * sm_mhz * 1e6
-        roofline["fma_frac_at_sampled_clock"] = (bulk_rows * cpu_ * fma_per_cell / per_kernel_s) / fma_peak
-        if fma_per_cell / 8.0 > 5.7:   # above the FMA/HBM balance (37.2 TFMA/s / 6.5 TB/s)
-            # FMA-bound: the binding roofline is the FP32 FMA pipe,
-            # 148 SMs x 128 FMA/clk x 2 flop x the SM clock sampled during the run
-            # (guide unit counts; nominal, not measured). The HBM figures stay as
-            # secondary keys.
-            flops_per_cell = 2.0 * fma_per_cell
-            t_launch = per_launch_s if world == 1 else per_kernel_s
-            rows_launch = slab_cells if world == 1 else bulk_rows * cpu_
-            alu_ach = flops_per_cell * rows_launch / t_launch / 1e12
-            alu_peak = 2.0 * fma_peak / 1e12
-            roofline = {"bound": "alu", "kernel": kernel, "achieved": alu_ach, "peak": alu_peak,
-                        "unit": "TFLOP/s", "frac": alu_ach / alu_peak,
-                        "flops_per_unit": flops_per_cell,
-                        "algorithmic_flops_per_launch": flops_per_cell * rows_launch,
-                        "peak_source": (f"derived: 148 SM x 128 FP32 FMA/clk x 2 flop x {sm_mhz:.0f} MHz "
-                                        "(sampled SM clock; B200_PROFILING.md unit counts)"),
-                        "traffic": roofline["traffic"],
-                        "hbm": {"achieved": achieved, "peak": peak_gbs, "unit": "GB/s",
-                                "frac": achieved / peak_gbs, "bytes_per_unit": bcell,
-                                "peak_source": peak_src},
-                        "kernel_ms_per_launch": per_kernel_s * 1e3,
-                        "note": f"FP32-FMA bound ({fma_per_cell / 8.0:.2f} FMA/B > 5.7 balance)"}
-
-    # halo-exchange exposure (N > 1): same steps without the exchange
-    exposure = None
-    if world > 1 and op != "histogram":
-        grid.set_option(M.OPT_NO_EXCHANGE, 1)
-        grid.iterate(n)
-        barrier()
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        e0.record(stream)
-        grid.iterate(n)
-        e1.record(stream)
-        barrier()
-        tt = torch.tensor([e0.elapsed_time(e1)], dtype=torch.float64, device=dev)
-        dist.all_reduce(tt, op=dist.ReduceOp.MAX)
-        grid.set_option(M.OPT_NO_EXCHANGE, 0)
-        exposure = {"ms_per_step_no_exchange": float(tt.item()),
-                    "exposed_pct": 100.0 * (ms_per_step - float(tt.item())) / ms_per_step}
-
-    # e2e: host buffers through the public API, copies inside the timed region
-    e2e_ms = 0.0
-    barrier()
-    for _ in range(args.e2e_steps):
-        e0 = torch.cuda.Event(enable_timing=True)
-        e1 = torch.cuda.Event(enable_timing=True)
-        barrier()
-        e0.record(stream)
-        grid.bind(h_in)
-        if op == "histogram":
-            M.mapsm_histogram(grid.handle, h_bins)
-        else:
-            grid.iterate(n)
-            M.mapsm_read(grid.handle, h_out, grid._rp(h_out))
-        e1.record(stream)
-        e1.synchronize()
-        e2e_ms += e0.elapsed_time(e1)
-    te = torch.tensor([e2e_ms], dtype=torch.float64, device=dev)
-    if world > 1:
-        dist.all_reduce(te, op=dist.ReduceOp.MAX)
-    e2e_value = units_per_step * args.e2e_steps / (float(te.item()) / 1e3)
-    elem = 4 if op == "conv" else 1
-    h2d = cells_total * elem
-    d2h = 256 * 8 * world if op == "histogram" else cells_total * elem
-
-    # Chained task: a Reductive-Static histogram task over
-    # the current generation, its data movement inferred by the Segment Location
-    # Monitor (Alg 2) — 0 bytes on the grid's own partition.  Timed per call
-    # (memset + kernel + aggregation + bins copy), after an L2 flush.
-    chained = None
-    if op != "histogram":
-        d_b = torch.zeros(256, dtype=torch.int64, device=dev)
-        _, moved = M.mapsm_task_histogram(grid.handle, 0, d_b)
-        c_ms = 0.0
-        for _ in range(args.steps):
-            flush.zero_()
-            e0 = torch.cuda.Event(enable_timing=True)
-            e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            M.mapsm_task_histogram(grid.handle, 0, d_b, sync=False)
-            e1.record(stream)
-            e1.synchronize()
-            c_ms += e0.elapsed_time(e1)
-        tc = torch.tensor([c_ms], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(tc, op=dist.ReduceOp.MAX)
-        c_s = float(tc.item()) / 1e3 / args.steps
-        tb = 0.125 if op == "life" else 4.0   # bytes read per cell (1 bit / one fp32)
-        ach = tb * rows * cpu_ / c_s / 1e9
-        chained = {"task": "histogram of the current generation (mapsm_task_histogram, grid's own partition)",
-                   "moved_bytes": int(moved), "ms_per_call": c_s * 1e3, "cells_per_s": cells_total / c_s,
-                   "roofline": {"bound": "hbm", "kernel": "histogram_life_kernel" if op == "life"
-                                else "histogram_f32_kernel", "bytes_per_unit": tb, "achieved": ach,
-                                "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
-                                "note": "whole call timed (memset + kernel + bins copy + sync)"}}
-
-    grid.close()
-
-    # Deep halos    grid.close()
-
-    # Deep halos (MAPSM_OPT_DEEP_HALO): the same workload
-    # with K generations per pass and K-row halos exchanged once per pass —
-    # reported separately because it is not the per-iteration exchange of the
-    # north_star design and is bound by the ALU pipe, not HBM.
-    deep = None
-    if op == "life" and args.deep_halo > 1:
-        K = args.deep_halo
-        dg = M.Grid(ctx, w, h, op, wl["r"], wl["b"], None, deep_halo=K)
-        dg.bind(h_in)
-        for _ in range(args.warmup):
-            dg.iterate(n)
-        barrier()
-        d_ms = 0.0
-        for _ in range(args.steps):
-            flush.zero_()
-            e0 = torch.cuda.Event(enable_timing=True)
-            e1 = torch.cuda.Event(enable_timing=True)
-            e0.record(stream)
-            dg.iterate(n)
-            e1.record(stream)
-            e1.synchronize()
-            d_ms += e0.elapsed_time(e1)
-        dinfo = dg.info()
-        # per-launch kernel time of the temporally blocked kernel (direct launches)
-        dg.set_option(M.OPT_TIMING, 1)
-        dg.iterate(n - n % K)
-        b_ms, b_n, bb_ms, bb_n = M.mapsm_get_timing(dg.handle)
-        dg.set_option(M.OPT_TIMING, 0)
-        dg.close()
-        td = torch.tensor([d_ms], dtype=torch.float64, device=dev)
-        if world > 1:
-            dist.all_reduce(td, op=dist.ReduceOp.MAX)
-        d_ms = float(td.item())
-        d_value = units_per_step * args.steps / (d_ms / 1e3)
-        # ALU roofline: 12 ALU-pipe ops (2 funnel shifts + 2 LOP3 for the
-        # 3-cell row sum, 8 LOP3 for the rule) per 32-cell word per generation;
-        # the ALU pipe retires 64 lanes/clk/SM (tools/pipebench.cu: LOP3 and
-        # SHF ~1.9 warp-instructions/clk/SM).
-        sm_mhz = clocks.get("sm_mhz") or 1965.0
-        alu_peak = 148 * 64 * sm_mhz * 1e6 / 1e12  # T lane-ops/s
-        kern_s = (b_ms / 1e3) / max(1, b_n)
-        bulk_rows = rows if bb_n == 0 else rows - 2 * K
-        cells_per_launch = bulk_rows * w * K
-        alu_achieved = cells_per_launch * 12 / 32 / kern_s / 1e12
-        deep = {"generations_per_pass": int(dinfo.gens_per_pass), "halo_rows": int(dinfo.halo_rows),
-                "value": d_value, "unit": metric_of(wl)[1], "ms_per_step": d_ms / args.steps,
-                "vs_per_generation_path": d_value / value,
-                "roofline": {"bound": "alu", "kernel": "life_tb_kernel", "achieved": alu_achieved,
-                             "peak": alu_peak, "unit": "T ALU lane-ops/s", "frac": alu_achieved / alu_peak,
-                             "ops_per_cell_update": 12 / 32, "kernel_ms_per_launch": kern_s * 1e3,
-                             "peak_source": "148 SMs x 64 ALU lanes/clk x sampled SM clock (B300_MICROARCH.md "
-                                            "alu rt=2/SMSP; tools/pipebench.cu)",
-                             "hbm_bytes_per_cell_update": 0.25 / K,
-                             "hbm_achieved_GBps": cells_per_launch * 0.25 / K / kern_s / 1e9}}
-    M.mapsm_ctx_destroy(ctx)
-
+    env = Env(args, rank, world, local_rank)
+    time.sleep(0.2)  # the clock sampler's first samples
+    head = measure(env, args.workload, wl, args.steps, args.warmup, args.e2e_steps, extras=True)
+    subs = {}
+    if args.workload == "life64k" and not args.no_configs:
+        for name in SUB_CONFIGS:
+            swl = dict(WORKLOADS[name])
+            if swl.get("single_gpu") and world > 1:
+                continue
+            subs[name] = measure(env, name, swl, args.steps, args.warmup, 1, min_region_s=0.3)
+    env.close()
     if rank == 0:
-        cb = None if args.no_cpu_baseline else cpu_baseline(wl)
-        nbuf = 1 if op == "histogram" else 2
-        ws_mib = nbuf * (rows + 2 * wl["r"]) * info0.pitch_bytes / 2**20
-        metric, unit = metric_of(wl)
-        dtype = {"life": "u32 bit-sliced (1 bit/cell)", "conv": "f32", "histogram": "u8 in, u32/u64 counts"}[op]
-        para = f"row-slab x{world}"
-        if world > 1:
-            para += " + NCCL allreduce of bins" if op == "histogram" else " + NCCL halo exchange"
-        line = {
-            "metric": metric, "value": value, "unit": unit, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
-            "scaling": wl["scaling"], "vs_baseline": None, "dtype": dtype, "data": "synthetic",
-            "config": {"workload": wl["label"], "w": w, "h": h, **({"d": d} if d else {}),
-                       "iterations_per_step": n, "radius": wl["r"],
-                       "boundary": wl["b"], "parallelism": para,
-                       "l2": f"L2 flushed between steps (256 MiB write, outside the events); per-GPU working set "
-                             f"{ws_mib:.0f} MiB vs 126 MB L2",
-                       "cuda_graphs": used_graphs},
-            "e2e": {"value": e2e_value, "unit": unit, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                    "how": ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step" if op == "histogram"
-                            else "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")},
-            "gpu_launches": total_launches,
-            "roofline": roofline,
-            "clocks": clocks,
-            "cpu_baseline": cb,
-        }
-        if exposure is not None:
-            line["halo_exposure"] = exposure
-        if deep is not None:
-            line["deep_halo"] = deep
-        if chained is not None:
-            line["chained_task"] = chained
-        print(json.dumps(line), flush=True)
-    if world > 1:
-        dist.barrier(device_ids=[local_rank])
-        dist.destroy_process_group()
+        if not args.no_cpu_baseline and world == 1:
+            head["cpu_baseline"] = cpu_baseline(wl)
+            for name, sub in subs.items():
+                sub["cpu_baseline"] = cpu_baseline(WORKLOADS[name])
+        else:
+            head["cpu_baseline"] = None
+        if subs:
+            head["configs"] = {name: {k: v for k, v in sub.items() if k not in ("n_gpus", "higher_is_better",
+                                                                                  "vs_baseline", "data")}
+                               for name, sub in subs.items()}
+        print(json.dumps(head), flush=True)
 
 
 if __name__ == "__main__":
