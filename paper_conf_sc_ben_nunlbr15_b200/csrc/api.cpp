@@ -24,6 +24,7 @@
 #include <cstring>
 #include <algorithm>
 #include <array>
+#include <mutex>
 #include <string>
 #include <vector>
 
@@ -154,6 +155,7 @@ struct mapsm_grid_s {
         char* ptr = nullptr;    // rows x pitch
         unsigned long long* hist = nullptr;
     };
+    int wslot = -1;             // conv r = 3..4: __constant__ weight slot (conv_upload_weights)
     int task_slabs = 0;         // target partition the task buffers belong to
     std::vector<TaskBuf> tbufs;  // one per target slab this process owns
     bool packed() const { return dtype == MAPSM_U8 && r == 1; }
@@ -163,6 +165,25 @@ struct mapsm_grid_s {
 };
 
 static const size_t kMailboxBytes = 64;  // >= sizeof(tma::Mailbox)
+
+// __constant__ weight slots of the r = 3..4 conv kernels, shared by all grids
+// of the process (kConvWeightSlots at a time).
+static std::mutex g_wslot_mu;
+static uint64_t g_wslot_used = 0;
+static int wslot_acquire() {
+    std::lock_guard<std::mutex> lk(g_wslot_mu);
+    for (int i = 0; i < kConvWeightSlots; ++i)
+        if (!(g_wslot_used >> i & 1)) {
+            g_wslot_used |= 1ull << i;
+            return i;
+        }
+    return -1;
+}
+static void wslot_release(int i) {
+    if (i < 0) return;
+    std::lock_guard<std::mutex> lk(g_wslot_mu);
+    g_wslot_used &= ~(1ull << i);
+}
 
 static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
     return s.base[b] + (y + g->halo) * g->pitch;
@@ -447,6 +468,25 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     return MAPSM_OK;
 }
 
+// The r = 3..4 conv kernels read their weights from a __constant__ slot of
+// each device (conv_impl.cuh): acquire one and upload (at bind, and at op_set
+// on a bound grid).  The grid's streams are drained first, so no kernel of
+// this grid reads the slot while it is rewritten.
+static mapsm_status upload_conv_weights(mapsm_grid_s* g) {
+    if (g->op != MAPSM_OP_CONV || g->d || g->r < 3 || g->r > 4) return MAPSM_OK;
+    if (g->wslot < 0) g->wslot = wslot_acquire();
+    if (g->wslot < 0)
+        return fail(MAPSM_ENOMEM, "more than %d live r = 3..4 convolution grids (weight slots)", kConvWeightSlots);
+    const int cm = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
+    DeviceGuard dg;
+    for (auto& s : g->slabs) {
+        CK(cudaSetDevice(s.device));
+        CK(cudaStreamSynchronize(s.main));
+        CK(conv_upload_weights(g->r, cm, g->wslot, g->wt));
+    }
+    return MAPSM_OK;
+}
+
 extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* weights) {
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
     if (g->state < ST_WINDOW) return fail(MAPSM_ESTATE, "op_set before window_set");
@@ -468,6 +508,7 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
     g->op = op;
     drop_graphs(g);
     if (g->state < ST_OP) g->state = ST_OP;
+    if (g->state >= ST_BOUND) TRY(upload_conv_weights(g));
     return MAPSM_OK;
 }
 
@@ -564,6 +605,7 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
     geom.plane_rows = g->d ? g->h : 0;
     geom.rpitch = g->rpitch;
     geom.rec = bulk ? &s.rec_bulk : &s.rec_bnd;
+    geom.wslot = g->wslot;
     TimingPair* tp = nullptr;
     if (g->opt_timing && &s == &g->slabs[0]) {
         auto& vec = bulk ? s.t_bulk : s.t_bnd;
@@ -1076,6 +1118,7 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     int pdev = -1;
     const bool on_dev = is_device_ptr(ptr, &pdev);
     const int64_t y_first = g->slabs[0].plan.y0;
+    TRY(upload_conv_weights(g));
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
         for (int b = 0; b < 2; ++b)
@@ -1533,6 +1576,7 @@ extern "C" mapsm_status mapsm_grid_destroy(mapsm_grid g) {
         cudaStreamSynchronize(s.side);
         free_slab(s);
     }
+    wslot_release(g->wslot);
     g->ctx->live_grids--;
     delete g;
     return MAPSM_OK;

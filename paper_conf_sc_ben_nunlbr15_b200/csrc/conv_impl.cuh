@@ -29,11 +29,14 @@
 namespace mapsm {
 namespace conv_detail {
 
+#ifndef MAPSM_CONV_BIG_PL
+#define MAPSM_CONV_BIG_PL 1  // TMA producer lanes for r >= 3
+#endif
 #ifndef MAPSM_CONV_BIG_CTAS
 #define MAPSM_CONV_BIG_CTAS 1
 #endif
 #ifndef MAPSM_CONV_BIG_NC
-#define MAPSM_CONV_BIG_NC 7
+#define MAPSM_CONV_BIG_NC 16
 #endif
 constexpr int kConvBigCtas = MAPSM_CONV_BIG_CTAS;  // CTAs per SM for r >= 3
 constexpr int kConvBigNC = MAPSM_CONV_BIG_NC;      // consumer warps per CTA for r >= 3
@@ -263,6 +266,7 @@ struct ConvTmaParams {
     // weight pairs for the FFMA2 path: wp[d * 2R + m - 1] = (W[d][m-1], W[d][m]),
     // m = 1..2R, 8-byte aligned so each is one 64-bit uniform-register pair
     float2 wp[(2 * R + 1) * 2 * R];
+    int slot;  // r >= kConvPairMinR: weight slot of c_conv_wp / c_conv_w
 };
 
 // FFMA2 (fma.rn.f32x2) pair accumulation, radius >= kConvPairMinR.
@@ -280,10 +284,10 @@ struct ConvTmaParams {
 #endif
 constexpr int kConvPairMinR = MAPSM_CONV_PAIR_MINR;
 typedef unsigned long long Acc2;
-__device__ __forceinline__ void fma_pair(Acc2& acc, float v, const float2& wv) {
+__device__ __forceinline__ void fma_pair(Acc2& acc, float v, unsigned long long wv) {
     asm("{\n\t.reg .b64 x;\n\tmov.b64 x, {%1, %1};\n\tfma.rn.f32x2 %0, x, %2, %0;\n\t}"
         : "+l"(acc)
-        : "f"(v), "l"(*reinterpret_cast<const unsigned long long*>(&wv)));
+        : "f"(v), "l"(wv));
 }
 __device__ __forceinline__ void fma_lo(Acc2& acc, float w, float v) {
     asm("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 l, %1, %2, l;\n\tmov.b64 %0, {l, h};\n\t}"
@@ -295,6 +299,51 @@ __device__ __forceinline__ void fma_hi(Acc2& acc, float w, float v) {
         : "+l"(acc)
         : "f"(w), "f"(v));
 }
+// The r >= 3 (FFMA2) kernels read their weights from __constant__ memory
+// through a uniform slot index the compiler cannot prove loop-invariant, so
+// every weight (pair) is re-loaded into a UNIFORM register (LDCU) right before
+// its FFMA2s instead of being hoisted into vector registers: the FFMA2 form
+// "broadcast value x uniform-register weight pair" issues at 1.91 warp-instr/
+// clk/SM, the vector-register-pair form at 1.46 (tools/pipebench3.cu), and the
+// hoisted weights (72 pairs = 144 registers) no longer occupy the register
+// file.  Slots are per grid (mapsm_bind uploads them; kConvWeightSlots live
+// r >= 3 grids at most); every translation unit has its own copy of the
+// arrays (internal linkage) and its own upload function.
+static __constant__ float2 c_conv_wp[kConvWeightSlots][kConvMaxPairs];
+static __constant__ float c_conv_w[kConvWeightSlots][kConvMaxTaps];
+
+// A weight (pair) load that ptxas may neither hoist nor merge; its address
+// is warp-uniform, so it becomes an LDCU into a uniform register.
+// `a` is a CONSTANT-space address (to_const below).
+__device__ __forceinline__ unsigned long long ldc_pair(unsigned long long a) {
+    unsigned long long r;
+    asm volatile("ld.const.b64 %0, [%1];" : "=l"(r) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ float ldc_one(unsigned long long a) {
+    float r;
+    asm volatile("ld.const.f32 %0, [%1];" : "=f"(r) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ unsigned long long to_const(const void* generic) {
+    unsigned long long r;
+    asm("cvta.to.const.u64 %0, %1;" : "=l"(r) : "l"(generic));
+    return r;
+}
+
+template <int R, int CM>
+cudaError_t conv_upload_weights_t(int slot, const float* weights) {
+    constexpr int K = 2 * R + 1;
+    static_assert(K * K <= kConvMaxTaps && K * (K - 1) <= kConvMaxPairs, "weight slot too small");
+    if (slot < 0 || slot >= kConvWeightSlots) return cudaErrorInvalidValue;
+    float2 wp[K * (K - 1)];
+    for (int d = 0; d < K; ++d)
+        for (int m = 1; m < K; ++m) wp[d * (K - 1) + m - 1] = make_float2(weights[d * K + m - 1], weights[d * K + m]);
+    cudaError_t e = cudaMemcpyToSymbol(c_conv_wp, wp, sizeof wp, sizeof(float2) * kConvMaxPairs * slot);
+    if (e != cudaSuccess) return e;
+    return cudaMemcpyToSymbol(c_conv_w, weights, sizeof(float) * K * K, sizeof(float) * kConvMaxTaps * slot);
+}
+
 __device__ __forceinline__ float acc_hi(Acc2 a) { return __uint_as_float((unsigned)(a >> 32)); }
 __device__ __forceinline__ float acc_lo(Acc2 a) { return __uint_as_float((unsigned)a); }
 
@@ -313,22 +362,33 @@ template <int R, int NC, int NS, int CM, int EPL, bool FUSED>
 __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) conv_tma_kernel(const __grid_constant__ ConvTmaParams<R> pp) {
     constexpr int K = 2 * R + 1;
     static_assert(NS % K == 0, "NS must be a multiple of 2R+1");
+    // consumer unroll: NS rows for the HBM-bound radii (static accumulator
+    // slots); the FMA-bound ones rotate their accumulators and run one row
+    // per iteration (their unrolled rows did not fit the instruction cache)
+    constexpr int U = R >= kConvPairMinR ? 1 : NS;
+    static_assert(NS % U == 0, "the unroll must divide NS");
     static_assert(R <= 4, "16-byte stage margins cover r <= 4");
     using G = tma::Geom<NC, EPL>;
     using VT = typename VecF<EPL>::T;
+    // this grid's weights: constant-space addresses (warp-uniform)
+    const unsigned long long cwp = to_const(&c_conv_wp[R >= kConvPairMinR ? pp.slot : 0][0]);
+    const unsigned long long cw = to_const(&c_conv_w[R >= kConvPairMinR ? pp.slot : 0][0]);
     const tma::RowStream& p = pp.s;
     extern __shared__ __align__(128) uint8_t smem[];
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
     uint64_t* empty = full + NS;
     tma::init_barriers<NS>(full, empty, NC);
-    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    // warp index through a full-mask shuffle: ptxas then knows the role
+    // branch below is warp-uniform and may use the uniform datapath (LDCU
+    // weights) inside the consumer code
+    const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
     tma::SegIter it = tma::seg_iter(p);
     tma::Seg sg;
     tma::RingPos ring;
 
     const tma::HaloLink& Lk = p.link;
     if (warp == NC) {
-        constexpr int PL = R <= 2 ? 2 : 1;  // producer lanes (see tma_rows.cuh)
+        constexpr int PL = R <= 2 ? 2 : MAPSM_CONV_BIG_PL;  // producer lanes (see tma_rows.cuh)
         if (lane < PL) {
             const unsigned int halo_target =
                 FUSED ? (unsigned int)(Lk.mine->gen * (unsigned long long)(Lk.r * p.nstrips)) : 0u;
@@ -361,9 +421,11 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         // Input row j: output rows o = j - d (d = 0..2R, tap row dy = d - R)
         // take their d-th tap row from it; o starts at d == 0 and completes
         // at d == 2R.
-        auto step = [&](int j, int k, bool check) {
-            tma::mbar_wait(&full[k], ph);
-            const float* st = reinterpret_cast<const float*>(smem + k * G::kStageBytes);
+        // Input row j lives in ring stage `stg` (= j % NS) with phase `phs`;
+        // k = j % U is static (U = the unroll: a multiple of 2R+1 dividing NS).
+        auto step = [&](int j, int k, int stg, uint32_t phs, bool check) {
+            tma::mbar_wait(&full[stg], phs);
+            const float* st = reinterpret_cast<const float*>(smem + stg * G::kStageBytes);
             // buf[m] = stage float t*EPL + m = strip element t*EPL - 4 + m
             float buf[EPL + 8];
 #pragma unroll
@@ -383,7 +445,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                 }
             }
             __syncwarp();
-            if (lane == 0) tma::mbar_arrive(&empty[k]);
+            if (lane == 0) tma::mbar_arrive(&empty[stg]);
             if (CM != COL_WRAP) {
                 if (row_first) {
                     const float e = (CM == COL_CLAMP) ? buf[4] : 0.f;
@@ -399,29 +461,35 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
             // v[q + e] = element t*EPL + q + e - R  ->  buf[4 - R + q + e]
             // Tap row d of output o = j - d lives in slot (k - d) mod K (== o mod K, NS % K == 0).
             if constexpr (PAIR) {
-                // Window value m outermost, then tap row d and pair jp: the 2R+1 x EPL/2
-                // accumulator chains of this input row are independent, so consecutive
-                // FFMA2s never wait on each other; each chain still takes m (= its dx)
-                // in increasing order.
+                // Rotating accumulators: acc2[d] is output row o = j - d.  Shift them
+                // (the finished row j - 2R left at the end of the previous row), start
+                // output j at +0.0f, then apply this input row's taps.  Window value m
+                // outermost, then tap row d and pair jp: 2R+1 x EPL/2 independent
+                // chains between dependent FFMA2s; each chain takes m (= its dx) in
+                // increasing order.  No skip tests: rows outside [0, n_out) are
+                // computed and never stored.
+#pragma unroll
+                for (int d = K - 1; d > 0; --d)
+#pragma unroll
+                    for (int jp = 0; jp < EPL / 2; ++jp) acc2[d][jp] = acc2[d - 1][jp];
+#pragma unroll
+                for (int jp = 0; jp < EPL / 2; ++jp) acc2[0][jp] = 0ull;  // (+0.0f, +0.0f)
 #pragma unroll
                 for (int m = 0; m <= K; ++m) {
 #pragma unroll
                     for (int d = 0; d < K; ++d) {
-                        const int o = j - d;
-                        const int slot = ((k - d) % K + K) % K;
-                        if (check && !(o >= 0 && o < n_out)) continue;
+                        if (m == 0 || m == K) {
+                            const float w = ldc_one(cw + 4 * (d * K + (m == 0 ? 0 : K - 1)));
 #pragma unroll
-                        for (int jp = 0; jp < EPL / 2; ++jp) {
-                            const float v = buf[4 - R + 2 * jp + m];
-                            Acc2& a = acc2[slot][jp];
-                            if (m == 0) {
-                                if (d == 0) a = 0ull;   // (+0.0f, +0.0f): output o starts here
-                                fma_hi(a, pp.wt[d * K], v);
-                            } else if (m == K) {
-                                fma_lo(a, pp.wt[d * K + K - 1], v);
-                            } else {
-                                fma_pair(a, v, pp.wp[d * (K - 1) + m - 1]);
+                            for (int jp = 0; jp < EPL / 2; ++jp) {
+                                const float v = buf[4 - R + 2 * jp + m];
+                                if (m == 0) fma_hi(acc2[d][jp], w, v);
+                                else fma_lo(acc2[d][jp], w, v);
                             }
+                        } else {
+                            const unsigned long long w = ldc_pair(cwp + 8 * (d * (K - 1) + m - 1));
+#pragma unroll
+                            for (int jp = 0; jp < EPL / 2; ++jp) fma_pair(acc2[d][jp], buf[4 - R + 2 * jp + m], w);
                         }
                     }
                 }
@@ -429,8 +497,8 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
 #pragma unroll
             for (int d = 0; d < K; ++d) {
                 const int o = j - d;
-                const int slot = ((k - d) % K + K) % K;
-                if (!check || (o >= 0 && o < n_out)) {
+                const int slot = PAIR ? d : ((k - d) % K + K) % K;
+                if (PAIR ? (d == K - 1 && o >= 0) : (!check || (o >= 0 && o < n_out))) {
                     float res[EPL];
                     if constexpr (PAIR) {
 #pragma unroll
@@ -471,23 +539,35 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         };
 
         const uint32_t ph0 = ph;
-        int j = 0;
-        if (n_in >= NS) {
+        // blocks of U rows: the first and last with full checks, the steady
+        // ones (every output touched lies in [0, n_out)) without
+        auto block = [&](int j0, bool check) {
+            const int sbase = j0 % NS;                                // a multiple of U
+            const uint32_t phb = ph0 ^ (uint32_t)((j0 / NS) & 1);     // the stage's use count parity
 #pragma unroll
-            for (int k = 0; k < NS; ++k) step(k, k, true);  // first trip: o < 0 for d > k (static)
-            ph ^= 1u;
-            // steady trips: every output touched lies in [0, n_out)
-            for (j = NS; j + NS <= n_in && j + NS - 1 < n_out; j += NS) {
-#pragma unroll
-                for (int k = 0; k < NS; ++k) step(j + k, k, false);
-                ph ^= 1u;
+            for (int k = 0; k < U; ++k)
+                if (!check || j0 + k < n_in) step(j0 + k, k, sbase + k, phb, check);
+        };
+        if constexpr (PAIR) {
+            // one row per iteration (rotating accumulators: no static slots),
+            // so the loop body stays small enough for the instruction cache
+            int stg = 0;
+            uint32_t phs = ph0;
+#pragma unroll 1
+            for (int j = 0; j < n_in; ++j) {
+                step(j, 0, stg, phs, false);
+                if (++stg == NS) {
+                    stg = 0;
+                    phs ^= 1u;
+                }
             }
-        }
-        for (; j < n_in; j += NS) {  // remaining rows: full checks
-#pragma unroll
-            for (int k = 0; k < NS; ++k)
-                if (j + k < n_in) step(j + k, k, true);
-            ph ^= 1u;
+        } else {
+            int j = 0;
+            if (n_in >= U) {
+                block(0, true);  // first block: o < 0 for d > k
+                for (j = U; j + U <= n_in && j + U - 1 < n_out; j += U) block(j, false);
+            }
+            for (; j < n_in; j += U) block(j, true);
         }
         ring.stage = n_in % NS;
         ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
@@ -524,6 +604,8 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     for (int j = 0; j < K * K; ++j) pp.wt[j] = weights[j];
     for (int d = 0; d < K; ++d)
         for (int m = 1; m < K; ++m) pp.wp[d * (K - 1) + m - 1] = make_float2(weights[d * K + m - 1], weights[d * K + m]);
+    pp.slot = g.wslot;
+    if (R >= kConvPairMinR && (g.wslot < 0 || g.wslot >= kConvWeightSlots)) return cudaErrorInvalidValue;
     const int smem = NS * G::kStageBytes + 2 * NS * 8;
     static int ctas_per_sm = 0;
     if (ctas_per_sm == 0) {
@@ -556,6 +638,7 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
 // unit (conv_r<R>_cm<CM>.cu) so their large unrolled kernels build in
 // parallel; conv_r<R>.cu declares them extern.
 #define MAPSM_CONV_BIG_INST(KW, R, NS, CM)                                                                        \
+    KW template cudaError_t conv_detail::conv_upload_weights_t<R, CM>(int, const float*);                       \
     KW template cudaError_t conv_detail::launch_conv_tma_t<R, 2, NS, CM, conv_detail::kConvBigEPL>(               \
         const StencilGeom&, const RowBands&, const float*, int, cudaStream_t, const FusedLink*);                 \
     KW template cudaError_t                                                                                      \
@@ -583,10 +666,13 @@ cudaError_t launch_conv_tma(const StencilGeom& g, const RowBands& b, const float
         if (nvec > 2 * 32) return go(std::integral_constant<int, 4>());
         return go(std::integral_constant<int, 2>());
     } else {
-        // FMA-bound radii: kConvBigNC consumer warps + the producer warp.  7
-        // keeps the CTA at 8 warps = 2 per SM sub-partition, so ptxas may give
-        // each thread 255 registers (9 warps put 3 on one sub-partition and
-        // cap it at 168: the FFMA2 kernel then spills).  Narrow rows: 2.
+        // FMA-bound radii: kConvBigNC (16) consumer warps + the producer warp,
+        // one CTA per SM.  With the weights in __constant__ slots (uniform
+        // registers) and rotating accumulators the consumer needs < 120
+        // registers, so 4 consumer warps per SM sub-partition hide the FFMA2
+        // and LDCU latencies (measured: 7 warps 281, 12: 317, 16: 337, 20: 335 G
+        // cell-updates/s on 32768 x 4096, profiles/r02_conv9_variants.txt).
+        // Narrow rows: 2.
         if (nvec > (kConvBigNC / 2) * 32) return go(std::integral_constant<int, kConvBigNC>());
         return go(std::integral_constant<int, 2>());
     }
@@ -666,7 +752,12 @@ cudaError_t launch_conv_t(const StencilGeom& g, const RowBands& b, const float* 
 }  // namespace conv_detail
 
 template <int R>
-constexpr int kConvNS = R == 1 ? 12 : R == 2 ? 10 : R == 3 ? 14 : 9;  // ring stages: multiples of 2R+1
+#ifndef MAPSM_CONV_BIG_RING
+#define MAPSM_CONV_BIG_RING 2
+#endif
+// ring stages: multiples of 2R+1; the FMA-bound radii keep MAPSM_CONV_BIG_RING
+// accumulator cycles of rows in flight
+constexpr int kConvNS = R == 1 ? 12 : R == 2 ? 10 : (2 * R + 1) * MAPSM_CONV_BIG_RING;
 
 template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,

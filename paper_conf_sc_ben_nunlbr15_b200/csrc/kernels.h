@@ -52,7 +52,15 @@ struct StencilGeom {
     // plane holds plane_rows rows of rpitch bytes (0 for 2-D grids)
     int64_t plane_rows = 0, rpitch = 0;
     LaunchRec* rec = nullptr;  // filled by the launcher when non-null
+    int wslot = -1;            // conv r >= 3: the grid's weight slot (conv_upload_weights)
 };
+
+// fp32 conv, r = 3..4 (FFMA2 kernels): weights live in __constant__ slots,
+// uploaded once per grid and device (conv_upload_weights, at bind); at most
+// kConvWeightSlots such grids at a time.  No-op for other radii.
+constexpr int kConvWeightSlots = 32;
+constexpr int kConvMaxPairs = 72, kConvMaxTaps = 81;
+cudaError_t conv_upload_weights(int r, int col_mode, int slot, const float* weights);
 
 // Output-row bands computed by one launch (1 band = all rows or interior;
 // 2 bands = the boundary rows [0,r) and [rows-r,rows)).

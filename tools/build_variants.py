@@ -29,9 +29,11 @@ def variant(name, defines=(), subs=(), src=None):
         open(p, "w").write(t.replace(a, b))
         touched.add(fname)
     macros = [x.split("=")[0] for x in defines]
-    for fname in os.listdir(cs):
-        if fname.endswith((".cu", ".cpp")) and any(m in open(os.path.join(cs, fname)).read() for m in macros):
-            touched.add(fname)
+    text = {f: open(os.path.join(cs, f)).read() for f in os.listdir(cs)}
+    marked = {f for f, t in text.items() if any(m in t for m in macros)}
+    for _ in range(3):  # files including a marked header (transitively)
+        marked |= {f for f, t in text.items() if any(f'"{h}"' in t for h in marked if not h.endswith((".cu", ".cpp")))}
+    touched |= {f for f in marked if f.endswith((".cu", ".cpp"))}
     import time
     now = time.time() + 1
     for fname in touched:

@@ -53,17 +53,23 @@ else:
     per = sorted(per_l)[len(per_l) // 2]
     gbs = bc * w * h / (per / 1e3) / 1e9
     g.set_option(M.OPT_TIMING, 0)
-# graphs region
+# graphs region (SM clock sampled during it: FMA-bound kernels run under the power cap)
+from bench import ClockSampler  # noqa: E402
+smp = ClockSampler(0).start()
+time.sleep(0.3)
 g.iterate(16)
 g.sync()
 torch.cuda.synchronize()
 t0 = time.perf_counter()
+tw0 = time.time()
 g.iterate(iters * 2)
 g.sync()
 reg = (time.perf_counter() - t0) * 1e3 / (iters * 2)  # wall: all slabs' streams
+clk = smp.region(tw0, time.time())
+smp.stop()
 print(json.dumps({"lib": os.environ.get("MAPSM_LIB", "default"), "workload": wl, "local": args.local,
                   "exchange": args.exchange, "deep": args.deep, "ms_per_launch": per,
                   "GBps": gbs, "region_ms_per_iter": reg, "region_GBps": bc * w * h / (reg / 1e3) / 1e9,
-                  "cells_per_s": w * h / (reg / 1e3)}))
+                  "cells_per_s": w * h / (reg / 1e3), "sm_mhz": clk.get("sm_mhz"), "reasons": clk.get("reasons")}))
 g.close()
 M.mapsm_ctx_destroy(ctx)
