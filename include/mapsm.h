@@ -447,15 +447,19 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         need those rows wait on it.  Needs rows per slab >
  *                         2r and the TMA kernels (Life w % 128 == 0, conv
  *                         w % 4 == 0); set before bind.
- *   MAPSM_OPT_DEEP_HALO   K in {2,3,4,6,8} (1 = off, default): Life grids keep
- *                         K*r halo rows per side and run K generations per
- *                         pass of ONE temporally blocked kernel (each CTA
- *                         carries its rows through K generations in
- *                         registers), exchanging K*r rows once per pass
- *                         instead of r rows every generation (SURVEY §8(f)
- *                         NEXT-2; the per-iteration exchange of P:L461 made
- *                         K-fold coarser).  HBM traffic per generation drops
- *                         K-fold; results are bit-identical.  Set before bind
+ *   MAPSM_OPT_DEEP_HALO   K > 1 (1 = off, default): the grid keeps K*r halo
+ *                         rows per side and exchanges them once per pass of
+ *                         K generations instead of r rows every generation
+ *                         (the per-iteration exchange of
+ *                         P:L461 made K-fold coarser).  Life: K in
+ *                         {2,3,4,6,8}, ONE temporally blocked kernel per pass
+ *                         (each CTA carries its rows through K generations in
+ *                         registers: HBM traffic per generation drops K-fold).
+ *                         fp32 conv (2-D and Window(3D)): K in 2..16, K
+ *                         single-generation launches per pass over a
+ *                         trapezoid of rows (the neighbours' halo rows are
+ *                         recomputed locally).  Results are bit-identical to
+ *                         the per-generation path.  Set before bind
  *                         (re-partitions and re-allocates: every slab needs
  *                         >= K*r rows when g > 1, else EINVAL).  n % K
  *                         trailing generations of an iterate call, slabs of

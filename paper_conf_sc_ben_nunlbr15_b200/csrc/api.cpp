@@ -346,11 +346,12 @@ static void free_slab(Slab& s) {
     s = Slab();
 }
 
-// Halo rows per side: r, or K*r for a Life grid with deep halos (K
-// generations per pass, MAPSM_OPT_DEEP_HALO).
+// Halo rows per side: r, or K*r with deep halos (K generations per pass,
+// MAPSM_OPT_DEEP_HALO; Life and the fp32 convolution).
 static int64_t halo_rows(const mapsm_grid_s* g, int radius) {
     const bool life = g->dtype == MAPSM_U8 && radius == 1;
-    return (int64_t)radius * (life && g->tb_k > 1 ? g->tb_k : 1);
+    const bool conv = g->dtype == MAPSM_F32 && radius >= 1;
+    return (int64_t)radius * ((life || conv) && g->tb_k > 1 ? g->tb_k : 1);
 }
 
 static void drop_graphs(mapsm_grid_s* g) {
@@ -655,9 +656,13 @@ static void split_bands(const Slab& s, int64_t r, RowBands& bnd, RowBands& inner
 // One pass for all local slabs, reading buffer b_in: one generation (K == 1,
 // halos of depth r), or K generations of the deep-halo kernel (halos of
 // depth K*r, exchanged once per pass).
-static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1) {
+static mapsm_status pass_conv_deep(mapsm_grid_s* g, int b_in, int K);
+
+// xdepth > 0: exchange that many rows (the last generation of a conv deep-halo pass)
+static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1, int64_t xdepth = 0) {
+    if (K > 1 && g->op == MAPSM_OP_CONV) return pass_conv_deep(g, b_in, K);
     mapsm_ctx c = g->ctx;
-    const int64_t depth = (int64_t)g->r * K;
+    const int64_t depth = xdepth > 0 ? xdepth : (int64_t)g->r * K;
     const bool exch = !g->opt_no_exchange;
     bool any_exchange = false;
     for (auto& s : g->slabs) any_exchange |= has_exchange(s);
@@ -702,6 +707,33 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1) {
         if (exch) CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
     }
     return MAPSM_OK;
+}
+
+// Deep halos for the fp32 convolution (reading t1): a
+// pass of K generations reads halos of depth K*r (exchanged once per pass)
+// and computes a trapezoid: generation j (1..K) writes rows
+// [-(K-j)*r, rows + (K-j)*r) on the exchanged sides (halo rows included, as
+// the neighbour computes them: same cells, same fmaf chain, so the values are
+// identical) and [0, rows) on the others.  Generation K is split into the
+// boundary rows (the K*r rows the neighbours need), the exchange on the side
+// stream and the interior, as the per-generation path does.  Every cell is
+// computed by the same kernel as in K single generations: bit-identical.
+static mapsm_status pass_conv_deep(mapsm_grid_s* g, int b_in, int K) {
+    const int64_t r = g->r;
+    int b = b_in;
+    for (int j = 1; j < K; ++j) {
+        for (auto& s : g->slabs) {
+            CK(cudaSetDevice(s.device));
+            const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+            RowBands tr;
+            tr.nbands = 1;
+            tr.begin[0] = top ? -(int64_t)(K - j) * r : 0;
+            tr.end[0] = s.plan.rows + (bot ? (int64_t)(K - j) * r : 0);
+            TRY(launch_step(g, s, b, tr, true));
+        }
+        b ^= 1;
+    }
+    return iterate_once(g, b, 1, (int64_t)K * r);  // generation K: boundary rows, K*r-row exchange, interior
 }
 
 // ------------------------------------------------ fused peer-memory exchange
@@ -832,10 +864,17 @@ static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
     return fused_now(g) ? iterate_fused(g, b_in) : iterate_once(g, b_in);
 }
 
-// Deep-halo passes apply: Life, TMA-kernel rows (w % 128 == 0), every slab at
-// least K rows (mirror rows at CLAMP edges), copy/NCCL exchange.
+// Deep-halo passes apply: Life with TMA-kernel rows (w % 128 == 0), every slab
+// at least K rows (mirror rows at CLAMP edges); the fp32 convolution (2-D and
+// Window(3D)) with every slab at least K*r units; copy/NCCL exchange.
 static bool tb_active(const mapsm_grid_s* g) {
-    if (g->op != MAPSM_OP_LIFE || g->tb_k <= 1 || g->opt_p2p) return false;
+    if (g->tb_k <= 1 || g->opt_p2p) return false;
+    if (g->op == MAPSM_OP_CONV) {
+        for (auto& s : g->slabs)
+            if (s.plan.rows < g->halo) return false;
+        return true;
+    }
+    if (g->op != MAPSM_OP_LIFE) return false;
     if (g->w % 128 != 0 || g->pitch % 16 != 0) return false;
     for (auto& s : g->slabs)
         if (s.plan.rows < g->tb_k) return false;
@@ -867,6 +906,10 @@ static mapsm_status refresh_deep_halos(mapsm_grid_s* g) {
     return MAPSM_OK;
 }
 
+// Buffer flips of one deep-halo pass: the Life kernel does K generations in
+// one launch (in -> out); the conv pass runs K single generations.
+static int pass_flips(const mapsm_grid_s* g, int K) { return g->op == MAPSM_OP_CONV ? (K & 1) : 1; }
+
 static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters, int K = 1) {
     CK(cudaSetDevice(s.device));
     const int64_t l0 = g->launches, x0 = g->exchanges;
@@ -875,7 +918,7 @@ static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64
     int cur = start_cur;
     for (int64_t k = 0; k < iters && st == MAPSM_OK; ++k) {
         st = K > 1 ? iterate_once(g, cur, K) : step_all(g, cur);
-        cur ^= 1;
+        cur ^= K > 1 ? pass_flips(g, K) : 1;
     }
     cudaGraph_t graph = nullptr;
     cudaError_t e = cudaStreamEndCapture(s.main, &graph);
@@ -917,6 +960,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
             RowBands bnd, inner;
             split_bands(s0, g->halo, bnd, inner);
             if (has_exchange(s0)) per_pass_launches = 1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0);
+            if (g->op == MAPSM_OP_CONV) per_pass_launches += K - 1;  // the trapezoid generations
             per_pass_exch = (has_exchange(s0) && !g->opt_no_exchange) ? s0.plan.n_recv : 0;
         }
         if (graphs) {
@@ -940,7 +984,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
         }
         for (; passes > 0; --passes) {
             TRY(iterate_once(g, g->cur, K));
-            g->cur ^= 1;
+            g->cur ^= pass_flips(g, K);
             g->gen += K;
             n -= K;
         }
@@ -1632,14 +1676,19 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             break;
         case MAPSM_OPT_DEEP_HALO: {
             const int k = v <= 1 ? 1 : (int)v;
-            if (k > 1 && !life_tb_supported(k))
-                return fail(MAPSM_EUNSUPPORTED, "deep halo: K must be 1 (off) or one of 2, 3, 4, 6, 8 (got %lld)", (long long)v);
+            const bool conv = g->dtype == MAPSM_F32;
+            if (k > 1 && !conv && !life_tb_supported(k))
+                return fail(MAPSM_EUNSUPPORTED, "deep halo (Life): K must be 1 (off) or one of 2, 3, 4, 6, 8 (got %lld)",
+                            (long long)v);
+            if (k > 1 && conv && k > 16)
+                return fail(MAPSM_EUNSUPPORTED, "deep halo (conv): K must be 1 (off) .. 16 (got %lld)", (long long)v);
             if (k == g->tb_k) break;
             if (g->state >= ST_BOUND) return fail(MAPSM_ESTATE, "set MAPSM_OPT_DEEP_HALO before bind (it sizes the halos)");
-            if (g->dtype != MAPSM_U8) return fail(MAPSM_EUNSUPPORTED, "deep halos are implemented for Life grids");
+            if (g->dtype == MAPSM_U8 && g->state >= ST_WINDOW && g->r != 1)
+                return fail(MAPSM_EUNSUPPORTED, "deep halos apply to iterated grids (Life, conv)");
             const int old = g->tb_k;
             g->tb_k = k;
-            if (g->state >= ST_WINDOW && g->r == 1) {  // re-partition and re-allocate with the new halo depth
+            if (g->state >= ST_WINDOW && g->r >= 1) {  // re-partition and re-allocate with the new halo depth
                 const int st = g->state;
                 mapsm_status e = alloc_slabs(g, g->r, g->boundary);
                 if (e != MAPSM_OK) {

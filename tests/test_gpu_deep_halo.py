@@ -135,13 +135,15 @@ def test_errors(ctx, local_ctx):
         M.mapsm_set_option(gh, M.OPT_DEEP_HALO, 4)  # unchanged value: fine
     finally:
         M.mapsm_grid_destroy(gh)
-    # conv grids: not implemented
+    # conv grids: K in 2..16 (tests/test_gpu_conv_deep_halo.py); K = 17 is refused
     gh = M.mapsm_grid_create(ctx, 128, 16, M.F32)
     try:
         M.mapsm_window_set(gh, 1, M.WRAP)
         with pytest.raises(M.MapsmError) as e:
-            M.mapsm_set_option(gh, M.OPT_DEEP_HALO, 4)
+            M.mapsm_set_option(gh, M.OPT_DEEP_HALO, 17)
         assert e.value.status == M.EUNSUPPORTED
+        M.mapsm_set_option(gh, M.OPT_DEEP_HALO, 4)
+        assert M.mapsm_get_info(gh).halo_rows == 4
     finally:
         M.mapsm_grid_destroy(gh)
     # g = 4 slabs of 5 rows cannot hold 8-row halos
