@@ -129,7 +129,7 @@ struct mapsm_grid_s {
     int r = 0;
     mapsm_boundary boundary = MAPSM_WRAP;
     mapsm_op op = MAPSM_OP_LIFE;
-    float wt[17 * 17] = {0};       // conv weights, up to r = 8
+    float wt[9 * 9 * 9] = {0};      // conv weights: (2r+1)^2 up to r = 8, (2r+1)^3 up to r = 4
     int state = ST_CREATED;
     int64_t pitch = 0;
     int64_t elem = 1;               // host bytes per cell
@@ -455,8 +455,8 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
         if (radius != 1 && radius != 0)
             return fail(MAPSM_EUNSUPPORTED, "u8 grids: radius 1 (Life) or 0 (histogram), got %d", radius);
     } else if (g->d) {
-        if (radius < 1 || radius > 2)
-            return fail(MAPSM_EUNSUPPORTED, "Window(3D) conv radius must be 1..2, got %d", radius);
+        if (radius < 1 || radius > 4)
+            return fail(MAPSM_EUNSUPPORTED, "Window(3D) conv radius must be 1..4, got %d", radius);
     } else {
         if (radius < 1 || radius > 8) return fail(MAPSM_EUNSUPPORTED, "conv radius must be 1..8, got %d", radius);
     }
@@ -502,7 +502,9 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
         if (g->dtype != MAPSM_F32) return fail(MAPSM_EUNSUPPORTED, "conv needs dtype F32");
         if (!weights) return fail(MAPSM_EINVAL, "conv needs (2r+1)^2 weights");
         const int k = 2 * g->r + 1;
-        memcpy(g->wt, weights, sizeof(float) * k * k * (g->d ? k : 1));
+        const size_t nw = (size_t)k * k * (g->d ? k : 1);
+        if (nw > sizeof(g->wt) / sizeof(g->wt[0])) return fail(MAPSM_EUNSUPPORTED, "too many weights (%zu)", nw);
+        memcpy(g->wt, weights, sizeof(float) * nw);
     } else {
         return fail(MAPSM_EUNSUPPORTED, "op %d", (int)op);
     }

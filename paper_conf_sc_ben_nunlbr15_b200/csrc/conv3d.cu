@@ -1,4 +1,4 @@
-// conv3d.cu — Window(3D) fp32 convolution, radius 1..2, sm_100a (SURVEY §8(f)
+// conv3d.cu — Window(3D) fp32 convolution, radius 1..4, sm_100a (SURVEY §8(f)
 // NEXT-2).
 //
 // Paper: Window (3D) input pattern with a Structured Injective output — "each
@@ -62,6 +62,11 @@ typedef unsigned long long Acc2;   // a pair of fp32 accumulators (see fma_pair)
 template <int R> struct Cfg;
 template <> struct Cfg<1> { static constexpr int RY = MAPSM_C3_RY1, MINB = MAPSM_C3_MINB1; };
 template <> struct Cfg<2> { static constexpr int RY = MAPSM_C3_RY2, MINB = MAPSM_C3_MINB2; };
+// r = 3..4 (343 / 729 FMA per cell): one output row per thread, rotating
+// accumulators (one plane per loop iteration: the 2r+1-plane unroll of the
+// static slots would not fit the instruction cache)
+template <> struct Cfg<3> { static constexpr int RY = 1, MINB = 2; };
+template <> struct Cfg<4> { static constexpr int RY = 1, MINB = 2; };
 
 template <int R>
 struct Conv3Params {
@@ -242,7 +247,9 @@ __device__ __forceinline__ void fma_hi(Acc2& acc, float w, float v) {
 // the thread (tile rows ly*RY + t) are read once each; row t is tap row
 // dy = t - R - i of the thread's output row i.  For a fixed accumulator the
 // taps arrive in (dy, dx) order (t increasing), planes in dz order.
-template <int R, int J>
+// ROT: rotating accumulators, acc[R + dz] is the output plane this plane's
+// tap dz goes to (static slot phases J otherwise).
+template <int R, int J, bool ROT = false>
 __device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const float* sm,
                                               Acc2 (&acc)[2 * R + 1][Cfg<R>::RY][2], int lx, int ly) {
     constexpr int K = 2 * R + 1;
@@ -260,7 +267,7 @@ __device__ __forceinline__ void compute_plane(const Conv3Params<R>& p, const flo
             if (dy < -R || dy > R) continue;
 #pragma unroll
             for (int dz = -R; dz <= R; ++dz) {
-                const int slot = ((J - R - dz) % K + K) % K;
+                const int slot = ROT ? R + dz : ((J - R - dz) % K + K) % K;
                 const float2* wq = p.wp + ((dz + R) * K + (dy + R)) * 2 * R + R - 1;   // wq[dx] = (W[dx-1], W[dx])
 #pragma unroll
                 for (int jp = 0; jp < 2; ++jp) {
@@ -331,6 +338,52 @@ __device__ __forceinline__ void run_chunk(const Conv3Params<R>& p, float* smbase
     cp_wait<0>();
 }
 
+// r >= 3: one plane per iteration; before plane j the accumulators shift
+// (acc[d] <- acc[d-1], acc[0] = +0.0f starts output plane j), after it
+// acc[2R] (output plane j - 2R, its dz = +R plane was this one) is complete.
+template <int R>
+__device__ __forceinline__ void run_chunk_rot(const Conv3Params<R>& p, float* smbase, int64_t zs, int64_t ze,
+                                              int64_t x0, int64_t y0, int lx, int ly) {
+    constexpr int K = 2 * R + 1;
+    constexpr int RY = Cfg<R>::RY;
+    constexpr int BUF = Items<R>::ROWS * SW;
+    Acc2 acc[K][RY][2];
+#pragma unroll
+    for (int s = 0; s < K; ++s)
+#pragma unroll
+        for (int i = 0; i < RY; ++i) acc[s][i][0] = acc[s][i][1] = 0ull;
+    Items<R> it;
+    items_init<R>(p, it, x0, y0);
+    const int64_t zlen = ze - zs;
+    const int64_t nsteps = zlen + 2 * R;
+#pragma unroll
+    for (int q = 0; q < NBUF - 1; ++q) {
+        if (q < nsteps) stage_issue<R>(p, it, smbase + q * BUF, zs - R + q, x0, y0);
+        cp_commit();
+    }
+#pragma unroll 1
+    for (int64_t j = 0; j < nsteps; ++j) {
+        __syncthreads();
+        if (j + NBUF - 1 < nsteps) stage_issue<R>(p, it, smbase + ((j + NBUF - 1) % NBUF) * BUF, zs - R + j + NBUF - 1, x0, y0);
+        cp_commit();
+        cp_wait<NBUF - 1>();
+        __syncthreads();
+#pragma unroll
+        for (int d = K - 1; d > 0; --d)
+#pragma unroll
+            for (int i = 0; i < RY; ++i) acc[d][i][0] = acc[d - 1][i][0], acc[d][i][1] = acc[d - 1][i][1];
+#pragma unroll
+        for (int i = 0; i < RY; ++i) acc[0][i][0] = acc[0][i][1] = 0ull;
+        compute_plane<R, 0, true>(p, smbase + (j % NBUF) * BUF, acc, lx, ly);
+        const int64_t oz = j - 2 * R;
+        if (oz >= 0 && oz < zlen) {
+#pragma unroll
+            for (int i = 0; i < RY; ++i) store_out<R>(p, zs + oz, y0 + ly * RY + i, x0 + 4 * lx, acc[K - 1][i]);
+        }
+    }
+    cp_wait<0>();
+}
+
 template <int R>
 __global__ void __launch_bounds__(NT, Cfg<R>::MINB) conv3d_kernel(const __grid_constant__ Conv3Params<R> p) {
     extern __shared__ __align__(16) float smbase[];
@@ -360,8 +413,10 @@ __global__ void __launch_bounds__(NT, Cfg<R>::MINB) conv3d_kernel(const __grid_c
         const int64_t zs = p.zbeg[b] + z;
         if constexpr (R == 1)
             run_chunk<R, 0, 1, 2>(p, smbase, zs, zs + len, x0, y0, lx, ly);
-        else
+        else if constexpr (R == 2)
             run_chunk<R, 0, 1, 2, 3, 4>(p, smbase, zs, zs + len, x0, y0, lx, ly);
+        else
+            run_chunk_rot<R>(p, smbase, zs, zs + len, x0, y0, lx, ly);
         u += len;
         __syncthreads();   // the next run refills the ring from slot 0
     }
@@ -442,6 +497,8 @@ cudaError_t launch_conv3d(const StencilGeom& g, const RowBands& b, int r, const 
     switch (r) {
         case 1: return launch_t<1>(g, b, weights, num_sms, s);
         case 2: return launch_t<2>(g, b, weights, num_sms, s);
+        case 3: return launch_t<3>(g, b, weights, num_sms, s);
+        case 4: return launch_t<4>(g, b, weights, num_sms, s);
         default: return cudaErrorInvalidValue;
     }
 }

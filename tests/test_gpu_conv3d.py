@@ -4,7 +4,7 @@ Table 1) through the C ABI vs the CPU oracle (oracle.conv3d).
 Bit-exact (both sides evaluate the same (dz, dy, dx) fmaf chain, reading v1),
 which implies the north_star gate max|d| <= 1e-5 * max(1, max|o|) that is also
 asserted.  Shapes span several 64 x 16 tiles with ragged x / y / z tails, one-
-plane and one-row volumes, radii 1-2, all boundaries, plane-slab partitions
+plane and one-row volumes, radii 1-4, all boundaries, plane-slab partitions
 g = 2..4 (halo planes exchanged every iteration), and the bench volume on
 light-cone samples."""
 import numpy as np
@@ -39,7 +39,7 @@ SHAPES = [(1, 1, 1), (1, 16, 64), (5, 7, 9), (8, 16, 64), (3, 17, 65), (12, 33, 
 
 
 @pytest.mark.parametrize("shape", SHAPES)
-@pytest.mark.parametrize("r", [1, 2])
+@pytest.mark.parametrize("r", [1, 2, 3, 4])
 @pytest.mark.parametrize("boundary", ["wrap", "clamp", "zero"])
 def test_vs_oracle(ctx, shape, r, boundary):
     d, h, w = shape
@@ -52,10 +52,10 @@ def test_vs_oracle(ctx, shape, r, boundary):
 
 
 @pytest.mark.parametrize("g", [2, 3, 4])
-@pytest.mark.parametrize("r", [1, 2])
+@pytest.mark.parametrize("r", [1, 2, 3, 4])
 @pytest.mark.parametrize("boundary", ["wrap", "clamp", "zero"])
 def test_plane_slabs_exchange(local_ctx, g, r, boundary):
-    d, h, w = 4 * g + 1, 19, 70
+    d, h, w = max(4, r) * g + 1, 19, 70
     vol = mi.volume_f32(3000 + g, w, h, d)
     W = mi.weights3d_f32(3100 + r, r)
     got, info = run(local_ctx(g), vol, W, 5, boundary)
@@ -86,7 +86,7 @@ def test_validation(ctx):
     g = M.mapsm_grid_create_3d(ctx, 8, 8, 8, M.F32)
     try:
         with pytest.raises(M.MapsmError) as e:
-            M.mapsm_window_set(g, 3, M.WRAP)
+            M.mapsm_window_set(g, 5, M.WRAP)   # Window(3D) radii 1..4
         assert e.value.status == M.EUNSUPPORTED
         M.mapsm_window_set(g, 1, M.WRAP)
         assert M.mapsm_grid_slab(g, 0) == (0, 8)
