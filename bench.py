@@ -562,7 +562,7 @@ def roofline_of(env, name, wl, kernel, cells_launch, t_launch_s, clocks, launch_
             "algorithmic_bytes_per_launch": bcell * cells_launch, "peak_source": peak_src}
 
 
-def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=False):
+def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=False, deep_k=0):
     """One workload: K timed steps + e2e (+ the headline's extras)."""
     M, torch, args = env.M, env.torch, env.args
     world, rank = env.world, env.rank
@@ -674,12 +674,14 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                                 "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
                                 "note": "whole call timed (kernel + bins, one launch)"}}
     grid.close()
-    if extras and op == "life" and args.deep_halo > 1:
-        # Deep halos: K generations per pass, K-row halos
-        # once per pass — reported separately (not the per-iteration exchange
-        # of the north_star design; bound by the ALU pipe, not HBM).
-        K = args.deep_halo
-        dg = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], None, deep_halo=K)
+    if (extras and op == "life" and args.deep_halo > 1) or (op == "conv" and deep_k > 1 and not d):
+        # Deep halos: K generations per pass, K*r-row
+        # halos exchanged once per pass — reported separately (not the
+        # per-iteration exchange of the north_star design).  Life: ONE
+        # temporally blocked kernel per pass (ALU-bound); conv: K launches per
+        # pass over a trapezoid of rows (same HBM traffic; fewer exchanges).
+        K = args.deep_halo if op == "life" else deep_k
+        dg = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, deep_halo=K)
         dg.bind(h_in)
         for _ in range(warmup):
             dg.iterate(n)
@@ -693,12 +695,17 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         d_value = units_per_step * steps / (d_ms / 1e3)
         passes = n // K
         t_pass = (d_ms / steps / 1e3) / max(1, passes)
-        droof = roofline_of(env, name, wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
-                            f"one pass = {K} generations ({dl} launches per step)")
+        if op == "life":
+            droof = roofline_of(env, name, wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
+                                f"one pass = {K} generations ({dl} launches per step)")
+        else:
+            droof = roofline_of(env, name, wl, kernel, slab_cells, t_pass / K, dclocks,
+                                f"one generation (a pass = {K} launches; {dl} launches per step)")
         deep = {"generations_per_pass": int(dinfo.gens_per_pass), "halo_rows": int(dinfo.halo_rows),
                 "value": d_value, "unit": metric_of(wl)[1], "ms_per_step": d_ms / steps,
                 "vs_per_generation_path": d_value / value, "roofline": droof, "clocks": dclocks,
-                "hbm_bytes_per_cell_update": 0.25 / K}
+                "hbm_bytes_per_cell_update": 0.25 / K if op == "life" else wl["bcell"],
+                "exchanged_rows_per_pass": K * wl["r"]}
 
     metric, unit_name = metric_of(wl)
     nbuf = 1 if op == "histogram" else 2
@@ -770,7 +777,8 @@ def main():
             swl = dict(WORKLOADS[name])
             if swl.get("single_gpu") and world > 1:
                 continue
-            subs[name] = measure(env, name, swl, args.steps, args.warmup, 1, min_region_s=0.3)
+            subs[name] = measure(env, name, swl, args.steps, args.warmup, 1, min_region_s=0.3,
+                                 deep_k=4 if name == "conv5" else 0)
     env.close()
     if rank == 0:
         if not args.no_cpu_baseline and world == 1:

@@ -44,6 +44,37 @@ for b in ("wrap", "clamp", "zero"):
                 g.bind(f0)
                 g.iterate(2)
                 check(f"conv r={r} {w}x{h} {b}", g.gather(), oracle.conv(f0, W, 2, b))
+    # round 2: SMEM-resident Life (one CTA and several), conv r = 3 (constant-slot
+    # FFMA2 kernel), conv deep halos (local slabs), Window(3D) r = 3, deep-halo Life
+    for (w, h) in ((256, 40), (2048, 300)):
+        g0 = mi.life_u8(8, w, h)
+        with M.Grid(ctx, w, h, "life", 1, b) as g:
+            g.bind(g0)
+            g.iterate(11)
+            check(f"life resident {w}x{h} {b}", g.gather(), oracle.life(g0, 11, b))
+    W = mi.weights_f32(9, 3)
+    f0 = mi.field_f32(10, 1024, 40)
+    with M.Grid(ctx, 1024, 40, "conv", 3, b, W) as g:
+        g.bind(f0)
+        g.iterate(2)
+        check(f"conv r=3 1024x40 {b}", g.gather(), oracle.conv(f0, W, 2, b))
+    W = mi.weights_f32(11, 2)
+    f0 = mi.field_f32(12, 256, 30)
+    with M.Grid(loc, 256, 30, "conv", 2, b, W, deep_halo=3) as g:
+        g.bind(f0)
+        g.iterate(7)
+        check(f"conv deep halo K=3 local g=3 {b}", g.gather(), oracle.conv(f0, W, 7, b))
+    W = mi.weights3d_f32(13, 3)
+    v0 = mi.volume_f32(14, 40, 10, 9)
+    with M.Grid(ctx, 40, 10, "conv", 3, b, W, d=9) as g:
+        g.bind(v0)
+        g.iterate(2)
+        check(f"conv3d r=3 {b}", g.gather(), oracle.conv3d(v0, W, 2, b))
+    g0 = mi.life_u8(15, 512, 60)
+    with M.Grid(loc, 512, 60, "life", 1, b, deep_halo=4) as g:
+        g.bind(g0)
+        g.iterate(9)
+        check(f"life deep halo K=4 local g=3 {b}", g.gather(), oracle.life(g0, 9, b))
 img = mi.image_u8(7, 300, 50)
 with M.Grid(ctx, 300, 50, "histogram") as g:
     g.bind(img)
