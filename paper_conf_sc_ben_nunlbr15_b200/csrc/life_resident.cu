@@ -252,17 +252,92 @@ __global__ void __launch_bounds__(kThreads, 1) life_resident_kernel(const __grid
     }
     __syncthreads();
 
+    // Rows [a, e) of one generation split over the row groups; two bands
+    // [a0, a1) and [b0, b1) split over the two halves of the row groups.
+    auto rows_split = [&](int a, int e, int g0, int ng) {
+        const int nr = e - a;
+        const int rr = rg - g0;
+        if (!has_work || nr <= 0 || rr < 0 || rr >= ng) return;
+        const int ys = a + rr * nr / ng, ye = a + (rr + 1) * nr / ng;
+        if (ys < ye) warp_gen<CM>(c, bcur + K * nw, bnxt + K * nw, nw, ys, ye, R, top_edge, bot_edge);
+    };
+    auto two_bands = [&](int a0, int a1, int b0, int b1) {
+        if (ngr >= 2) {
+            rows_split(a0, a1, 0, ngr / 2);
+            rows_split(b0, b1, ngr / 2, ngr - ngr / 2);
+        } else {
+            rows_split(a0, a1, 0, 1);
+            rows_split(b0, b1, 0, 1);
+        }
+    };
+    const size_t side = (size_t)K * nw, slot = 2 * side;
+    // ---- halo exchange with the two neighbour CTAs, through L2.
+    // publish(q): my first / last K rows of the current generation into my
+    // slot of parity q, then my pass counter := q + 1 (release; no wait).
+    auto publish = [&](unsigned int q) {
+        const uint32_t* mine = bcur + K * nw;  // owned row 0
+        uint32_t* my = p.xbuf + ((size_t)b * 2 + (q & 1)) * slot;
+        const int nq = (int)(side / 4);
+        for (int i = threadIdx.x; i < 2 * nq; i += kThreads) {
+            const int sd = i / nq, k = i % nq;
+            const uint4 v = reinterpret_cast<const uint4*>(mine + (sd == 0 ? 0 : (R - K) * nw))[k];
+            __stcg(reinterpret_cast<uint4*>(my + sd * side) + k, v);
+        }
+        __syncthreads();
+        if (threadIdx.x == 0) {
+            __threadfence();
+            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.flags + b) : "memory");
+        }
+    };
+    // receive(q): wait for both neighbours' pass q (acquire), then read their
+    // rows into my halo rows [-K, 0) and [R, R+K) of the current buffer.
+    auto receive = [&](unsigned int q) {
+        if (threadIdx.x == 0) {
+            const unsigned int target = q + 1;
+            if (!top_edge)
+                while ((int)(ld_acquire_gpu(p.flags + up) - target) < 0) __nanosleep(32);
+            if (!bot_edge)
+                while ((int)(ld_acquire_gpu(p.flags + down) - target) < 0) __nanosleep(32);
+            __threadfence();
+        }
+        __syncthreads();
+        uint32_t* hrow = bcur;  // row -K
+        const uint32_t* su = p.xbuf + ((size_t)up * 2 + (q & 1)) * slot + side;  // up's last K rows
+        const uint32_t* sd = p.xbuf + ((size_t)down * 2 + (q & 1)) * slot;      // down's first K rows
+        const int nq = (int)(side / 4);
+        for (int i = threadIdx.x; i < 2 * nq; i += kThreads) {
+            const int sdx = i / nq, k = i % nq;
+            if (sdx == 0 && top_edge) continue;
+            if (sdx == 1 && bot_edge) continue;
+            const uint4 v = __ldcg(reinterpret_cast<const uint4*>(sdx == 0 ? su : sd) + k);
+            reinterpret_cast<uint4*>(hrow + (sdx == 0 ? 0 : (R + K) * nw))[k] = v;
+        }
+        __syncthreads();
+    };
+
+    // A pass publishes its last generation's edge rows and goes on: the
+    // next pass's first generation computes the rows that need no halo
+    // ([1, R-1), from the owned rows only) while the neighbours' rows are in
+    // flight, then receives them and computes the edge rows of the
+    // trapezoid — the exchange overlaps a generation of compute.
     unsigned int pass = 0;
+    bool pending = false;  // the current buffer's halos are still to be received (pass - 1)
     for (int64_t done = 0; done < p.n;) {
         const int kk = (p.n - done < K) ? (int)(p.n - done) : K;
         for (int j = 1; j <= kk; ++j) {
             const int lo = top_edge ? 0 : -kk + j;
             const int hi = bot_edge ? R : R + kk - j;
-            if (has_work) {
-                const int nr = hi - lo;
-                const int ys = lo + rg * nr / ngr, ye = lo + (rg + 1) * nr / ngr;
-                if (ys < ye)
-                    warp_gen<CM>(c, bcur + K * nw, bnxt + K * nw, nw, ys, ye, R, top_edge, bot_edge);
+            if (pending && R >= 3) {
+                rows_split(1, R - 1, 0, ngr);
+                receive(pass - 1);
+                two_bands(lo, 1, R - 1, hi);
+                pending = false;
+            } else {
+                if (pending) {
+                    receive(pass - 1);
+                    pending = false;
+                }
+                rows_split(lo, hi, 0, ngr);
             }
             __syncthreads();
             uint32_t* t = bcur;
@@ -271,44 +346,8 @@ __global__ void __launch_bounds__(kThreads, 1) life_resident_kernel(const __grid
         }
         done += kk;
         if (done >= p.n) break;
-        // ---- halo exchange with the two neighbour CTAs, via L2
-        const uint32_t* mine = bcur + K * nw;  // owned row 0
-        const size_t side = (size_t)K * nw, slot = 2 * side;
-        uint32_t* my = p.xbuf + ((size_t)b * 2 + (pass & 1)) * slot;
-        {
-            const int q = (int)(side / 4);
-            for (int i = threadIdx.x; i < 2 * q; i += kThreads) {
-                const int s = i / q, k = i % q;
-                const uint4 v = reinterpret_cast<const uint4*>(mine + (s == 0 ? 0 : (R - K) * nw))[k];
-                __stcg(reinterpret_cast<uint4*>(my + s * side) + k, v);
-            }
-        }
-        __syncthreads();
-        if (threadIdx.x == 0) {
-            __threadfence();
-            asm volatile("red.release.gpu.global.add.u32 [%0], 1;" ::"l"(p.flags + b) : "memory");
-            const unsigned int target = pass + 1;
-            if (!top_edge)
-                while ((int)(ld_acquire_gpu(p.flags + up) - target) < 0) __nanosleep(32);
-            if (!bot_edge)
-                while ((int)(ld_acquire_gpu(p.flags + down) - target) < 0) __nanosleep(32);
-            __threadfence();
-        }
-        __syncthreads();
-        {
-            uint32_t* h = bcur;  // row -K
-            const uint32_t* su = p.xbuf + ((size_t)up * 2 + (pass & 1)) * slot + side;  // up's last K rows
-            const uint32_t* sd = p.xbuf + ((size_t)down * 2 + (pass & 1)) * slot;      // down's first K rows
-            const int q = (int)(side / 4);
-            for (int i = threadIdx.x; i < 2 * q; i += kThreads) {
-                const int s = i / q, k = i % q;
-                if (s == 0 && top_edge) continue;
-                if (s == 1 && bot_edge) continue;
-                const uint4 v = __ldcg(reinterpret_cast<const uint4*>(s == 0 ? su : sd) + k);
-                reinterpret_cast<uint4*>(h + (s == 0 ? 0 : (R + K) * nw))[k] = v;
-            }
-        }
-        __syncthreads();
+        publish(pass);
+        pending = true;
         ++pass;
     }
     // generation n -> global (owned rows)
