@@ -155,7 +155,7 @@ struct mapsm_grid_s {
         char* ptr = nullptr;    // rows x pitch
         unsigned long long* hist = nullptr;
     };
-    int wslot = -1;             // conv r = 3..4: __constant__ weight slot (conv_upload_weights)
+    int wslot = -1;             // conv r = 2..4: __constant__ weight slot (conv_upload_weights)
     int task_slabs = 0;         // target partition the task buffers belong to
     std::vector<TaskBuf> tbufs;  // one per target slab this process owns
     bool packed() const { return dtype == MAPSM_U8 && r == 1; }
@@ -166,7 +166,7 @@ struct mapsm_grid_s {
 
 static const size_t kMailboxBytes = 64;  // >= sizeof(tma::Mailbox)
 
-// __constant__ weight slots of the r = 3..4 conv kernels, shared by all grids
+// __constant__ weight slots of the r = 2..4 conv kernels, shared by all grids
 // of the process (kConvWeightSlots at a time).
 static std::mutex g_wslot_mu;
 static uint64_t g_wslot_used = 0;
@@ -469,15 +469,15 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
     return MAPSM_OK;
 }
 
-// The r = 3..4 conv kernels read their weights from a __constant__ slot of
+// The r = 2..4 conv kernels read their weights from a __constant__ slot of
 // each device (conv_impl.cuh): acquire one and upload (at bind, and at op_set
 // on a bound grid).  The grid's streams are drained first, so no kernel of
 // this grid reads the slot while it is rewritten.
 static mapsm_status upload_conv_weights(mapsm_grid_s* g) {
-    if (g->op != MAPSM_OP_CONV || g->d || g->r < 3 || g->r > 4) return MAPSM_OK;
+    if (g->op != MAPSM_OP_CONV || g->d || !conv_uses_weight_slot(g->r)) return MAPSM_OK;
     if (g->wslot < 0) g->wslot = wslot_acquire();
     if (g->wslot < 0)
-        return fail(MAPSM_ENOMEM, "more than %d live r = 3..4 convolution grids (weight slots)", kConvWeightSlots);
+        return fail(MAPSM_ENOMEM, "more than %d live r = 2..4 convolution grids (weight slots)", kConvWeightSlots);
     const int cm = g->boundary == MAPSM_WRAP ? COL_WRAP : g->boundary == MAPSM_CLAMP ? COL_CLAMP : COL_ZERO;
     DeviceGuard dg;
     for (auto& s : g->slabs) {

@@ -11,10 +11,12 @@ template <int R>
 cudaError_t launch_conv_radius(const StencilGeom& g, const RowBands& b, const float* weights, int num_sms,
                                cudaStream_t s, const FusedLink* link);
 
+cudaError_t conv_upload_weights_r2(int cm, int slot, const float* w);
 cudaError_t conv_upload_weights_r3(int cm, int slot, const float* w);
 cudaError_t conv_upload_weights_r4(int cm, int slot, const float* w);
 
 cudaError_t conv_upload_weights(int r, int cm, int slot, const float* w) {
+    if (r == 2) return conv_upload_weights_r2(cm, slot, w);
     if (r == 3) return conv_upload_weights_r3(cm, slot, w);
     if (r == 4) return conv_upload_weights_r4(cm, slot, w);
     return cudaSuccess;

@@ -55,12 +55,13 @@ struct StencilGeom {
     int wslot = -1;            // conv r >= 3: the grid's weight slot (conv_upload_weights)
 };
 
-// fp32 conv, r = 3..4 (FFMA2 kernels): weights live in __constant__ slots,
+// fp32 conv, r = 2..4 (FFMA2 kernels): weights live in __constant__ slots,
 // uploaded once per grid and device (conv_upload_weights, at bind); at most
 // kConvWeightSlots such grids at a time.  No-op for other radii.
 constexpr int kConvWeightSlots = 32;
 constexpr int kConvMaxPairs = 72, kConvMaxTaps = 81;
 cudaError_t conv_upload_weights(int r, int col_mode, int slot, const float* weights);
+bool conv_uses_weight_slot(int r);  // the radii whose kernels read a weight slot (FFMA2 pairs)
 
 // Output-row bands computed by one launch (1 band = all rows or interior;
 // 2 bands = the boundary rows [0,r) and [rows-r,rows)).
