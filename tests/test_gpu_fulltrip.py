@@ -99,9 +99,9 @@ def test_config1_8192_full_grid_1000_generations(ctx):
 
 
 # conv: (r, w, h).  r = 2 at the 5x5 bench's row width (16 consumer warps, 8
-# strips of 2048 floats, 1 CTA/SM); r = 4 at the 9x9 bench's width (7 consumer
-# warps, 37 strips of 896 floats); r = 1, 3 at widths that select the same
-# instantiations.
+# strips of 2048 floats, 1 CTA/SM); r = 4 at the 9x9 bench's width (16
+# consumer warps, 16 strips of 2048 floats, weights in a constant slot); r =
+# 1, 3 at widths that select the same instantiations.
 CONV_SHAPES = [(2, 16384, 2048 + 3), (4, 32768, 1024 + 5), (1, 16384, 2048 + 1), (3, 32768, 512 + 7)]
 
 
@@ -125,3 +125,87 @@ def test_conv_full_ring_trips_vs_oracle(ctx, shape, b):
     tol = 1e-5 * max(1.0, float(np.abs(exp2).max()))
     assert float(np.abs(got2.astype(np.float64) - exp2).max()) <= tol
     assert np.array_equal(got2.view(np.uint32), exp2.view(np.uint32)), "iteration 2"
+
+
+# ---------------------------------------------------------------------------
+# BASELINE full sizes, the bench's exact launch configuration, EVERY cell
+# (the oracle runs a few iterations of the full grid in seconds; the long
+# runs of the bench are covered by the light-cone tests of test_gpu_life.py /
+# test_gpu_conv.py / test_gpu_conv3d.py)
+
+def test_config2_65536_full_grid_two_generations(ctx):
+    """BASELINE configs[2] at N = 1: 65536^2 WRAP (seed 0x5EED0003), 148 CTAs
+    x ~443 rows through the 24-stage ring — generations 1 and 2, every cell."""
+    import torch
+
+    w = h = 65536
+    g0 = np.empty((h, w), np.uint8)
+    mi.life_u8(mi.SEED_LIFE_64K, w, h, out=g0)
+    dev = torch.empty((h, w), dtype=torch.uint8, device="cuda")
+    with M.Grid(ctx, w, h, "life", 1, "wrap") as g:
+        g.bind(g0)
+        g.iterate(1)
+        li = g.launch()
+        _assert_full_trips(li, 2, KERNEL_LIFE_TMA, 16)
+        assert li.ctas == 148 and li.min_cta_seg_rows >= 400
+        M.mapsm_read(g.handle, dev)
+        torch.cuda.synchronize()
+        exp = oracle.life(g0, 1, "wrap")
+        del g0
+        assert torch.equal(dev, torch.from_numpy(exp).cuda()), "generation 1"
+        g.iterate(1)
+        M.mapsm_read(g.handle, dev)
+        torch.cuda.synchronize()
+    exp = oracle.life(exp, 1, "wrap")
+    assert torch.equal(dev, torch.from_numpy(exp).cuda()), "generation 2"
+
+
+def test_config3_5x5_16384_full_grid(ctx):
+    """BASELINE configs[3]: 16384^2 CLAMP 5x5 (seeds 0x5EED0004 / 0x5EED0044),
+    the bench's kernel and grid — iterations 1 and 2, every cell."""
+    w = h = 16384
+    f0 = mi.field_f32(mi.SEED_CONV5_FIELD, w, h)
+    W = mi.weights_f32(mi.SEED_CONV5_W, 2)
+    with M.Grid(ctx, w, h, "conv", 2, "clamp", W) as g:
+        g.bind(f0)
+        g.iterate(1)
+        _assert_full_trips(g.launch(), 4, KERNEL_CONV_TMA, steady_on_out=True)
+        got1 = g.gather()
+        g.iterate(1)
+        got2 = g.gather()
+    exp1 = oracle.conv(f0, W, 1, "clamp")
+    assert np.array_equal(got1.view(np.uint32), exp1.view(np.uint32))
+    exp2 = oracle.conv(exp1, W, 1, "clamp")
+    assert np.array_equal(got2.view(np.uint32), exp2.view(np.uint32))
+
+
+def test_config4_9x9_slab_full_grid(ctx):
+    """BASELINE configs[4] per-GPU slab: 32768 x 4096 ZERO 9x9 (seeds
+    0x5EED0005 / 0x5EED0055), the bench's kernel (16 consumer warps, weights
+    in a constant slot) — iteration 1 and 2, every cell."""
+    w, h = 32768, 4096
+    f0 = mi.field_f32(mi.SEED_CONV9_FIELD, w, h)
+    W = mi.weights_f32(mi.SEED_CONV9_W, 4)
+    with M.Grid(ctx, w, h, "conv", 4, "zero", W) as g:
+        g.bind(f0)
+        g.iterate(2)
+        li = g.launch()
+        assert li.kernel == KERNEL_CONV_TMA and li.consumer_warps == 16
+        got = g.gather()
+    exp = oracle.conv(f0, W, 2, "zero")
+    assert np.array_equal(got.view(np.uint32), exp.view(np.uint32))
+
+
+@pytest.mark.parametrize("r,b,n", [(1, "zero", 2), (2, "clamp", 1)])
+def test_window3d_bench_volume_full_grid(ctx, r, b, n):
+    """The Window(3D) bench volume 512^3 (r = 1) and a 256^3 r = 2 volume,
+    every cell after n iterations."""
+    d = h = w = 512 if r == 1 else 256
+    v0 = mi.volume_f32(mi.SEED_CONV3D_FIELD, w, h, d)
+    W = mi.weights3d_f32(mi.SEED_CONV3D_W + r - 1, r)
+    with M.Grid(ctx, w, h, "conv", r, b, W, d=d) as g:
+        g.bind(v0)
+        g.iterate(n)
+        got = g.gather()
+    exp = oracle.conv3d(v0, W, n, b)
+    assert np.array_equal(got.view(np.uint32), exp.view(np.uint32))
