@@ -640,21 +640,6 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         grid.set_option(M.OPT_NO_EXCHANGE, 0)
         exposure = {"ms_per_step_no_exchange": ne, "exposed_pct": 100.0 * (ms_per_step - ne) / ms_per_step}
 
-    # e2e: host buffers through the public API, copies inside the timed region
-    def e2e_step():
-        grid.bind(h_in)
-        if op == "histogram":
-            M.mapsm_histogram(grid.handle, h_bins)
-        else:
-            grid.iterate(n)
-            M.mapsm_read(grid.handle, h_out, grid._rp(h_out))
-
-    e2e_ms, _, _ = env.timed(e2e_step, e2e_steps, flush=False)
-    e2e_value = units_per_step * e2e_steps / (env.max_over_ranks(e2e_ms) / 1e3)
-    elem = 4 if op == "conv" else 1
-    h2d = cells_total * elem
-    d2h = 256 * 8 * world if op == "histogram" else cells_total * elem
-
     chained = deep = None
     if extras and op != "histogram":
         # Chained task: a Reductive-Static histogram of the
@@ -673,6 +658,78 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                                 else "histogram_f32_kernel", "bytes_per_unit": tb, "achieved": ach,
                                 "peak": peak_gbs, "unit": "GB/s", "frac": ach / peak_gbs,
                                 "note": "whole call timed (kernel + bins, one launch)"}}
+    # e2e: host buffers through the public API, copies inside the timed region.
+    # Sequential: bind -> iterate -> read, one step at a time (host waits).
+    def e2e_step():
+        grid.bind(h_in)
+        if op == "histogram":
+            M.mapsm_histogram(grid.handle, h_bins)
+        else:
+            grid.iterate(n)
+            M.mapsm_read(grid.handle, h_out, grid._rp(h_out))
+
+    seq_ms, _, _ = env.timed(e2e_step, 1, flush=False)
+    seq_value = units_per_step / (env.max_over_ranks(seq_ms) / 1e3)
+    e2e_value, e2e_how = seq_value, ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step"
+                                     if op == "histogram" else
+                                     "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")
+    pipe = None
+    if op != "histogram" and args.e2e_pipeline > 1:
+        # Pipelined: P grids of the same workload on their own streams
+        # (MAPSM_OPT_OWN_STREAM), each step = mapsm_bind_async(pinned host
+        # input) + mapsm_iterate(n) + mapsm_read_async(pinned host output) on
+        # the next grid: one step's upload, another's generations and a third's
+        # download run together (PCIe is full duplex).  Every step still moves
+        # its whole input in and its whole result out inside the timed region
+        # (events: start on the bench stream, every grid stream waits on it;
+        # end after every grid stream's last read).  The library orders the
+        # own-stream grids' host transfers FIFO per direction (xfer_begin).
+        P = args.e2e_pipeline
+        k_steps = max(e2e_steps, 4 * P)
+        pgrids = [grid]
+        grid.set_option(M.OPT_OWN_STREAM, 1)
+        for _ in range(P - 1):
+            pg = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, d=d)
+            pg.set_option(M.OPT_OWN_STREAM, 1)
+            pg.bind(h_in)
+            pgrids.append(pg)
+        pouts = [h_out] + [torch.empty_like(h_in, pin_memory=True) for _ in range(P - 1)]
+        gstreams = [torch.cuda.ExternalStream(M.mapsm_grid_stream(pg.handle)) for pg in pgrids]
+        for pg in pgrids:  # warm the graphs / streams
+            pg.iterate(n)
+            pg.sync()
+        env.barrier()
+        e0 = torch.cuda.Event(enable_timing=True)
+        e1 = torch.cuda.Event(enable_timing=True)
+        e0.record(env.stream)
+        for gs in gstreams:
+            gs.wait_event(e0)
+        for k in range(k_steps):
+            pg = pgrids[k % P]
+            M.mapsm_bind_async(pg.handle, h_in)
+            pg.iterate(n)
+            M.mapsm_read_async(pg.handle, pouts[k % P], pg._rp(pouts[k % P]))
+        for gs in gstreams:
+            ev = torch.cuda.Event()
+            ev.record(gs)
+            env.stream.wait_event(ev)
+        e1.record(env.stream)
+        e1.synchronize()
+        for pg in pgrids:
+            pg.sync()
+        pipe_ms = env.max_over_ranks(e0.elapsed_time(e1))
+        pipe = {"value": units_per_step * k_steps / (pipe_ms / 1e3), "steps": k_steps, "grids": P,
+                "ms_per_step": pipe_ms / k_steps}
+        e2e_value = pipe["value"]
+        e2e_how = (f"{P} grids on their own streams, each step mapsm_bind_async(pinned host input) + "
+                   f"mapsm_iterate(n) + mapsm_read_async(pinned host output) on the next grid; {k_steps} steps "
+                   "timed end to end (device events, all grid streams joined)")
+        for pg in pgrids[1:]:
+            pg.close()
+    elem = 4 if op == "conv" else 1
+    h2d = cells_total * elem
+    d2h = 256 * 8 * world if op == "histogram" else cells_total * elem
+
     grid.close()
     if (extras and op == "life" and args.deep_halo > 1) or (op == "conv" and deep_k > 1 and not d):
         # Deep halos: K generations per pass, K*r-row
@@ -726,8 +783,8 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                                                 "smem_bytes": int(li.smem_bytes),
                                                 "ring_stages": int(li.ring_stages)}},
         "e2e": {"value": e2e_value, "unit": unit_name, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
-                "how": ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step" if op == "histogram"
-                        else "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")},
+                "how": e2e_how, "sequential_value": seq_value,
+                "sequential_how": "one step: mapsm_bind + mapsm_iterate + mapsm_read, host waits between steps"},
         "gpu_launches": total_launches,
         "roofline": roofline,
         "clocks": clocks,
@@ -749,6 +806,8 @@ def main():
     ap.add_argument("--impl", default="mapsm", choices=["mapsm", "reference"])
     ap.add_argument("--workload", default="life64k", choices=sorted(WORKLOADS))
     ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-pipeline", type=int, default=3,
+                    help="grids pipelined for the e2e measurement (1 = sequential steps only)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="headline only (no BASELINE sub-configurations)")
     ap.add_argument("--graph-iters", type=int, default=0)

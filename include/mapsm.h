@@ -395,6 +395,17 @@ int mapsm_routine_saxpy(void* context, int slab, int device, void* stream, const
 /* Copy only this process's own rows (same row range as mapsm_bind) to `ptr`;
  * not collective; synchronises.                                              */
 mapsm_status mapsm_read(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes);
+/* Asynchronous Bind / read (the Bind and Gather of Table 2, P:L139/P:L157,
+ * without the host waits): the copies (and the Life pack / unpack) are
+ * enqueued on the grid's stream and the call returns; `ptr` must stay valid
+ * and unmodified (bind) / unread (read) until mapsm_sync(grid) or any later
+ * synchronisation of the grid's stream.  Use pinned host (or device) memory:
+ * pageable memory makes the copies synchronous.  mapsm_bind_async is
+ * collective like mapsm_bind (the first halo exchange is stream-ordered too);
+ * mapsm_read_async copies this process's rows only.  Errors of the enqueued
+ * work surface at mapsm_sync.                                               */
+mapsm_status mapsm_bind_async(mapsm_grid grid, const void* ptr, int64_t row_pitch_bytes);
+mapsm_status mapsm_read_async(mapsm_grid grid, void* ptr, int64_t row_pitch_bytes);
 
 mapsm_status mapsm_grid_destroy(mapsm_grid grid);
 
@@ -447,6 +458,11 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         need those rows wait on it.  Needs rows per slab >
  *                         2r and the TMA kernels (Life w % 128 == 0, conv
  *                         w % 4 == 0); set before bind.
+ *   MAPSM_OPT_OWN_STREAM  1: the grid's slabs run on streams of their own
+ *                         instead of the ctx stream (mapsm_grid_stream), so
+ *                         several grids of one ctx overlap (e.g. one grid's
+ *                         upload with another's compute and a third's
+ *                         download); 0 (default): the ctx stream
  *   MAPSM_OPT_DEEP_HALO   K > 1 (1 = off, default): the grid keeps K*r halo
  *                         rows per side and exchanges them once per pass of
  *                         K generations instead of r rows every generation
@@ -475,7 +491,8 @@ typedef enum {
     MAPSM_OPT_TIMING = 4,
     MAPSM_OPT_PERSISTENT = 5,
     MAPSM_OPT_EXCHANGE = 6,
-    MAPSM_OPT_DEEP_HALO = 7
+    MAPSM_OPT_DEEP_HALO = 7,
+    MAPSM_OPT_OWN_STREAM = 8
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

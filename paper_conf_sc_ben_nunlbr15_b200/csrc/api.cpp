@@ -138,6 +138,7 @@ struct mapsm_grid_s {
     int64_t gen = 0, launches = 0, exchanges = 0, device_bytes = 0;
     bool opt_graphs = true, opt_no_exchange = false, opt_timing = false, opt_persistent = true;
     int opt_persistent_mode = 1;  // 1: SMEM-resident kernel when the slab fits, 2: grid-barrier kernel only
+    bool opt_own_stream = false;  // the grid's slabs use private streams instead of the ctx stream
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
     int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
     int64_t halo = 0;           // halo rows allocated above/below each slab (r, or K*r with deep halos)
@@ -156,6 +157,7 @@ struct mapsm_grid_s {
         unsigned long long* hist = nullptr;
     };
     int wslot = -1;             // conv r = 2..4: __constant__ weight slot (conv_upload_weights)
+    bool wslot_current = false; // the slot holds the current weights on every slab device
     int task_slabs = 0;         // target partition the task buffers belong to
     std::vector<TaskBuf> tbufs;  // one per target slab this process owns
     bool packed() const { return dtype == MAPSM_U8 && r == 1; }
@@ -286,6 +288,8 @@ extern "C" mapsm_status mapsm_ctx_destroy(mapsm_ctx c) {
     if (c->live_grids > 0) return fail(MAPSM_ESTATE, "ctx still has %d grids", c->live_grids);
     if (c->comm) g_nccl.commDestroy(c->comm);
     blas_release(c);
+    if (c->ev_h2d) cudaEventDestroy(c->ev_h2d);
+    if (c->ev_d2h) cudaEventDestroy(c->ev_d2h);
     delete c;
     return MAPSM_OK;
 }
@@ -379,6 +383,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
     g->slabs.clear();
     g->device_bytes = 0;
     g->r = radius;
+    g->wslot_current = false;  // (the boundary selects the kernel's translation unit; new slab devices)
     g->halo = halo;
     g->boundary = boundary;
     const int64_t row_bytes = g->packed() ? (g->w + 31) / 32 * 4 : g->w * g->elem;
@@ -416,7 +421,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
             CK(cudaMemset(s.base[b], 0, bytes));  // ZERO halos are written once, here
             g->device_bytes += (int64_t)bytes;
         }
-        if (!c->local && c->user_stream) {
+        if (!c->local && c->user_stream && !g->opt_own_stream) {
             s.main = c->user_stream;
             s.own_main = false;
         } else {
@@ -475,6 +480,7 @@ extern "C" mapsm_status mapsm_window_set(mapsm_grid g, int radius, mapsm_boundar
 // this grid reads the slot while it is rewritten.
 static mapsm_status upload_conv_weights(mapsm_grid_s* g) {
     if (g->op != MAPSM_OP_CONV || g->d || !conv_uses_weight_slot(g->r)) return MAPSM_OK;
+    if (g->wslot >= 0 && g->wslot_current) return MAPSM_OK;
     if (g->wslot < 0) g->wslot = wslot_acquire();
     if (g->wslot < 0)
         return fail(MAPSM_ENOMEM, "more than %d live r = 2..4 convolution grids (weight slots)", kConvWeightSlots);
@@ -485,6 +491,7 @@ static mapsm_status upload_conv_weights(mapsm_grid_s* g) {
         CK(cudaStreamSynchronize(s.main));
         CK(conv_upload_weights(g->r, cm, g->wslot, g->wt));
     }
+    g->wslot_current = true;
     return MAPSM_OK;
 }
 
@@ -509,6 +516,7 @@ extern "C" mapsm_status mapsm_op_set(mapsm_grid g, mapsm_op op, const float* wei
         return fail(MAPSM_EUNSUPPORTED, "op %d", (int)op);
     }
     g->op = op;
+    g->wslot_current = false;
     drop_graphs(g);
     if (g->state < ST_OP) g->state = ST_OP;
     if (g->state >= ST_BOUND) TRY(upload_conv_weights(g));
@@ -1156,7 +1164,32 @@ static mapsm_status ensure_staging(Slab& s, int64_t bytes) {
 
 static const int64_t kStagingBytes = 64ll << 20;
 
-extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch) {
+// Host transfers of own-stream grids (MAPSM_OPT_OWN_STREAM) of a one-device
+// ctx are ordered FIFO across the grids: a grid's copies start after the
+// previously issued transfer in the same direction completed.  With several
+// grids pipelined (one uploading, one computing, one downloading) this keeps
+// each grid's data arriving as early as possible instead of all in-flight
+// uploads sharing the copy engine and finishing together — which serialised
+// the uploads against the downloads (measured, profiles/r02_e2e_pipeline.txt).
+static mapsm_status xfer_begin(mapsm_grid_s* g, Slab& s, bool h2d) {
+    mapsm_ctx c = g->ctx;
+    if (c->local || !g->opt_own_stream) return MAPSM_OK;
+    cudaEvent_t& ev = h2d ? c->ev_h2d : c->ev_d2h;
+    if (!ev) {
+        CK(cudaEventCreateWithFlags(&ev, cudaEventDisableTiming));
+        return MAPSM_OK;  // nothing recorded yet
+    }
+    CK(cudaStreamWaitEvent(s.main, ev, 0));
+    return MAPSM_OK;
+}
+static mapsm_status xfer_end(mapsm_grid_s* g, Slab& s, bool h2d) {
+    mapsm_ctx c = g->ctx;
+    if (c->local || !g->opt_own_stream) return MAPSM_OK;
+    CK(cudaEventRecord(h2d ? c->ev_h2d : c->ev_d2h, s.main));
+    return MAPSM_OK;
+}
+
+static mapsm_status bind_impl(mapsm_grid_s* g, const void* ptr, int64_t pitch, bool async) {
     if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
     if (g->state < ST_OP) return fail(MAPSM_ESTATE, "bind before window_set/op_set");
     if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch %lld < row bytes", (long long)pitch);
@@ -1165,10 +1198,11 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     const bool on_dev = is_device_ptr(ptr, &pdev);
     const int64_t y_first = g->slabs[0].plan.y0;
     TRY(upload_conv_weights(g));
+    // (captured iteration graphs stay valid: they hold the slab buffers, which
+    // a Bind refills in place, and start from buffer 0 like every Bind)
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
-        for (int b = 0; b < 2; ++b)
-            if (s.graph[b]) { cudaGraphExecDestroy(s.graph[b]); s.graph[b] = nullptr; }
+        if (!on_dev) TRY(xfer_begin(g, s, true));
         const char* src = static_cast<const char*>(ptr) + (s.plan.y0 - y_first) * g->rows_per_unit() * pitch;
         const int64_t rows = s.plan.rows;
         if (!g->packed()) {  // planes of a 3-D slab are rows_per_unit contiguous device rows each
@@ -1193,7 +1227,9 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
     }
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
-        CK(cudaStreamSynchronize(s.main));
+        if (!on_dev) TRY(xfer_end(g, s, true));
+        if (!async) CK(cudaStreamSynchronize(s.main));
+        CK(cudaEventRecord(s.ev_b, s.main));  // the uploaded rows, for the first exchange
     }
     g->cur = 0;
     g->gen = 0;
@@ -1213,19 +1249,35 @@ extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch)
             CK(cudaStreamSynchronize(s.main));
         }
     }
-    // Fill the halos of the current buffer once (the first exchange).
+    // Fill the halos of the current buffer once (the first exchange), after
+    // every slab's upload (ev_b), before the next compute on the slab (ev_h).
     bool any = false;
     for (auto& s : g->slabs) any |= has_exchange(s);
     if (any) {
         if (g->ctx->local) {
-            TRY(exchange_local(g, 0, false, g->halo));
+            TRY(exchange_local(g, 0, true, g->halo));
         } else {
+            Slab& s = g->slabs[0];
+            CK(cudaStreamWaitEvent(s.side, s.ev_b, 0));
             TRY(exchange_nccl(g, 0, g->halo));
+            CK(cudaEventRecord(s.ev_h, s.side));
+        }
+        for (auto& s : g->slabs) {
+            CK(cudaSetDevice(s.device));
+            CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
         }
         g->exchanges = 0;
     }
     g->deep_valid = true;
-    return check_async(g);
+    return async ? MAPSM_OK : check_async(g);
+}
+
+extern "C" mapsm_status mapsm_bind(mapsm_grid g, const void* ptr, int64_t pitch) {
+    return bind_impl(g, ptr, pitch, false);
+}
+
+extern "C" mapsm_status mapsm_bind_async(mapsm_grid g, const void* ptr, int64_t pitch) {
+    return bind_impl(g, ptr, pitch, true);
 }
 
 // Copy owned rows of the current buffer of slab s to dst (pitch dpitch).
@@ -1266,12 +1318,18 @@ static mapsm_status read_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, bool as
     for (auto& s : g->slabs) {
         CK(cudaSetDevice(s.device));
         char* dst = static_cast<char*>(ptr) + (s.plan.y0 - y_first) * g->rows_per_unit() * pitch;
+        if (!on_dev) TRY(xfer_begin(g, s, false));
         TRY(read_slab(g, s, dst, pitch, on_dev && pdev == s.device));
+        if (!on_dev) TRY(xfer_end(g, s, false));
     }
     return async ? MAPSM_OK : check_async(g);
 }
 
 extern "C" mapsm_status mapsm_read(mapsm_grid g, void* ptr, int64_t pitch) { return read_impl(g, ptr, pitch, false); }
+
+extern "C" mapsm_status mapsm_read_async(mapsm_grid g, void* ptr, int64_t pitch) {
+    return read_impl(g, ptr, pitch, true);
+}
 
 // Gather / GatherAsync (Table 2).  `async`: only enqueue (the caller
 // waits with mapsm_sync); the root's receive buffer is stream-ordered memory.
@@ -1676,6 +1734,19 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;
             break;
+        case MAPSM_OPT_OWN_STREAM: {
+            g->opt_own_stream = v != 0;
+            if (!g->opt_own_stream) break;
+            DeviceGuard dg;
+            for (auto& s : g->slabs) {  // already allocated: switch to a private stream now
+                if (s.own_main) continue;
+                CK(cudaSetDevice(s.device));
+                CK(cudaStreamSynchronize(s.main));
+                CK(cudaStreamCreateWithFlags(&s.main, cudaStreamNonBlocking));
+                s.own_main = true;
+            }
+            break;
+        }
         case MAPSM_OPT_DEEP_HALO: {
             const int k = v <= 1 ? 1 : (int)v;
             const bool conv = g->dtype == MAPSM_F32;

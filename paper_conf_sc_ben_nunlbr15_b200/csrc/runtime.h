@@ -86,4 +86,8 @@ struct mapsm_ctx_s {
     ncclComm_t comm = nullptr;
     int live_grids = 0;
     void* blas = nullptr;          // unmodified-routine state (unmodified.cpp), created on first use
+    // FIFO order of the host<->device transfers of the ctx's own-stream grids
+    // (api.cpp xfer_begin / xfer_end): the transfer issued first completes
+    // first, instead of all in-flight uploads sharing the copy engine.
+    cudaEvent_t ev_h2d = nullptr, ev_d2h = nullptr;
 };

@@ -24,6 +24,7 @@ WRAP, CLAMP, ZERO, NO_CHECKS = 0, 1, 2, 3
 OP_LIFE, OP_CONV, OP_HISTOGRAM = 0, 1, 2
 HALO_EXCHANGE, HALO_WRAP_LOCAL, HALO_CLAMP, HALO_ZERO = 0, 1, 2, 3
 OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING, OPT_PERSISTENT, OPT_EXCHANGE, OPT_DEEP_HALO = 1, 2, 3, 4, 5, 6, 7
+OPT_OWN_STREAM = 8
 EXCHANGE_COPY, EXCHANGE_P2P = 0, 1
 
 BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO, "no_checks": NO_CHECKS}
@@ -38,6 +39,7 @@ EXPORTED = [
     "mapsm_grid_create_3d", "mapsm_matrix_create", "mapsm_matrix_destroy", "mapsm_matrix_bind",
     "mapsm_invoke_unmodified", "mapsm_matrix_sync", "mapsm_matrix_gather", "mapsm_routine_sgemm",
     "mapsm_routine_saxpy", "mapsm_launch_query", "mapsm_exchange_plan", "mapsm_gather_plan",
+    "mapsm_bind_async", "mapsm_read_async",
 ]
 MSG_SEND, MSG_RECV = 0, 1
 (KERNEL_NONE, KERNEL_LIFE_TMA, KERNEL_LIFE_REG, KERNEL_LIFE_ANYW, KERNEL_LIFE_PERSIST, KERNEL_LIFE_TB,
@@ -129,6 +131,8 @@ def lib() -> ctypes.CDLL:
         "mapsm_op_set": [vp, ci, vp],
         "mapsm_grid_slab": [vp, ci, P(i64), P(i64)],
         "mapsm_bind": [vp, vp, i64],
+        "mapsm_bind_async": [vp, vp, i64],
+        "mapsm_read_async": [vp, vp, i64],
         "mapsm_iterate": [vp, i64],
         "mapsm_sync": [vp],
         "mapsm_gather": [vp, vp, i64, ci],
@@ -284,6 +288,11 @@ def mapsm_bind(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
     _check(lib().mapsm_bind(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_bind")
 
 
+def mapsm_bind_async(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
+    """Stream-ordered Bind: `buf` (pinned host or device) must stay valid until mapsm_sync."""
+    _check(lib().mapsm_bind_async(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_bind_async")
+
+
 def mapsm_iterate(grid: int, n: int) -> None:
     _check(lib().mapsm_iterate(grid, n), "mapsm_iterate")
 
@@ -307,6 +316,11 @@ def mapsm_gather_async(grid: int, buf, row_pitch_bytes: int | None = None, root:
 
 def mapsm_read(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
     _check(lib().mapsm_read(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read")
+
+
+def mapsm_read_async(grid: int, buf, row_pitch_bytes: int | None = None) -> None:
+    """Stream-ordered read of this process's rows: `buf` is complete after mapsm_sync."""
+    _check(lib().mapsm_read_async(grid, _ptr(buf), row_pitch_bytes or _pitch(buf, 0)), "mapsm_read_async")
 
 
 def _is_cuda_tensor(buf) -> bool:
