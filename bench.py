@@ -674,7 +674,10 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                                      if op == "histogram" else
                                      "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")
     pipe = None
-    if op != "histogram" and args.e2e_pipeline > 1:
+    if op != "histogram" and args.e2e_pipeline > 1 and world == 1:
+        # (N = 1 only: with N > 1 every Bind is a collective; several grids'
+        # NCCL exchanges on different streams of one communicator are not
+        # pipelined here — the multi-GPU e2e stays sequential)
         # Pipelined: P grids of the same workload on their own streams
         # (MAPSM_OPT_OWN_STREAM), each step = mapsm_bind_async(pinned host
         # input) + mapsm_iterate(n) + mapsm_read_async(pinned host output) on
