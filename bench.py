@@ -738,8 +738,9 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         # Deep halos: K generations per pass, K*r-row
         # halos exchanged once per pass — reported separately (not the
         # per-iteration exchange of the north_star design).  Life: ONE
-        # temporally blocked kernel per pass (ALU-bound); conv: K launches per
-        # pass over a trapezoid of rows (same HBM traffic; fewer exchanges).
+        # temporally blocked kernel per pass (ALU-bound); conv r <= 2 with
+        # K = 2: the fused two-generation kernel (one HBM pass per two
+        # generations); other conv: K launches per pass over a trapezoid.
         K = args.deep_halo if op == "life" else deep_k
         dg = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, deep_halo=K)
         dg.bind(h_in)
@@ -832,7 +833,8 @@ def main():
 
     env = Env(args, rank, world, local_rank)
     time.sleep(0.2)  # the clock sampler's first samples
-    head = measure(env, args.workload, wl, args.steps, args.warmup, args.e2e_steps, extras=True)
+    head = measure(env, args.workload, wl, args.steps, args.warmup, args.e2e_steps, extras=True,
+                   deep_k=2 if wl["op"] == "conv" and not wl.get("d") else 0)
     subs = {}
     if args.workload == "life64k" and not args.no_configs:
         for name in SUB_CONFIGS:
@@ -840,7 +842,7 @@ def main():
             if swl.get("single_gpu") and world > 1:
                 continue
             subs[name] = measure(env, name, swl, args.steps, args.warmup, 1, min_region_s=0.3,
-                                 deep_k=4 if name == "conv5" else 0)
+                                 deep_k=2 if name == "conv5" else 0)
     env.close()
     if rank == 0:
         if not args.no_cpu_baseline and world == 1:

@@ -516,7 +516,7 @@ typedef enum {
     MAPSM_KERNEL_NONE = 0, MAPSM_KERNEL_LIFE_TMA = 1, MAPSM_KERNEL_LIFE_REG = 2, MAPSM_KERNEL_LIFE_ANYW = 3,
     MAPSM_KERNEL_LIFE_PERSIST = 4, MAPSM_KERNEL_LIFE_TB = 5, MAPSM_KERNEL_CONV_TMA = 6, MAPSM_KERNEL_CONV_REG = 7,
     MAPSM_KERNEL_CONV_GENERIC = 8, MAPSM_KERNEL_CONV_WIDE = 9, MAPSM_KERNEL_CONV3D = 10,
-    MAPSM_KERNEL_LIFE_TB_PERSIST = 11
+    MAPSM_KERNEL_LIFE_TB_PERSIST = 11, MAPSM_KERNEL_CONV_TB2 = 12
 } mapsm_kernel;
 typedef struct {
     int kernel;              /* mapsm_kernel */

@@ -602,6 +602,12 @@ static mapsm_status exchange_nccl(mapsm_grid_s* g, int b, int64_t depth) {
 
 // ------------------------------------------------------------- compute step
 
+// Deep halos with K = 2 on a 2-D r = 1..2 conv grid run the fused
+// two-generation kernel (conv_tb.cuh): one HBM pass per two generations.
+static bool conv_tb2_ok(const mapsm_grid_s* g) {
+    return g->op == MAPSM_OP_CONV && !g->d && g->tb_k == 2 && conv_tb2_supported(g->r, g->w, g->pitch);
+}
+
 static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk,
                                 const FusedLink* link = nullptr, int K = 1) {
     StencilGeom geom;
@@ -631,7 +637,10 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
         CK(cudaEventRecord(tp->a, s.main));
     }
     cudaError_t e;
-    if (g->op == MAPSM_OP_LIFE && K > 1)
+    if (g->op == MAPSM_OP_CONV && K == 2 && conv_tb2_ok(g))
+        e = launch_conv_tb2(geom, bands, g->r, s.plan.top_kind == MAPSM_HALO_ZERO, s.plan.bottom_kind == MAPSM_HALO_ZERO,
+                            s.num_sms, s.main);
+    else if (g->op == MAPSM_OP_LIFE && K > 1)
         e = launch_life_tb(geom, bands, K, s.plan.top_kind == MAPSM_HALO_ZERO, s.plan.bottom_kind == MAPSM_HALO_ZERO,
                            s.num_sms, s.main);
     else if (g->op == MAPSM_OP_LIFE)
@@ -670,7 +679,7 @@ static mapsm_status pass_conv_deep(mapsm_grid_s* g, int b_in, int K);
 
 // xdepth > 0: exchange that many rows (the last generation of a conv deep-halo pass)
 static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1, int64_t xdepth = 0) {
-    if (K > 1 && g->op == MAPSM_OP_CONV) return pass_conv_deep(g, b_in, K);
+    if (K > 1 && g->op == MAPSM_OP_CONV && !conv_tb2_ok(g)) return pass_conv_deep(g, b_in, K);
     mapsm_ctx c = g->ctx;
     const int64_t depth = xdepth > 0 ? xdepth : (int64_t)g->r * K;
     const bool exch = !g->opt_no_exchange;
@@ -918,7 +927,9 @@ static mapsm_status refresh_deep_halos(mapsm_grid_s* g) {
 
 // Buffer flips of one deep-halo pass: the Life kernel does K generations in
 // one launch (in -> out); the conv pass runs K single generations.
-static int pass_flips(const mapsm_grid_s* g, int K) { return g->op == MAPSM_OP_CONV ? (K & 1) : 1; }
+static int pass_flips(const mapsm_grid_s* g, int K) {
+    return g->op == MAPSM_OP_CONV && !conv_tb2_ok(g) ? (K & 1) : 1;
+}
 
 static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters, int K = 1) {
     CK(cudaSetDevice(s.device));
@@ -970,7 +981,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
             RowBands bnd, inner;
             split_bands(s0, g->halo, bnd, inner);
             if (has_exchange(s0)) per_pass_launches = 1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0);
-            if (g->op == MAPSM_OP_CONV) per_pass_launches += K - 1;  // the trapezoid generations
+            if (g->op == MAPSM_OP_CONV && !conv_tb2_ok(g)) per_pass_launches += K - 1;  // the trapezoid generations
             per_pass_exch = (has_exchange(s0) && !g->opt_no_exchange) ? s0.plan.n_recv : 0;
         }
         if (graphs) {

@@ -23,7 +23,7 @@ enum ColMode : int { COL_WRAP = 0, COL_CLAMP = 1, COL_ZERO = 2 };
 enum LaunchKernel : int {
     LK_NONE = 0, LK_LIFE_TMA = 1, LK_LIFE_REG = 2, LK_LIFE_ANYW = 3, LK_LIFE_PERSIST = 4, LK_LIFE_TB = 5,
     LK_CONV_TMA = 6, LK_CONV_REG = 7, LK_CONV_GENERIC = 8, LK_CONV_WIDE = 9, LK_CONV3D = 10,
-    LK_LIFE_TB_PERSIST = 11
+    LK_LIFE_TB_PERSIST = 11, LK_CONV_TB2 = 12
 };
 struct LaunchRec {
     int kernel = LK_NONE;
@@ -119,6 +119,12 @@ cudaError_t launch_unpack_life(const void* src, int64_t src_pitch, uint8_t* dst,
 // conv_wide.cu).
 cudaError_t launch_conv_step(const StencilGeom& g, const RowBands& b, int r, const float* weights,
                              int num_sms, cudaStream_t s, const FusedLink* link = nullptr);
+// Two generations of the fp32 convolution in ONE pass (conv_tb.cuh), r = 1..2,
+// w % 4 == 0: reads g.in rows [-2r, rows+2r) (halo rows valid to depth 2r,
+// i.e. MAPSM_OPT_DEEP_HALO = 2), writes generation t+2 of the bands to g.out.
+bool conv_tb2_supported(int r, int64_t w, int64_t pitch);
+cudaError_t launch_conv_tb2(const StencilGeom& g, const RowBands& b, int r, int zero_top, int zero_bot, int num_sms,
+                            cudaStream_t s);
 
 // Window(3D) fp32 convolution (conv3d.cu), radius 1..2, (2r+1)^3 weights
 // ordered (dz, dy, dx); bands are plane ranges; col_mode is the y/x boundary.

@@ -44,10 +44,11 @@ EXPORTED = [
 MSG_SEND, MSG_RECV = 0, 1
 (KERNEL_NONE, KERNEL_LIFE_TMA, KERNEL_LIFE_REG, KERNEL_LIFE_ANYW, KERNEL_LIFE_PERSIST, KERNEL_LIFE_TB,
  KERNEL_CONV_TMA, KERNEL_CONV_REG, KERNEL_CONV_GENERIC, KERNEL_CONV_WIDE, KERNEL_CONV3D,
- KERNEL_LIFE_TB_PERSIST) = range(12)
+ KERNEL_LIFE_TB_PERSIST, KERNEL_CONV_TB2) = range(13)
 KERNEL_NAMES = {0: "none", 1: "life_tma_kernel", 2: "life_step_kernel", 3: "life_anyw_kernel",
                 4: "life_persist_kernel", 5: "life_tb_kernel", 6: "conv_tma_kernel", 7: "conv_step_kernel",
-                8: "conv_generic_kernel", 9: "conv_wide_kernel", 10: "conv3d_kernel", 11: "life_tb_persist_kernel"}
+                8: "conv_generic_kernel", 9: "conv_wide_kernel", 10: "conv3d_kernel", 11: "life_tb_persist_kernel",
+                12: "conv_tb2_kernel"}
 MAX_DIMS = 3
 MAX_PARAMS = 8
 PAT_BLOCK2D, PAT_BLOCK2D_T, PAT_OUT_SI, PAT_INOUT_SI = 0, 1, 2, 3

@@ -44,7 +44,7 @@ def same_bits(a, b):
 
 @pytest.mark.parametrize("g", [1, 2, 4, 8])
 @pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
-@pytest.mark.parametrize("r,K", [(1, 2), (1, 5), (2, 3), (2, 4), (4, 2), (5, 2)])
+@pytest.mark.parametrize("r,K", [(1, 2), (2, 2), (1, 5), (2, 3), (2, 4), (4, 2), (5, 2)])
 def test_local_slabs_vs_oracle(local_ctx, ctx, g, b, r, K):
     w = 512 + 4
     h = g * K * r + 2 * g + 1  # ragged: slabs of K*r + 2 or + 3 rows
@@ -93,3 +93,57 @@ def test_window3d_deep_halo(local_ctx, ctx, g, b):
     out, info = run(c, v0, W, K, b, [2 * K + 1], d=d)
     assert info.halo_rows == K * r
     assert same_bits(out, oracle.conv3d(v0, W, 2 * K + 1, b))
+
+
+# ---- the fused two-generation kernel (conv_tb.cuh): K = 2, r = 1..2
+
+@pytest.mark.parametrize("r", [1, 2])
+@pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
+@pytest.mark.parametrize("w", [4, 12, 516, 2048, 2052, 8192 + 4])
+def test_two_generation_kernel_widths(ctx, r, b, w):
+    """Strip edges, partial last strips, whole-row strips, rows narrower than
+    the window: one slab, 2 passes + a single generation."""
+    h = 37
+    f0 = mi.field_f32(4000 + w + r, w, h)
+    W = mi.weights_f32(4100 + r, r)
+    with M.Grid(ctx, w, h, "conv", r, b, W, deep_halo=2) as g:
+        g.bind(f0)
+        g.iterate(4)
+        li = g.launch()
+        mid = g.gather()
+        g.iterate(1)  # the remainder runs a single generation
+        out = g.gather()
+    assert li.kernel == M.KERNEL_CONV_TB2, M.KERNEL_NAMES.get(li.kernel)
+    exp4 = oracle.conv(f0, W, 4, b)
+    assert same_bits(mid, exp4)
+    assert same_bits(out, oracle.conv(exp4, W, 1, b))
+
+
+def test_two_generation_kernel_config3_full_grid(ctx):
+    """BASELINE configs[3] (16384^2 CLAMP 5x5) through the two-generation
+    kernel: 2 passes = 4 iterations, every cell."""
+    w = h = 16384
+    f0 = mi.field_f32(mi.SEED_CONV5_FIELD, w, h)
+    W = mi.weights_f32(mi.SEED_CONV5_W, 2)
+    with M.Grid(ctx, w, h, "conv", 2, "clamp", W, deep_halo=2) as g:
+        g.bind(f0)
+        g.iterate(4)
+        li = g.launch()
+        out = g.gather()
+    assert li.kernel == M.KERNEL_CONV_TB2 and li.gens_per_launch == 2
+    assert same_bits(out, oracle.conv(f0, W, 4, "clamp"))
+
+
+def test_two_generation_kernel_negative_weights(ctx):
+    """Signed weights and signed zeros: the ZERO-row feeds at the global
+    edges are the oracle's fmaf(w, 0, acc) terms, sign of zero included."""
+    rng = np.random.default_rng(9)
+    f0 = (rng.standard_normal((40, 256))).astype(np.float32)
+    f0[0, :8] = -0.0
+    W = (rng.standard_normal((5, 5))).astype(np.float32)
+    W[2, 2] = -0.0
+    with M.Grid(ctx, 256, 40, "conv", 2, "zero", W, deep_halo=2) as g:
+        g.bind(f0)
+        g.iterate(4)
+        out = g.gather()
+    assert same_bits(out, oracle.conv(f0, W, 4, "zero"))

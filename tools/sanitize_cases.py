@@ -64,6 +64,14 @@ for b in ("wrap", "clamp", "zero"):
         g.bind(f0)
         g.iterate(7)
         check(f"conv deep halo K=3 local g=3 {b}", g.gather(), oracle.conv(f0, W, 7, b))
+    for r in (1, 2):  # fused two-generation conv kernel (conv_tb.cuh)
+        W = mi.weights_f32(16 + r, r)
+        for (w, h) in ((516, 21), (12, 9)):
+            f0 = mi.field_f32(18, w, h)
+            with M.Grid(loc, w, h, "conv", r, b, W, deep_halo=2) as g:
+                g.bind(f0)
+                g.iterate(5)
+                check(f"conv tb2 r={r} {w}x{h} local g=3 {b}", g.gather(), oracle.conv(f0, W, 5, b))
     W = mi.weights3d_f32(13, 3)
     v0 = mi.volume_f32(14, 40, 10, 9)
     with M.Grid(ctx, 40, 10, "conv", 3, b, W, d=9) as g:
