@@ -6,6 +6,8 @@ namespace mapsm {
 template cudaError_t launch_conv_radius<1>(const StencilGeom&, const RowBands&, const float*, int, cudaStream_t,
                                                const FusedLink*);
 cudaError_t conv_upload_weights_r1(int cm, int slot, const float* w) {
+    const cudaError_t e = conv_detail::tb2_upload_weights<1>(slot, w);  // two-generation kernel's pairs
+    if (e != cudaSuccess) return e;
     switch (cm) {
         case COL_WRAP: return conv_detail::conv_upload_weights_t<1, COL_WRAP>(slot, w);
         case COL_CLAMP: return conv_detail::conv_upload_weights_t<1, COL_CLAMP>(slot, w);

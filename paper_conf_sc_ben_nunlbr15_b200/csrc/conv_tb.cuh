@@ -14,18 +14,22 @@
 // boundary values synthesised by the same rules) and generation t+2 is the
 // same chain over them — bit-identical to two single generations.
 //
-// Layout.  A CTA = NC consumer warps + 1 ghost warp + 1 producer warp.  The
-// producer streams the input rows [ys-2r, ye+2r) of the CTA's (strip, rows)
-// segments through an NS-stage TMA ring whose stages carry 8-float margins
-// (level 1 of the strip's edge vectors reads 4+r floats past the strip).
-// Consumer lane t owns columns [4t, 4t+4) of the strip at both levels; the
-// ghost warp's lanes 0 / 1 compute the level-1 vectors just left / right of
-// the strip (columns [-4, 0) / [S, S+4)), which level 2 of the edge lanes
-// reads.  Per input row: level 1 advances 2r+1 rotating accumulator rows
-// (FFMA2 pairs, weights from the constant slot on the uniform datapath, as
-// conv_impl.cuh); the level-1 row that completes goes to a 2-row shared
-// buffer; a named barrier; level 2 consumes it (2r+1 rotating accumulators)
-// and stores its completed row of generation t+2.
+// Layout.  A CTA (1024 threads) = NW level-1 warps + NW level-2 warps + 1
+// ghost warp + 1 producer warp.  The producer streams the input rows
+// [ys-2r, ye+2r) of the CTA's (strip, rows) segments through an NS-stage TMA
+// ring whose stages carry 8-float margins.  Level-1 lane t owns the vector
+// (4 columns) t of the strip; the ghost warp's lanes 0 / 1 compute the
+// level-1 vectors just left / right of the strip (columns [-4, 0) / [S, S+4)).
+// Per input row, level 1 advances 2r+1 accumulator rows (register-renamed by
+// the row phase: no accumulator moves) with one FFMA2 per tap and pair of
+// outputs, and writes its completed generation-t+1 row into a D-row shared
+// ring.  The level-2 warps consume that ring the same way (lane t: vector t)
+// and store generation t+2.  The two levels synchronise per ring row with
+// mbarriers only (full: written by every level-1 warp; empty: released by
+// every level-2 warp), so neither waits for the other in lock-step, each warp
+// holds ONE set of accumulators, and the 32 warps spread the FFMA2 work evenly
+// over the 4 SM sub-partitions (the ghost warp sits on the one with a level-1
+// warp less).
 //
 // Boundaries.  Columns: level 1 synthesises inputs outside the grid (CLAMP:
 // the edge column, ZERO: 0; WRAP: the producer copies the row's other end
@@ -34,8 +38,10 @@
 // while under WRAP the ghost / neighbour lanes computed them from wrapped
 // inputs.  Rows: exchanged halos and one-slab WRAP give real generation t+1
 // rows outside the slab; at a global CLAMP edge level 2 consumes the
-// generation t+1 edge row in place of the r rows outside (fed r+1 times),
-// at a ZERO edge it consumes r zero rows (the oracle's fmaf(w, 0, acc) terms).
+// generation t+1 edge row in place of the r rows outside (r+1 times), at a
+// ZERO edge it consumes r zero rows (the oracle's fmaf(w, 0, acc) terms).
+#include <utility>
+
 #include "conv_impl.cuh"
 
 namespace mapsm {
@@ -76,164 +82,396 @@ __device__ __forceinline__ void tb2_produce(const tma::RowStream& p, const tma::
     }
 }
 
-// The 12 floats [c0-4, c0+8) of a row around the 4-column vector at strip
-// column c0 (`base` = the row's strip column 0), with the grid's column
-// boundary applied to columns outside [0, n) (global column = e0 + c):
-// CLAMP -> the edge column, ZERO -> 0 (WRAP: the margins hold real data).
-template <int CM>
-__device__ __forceinline__ void window12(const float* base, int c0, int64_t e0, int64_t n, bool edge, float (&b)[12]) {
-#pragma unroll
-    for (int m = 0; m < 12; m += 4) {
-        const float4 q = *reinterpret_cast<const float4*>(base + c0 - 4 + m);
-        b[m] = q.x; b[m + 1] = q.y; b[m + 2] = q.z; b[m + 3] = q.w;
-    }
-    if (CM != COL_WRAP && edge) {
-#pragma unroll
-        for (int m = 0; m < 12; ++m) {
-            const int64_t gcol = e0 + c0 - 4 + m;
-            if (gcol < 0) b[m] = CM == COL_CLAMP ? base[-e0] : 0.f;
-            else if (gcol >= n) b[m] = CM == COL_CLAMP ? base[n - 1 - e0] : 0.f;
-        }
+// Weight pairs of the two-generation kernel: c_tb_wq[slot][d*2R + s-1] =
+// (lo: W[d][s], hi: W[d][s-1]), s = 1..2R.  A lane's 4 outputs form two pairs
+// (out c, out c+1) in one 64-bit accumulator, LOW half = the even column c,
+// so a completed row is stored with one 16-byte store.  Input value x of
+// column c-R+s (s = 0..2R+1) feeds out c with tap s (s <= 2R) and out c+1
+// with tap s-1 (s >= 1): one fma.rn.f32x2 with x broadcast and the pair from
+// a uniform register for s = 1..2R, one scalar fma on a half for s = 0 /
+// 2R+1 (the conv_impl.cuh scheme with the halves swapped).  Each half is an
+// IEEE fma (RN-even) and each output takes its taps in increasing (d, s) —
+// the oracle's fmaf chain (reading c11).
+constexpr int kTbMaxPairs = 5 * 4;
+static __constant__ float2 c_tb_wq[kConvWeightSlots][kTbMaxPairs];
+
+template <int R>
+cudaError_t tb2_upload_weights(int slot, const float* weights) {
+    constexpr int K = 2 * R + 1;
+    static_assert(K * (K - 1) <= kTbMaxPairs, "weight slot too small");
+    if (slot < 0 || slot >= kConvWeightSlots) return cudaErrorInvalidValue;
+    float2 wq[K * (K - 1)];
+    for (int d = 0; d < K; ++d)
+        for (int s = 1; s < K; ++s) wq[d * (K - 1) + s - 1] = make_float2(weights[d * K + s], weights[d * K + s - 1]);
+    return cudaMemcpyToSymbol(c_tb_wq, wq, sizeof wq, sizeof(float2) * kTbMaxPairs * slot);
+}
+
+// The 2R+4 floats of columns [c0-R, c0+4+R) of a row (`base` = the row's
+// strip column 0): the inputs of the 4-column vector at strip column c0.
+template <int R>
+__device__ __forceinline__ void window(const float* base, int c0, float (&b)[2 * R + 4]) {
+    static_assert(R == 1 || R == 2, "two-generation kernel: R = 1, 2");
+    const float4 q = *reinterpret_cast<const float4*>(base + c0);
+    b[R] = q.x; b[R + 1] = q.y; b[R + 2] = q.z; b[R + 3] = q.w;
+    if (R == 2) {
+        const float2 l = *reinterpret_cast<const float2*>(base + c0 - 2);
+        const float2 h = *reinterpret_cast<const float2*>(base + c0 + 4);
+        b[0] = l.x; b[1] = l.y; b[R + 4] = h.x; b[R + 5] = h.y;
+    } else {
+        b[0] = base[c0 - 1];
+        b[R + 4] = base[c0 + 4];
     }
 }
 
-// One input row's taps into 2R+1 rotating accumulator rows (pairs of outputs;
-// hi = out(2j), lo = out(2j+1)); acc[2R] completes with this row.
-template <int R>
-__device__ __forceinline__ void rot_taps(Acc2 (&acc)[2 * R + 1][2], const float (&b)[12], unsigned long long cwp,
-                                         unsigned long long cw) {
+__device__ __forceinline__ void vfma_pair(Acc2& acc, float v, unsigned long long wv) {
+    asm volatile("{\n\t.reg .b64 x;\n\tmov.b64 x, {%1, %1};\n\tfma.rn.f32x2 %0, x, %2, %0;\n\t}" : "+l"(acc) : "f"(v), "l"(wv));
+}
+__device__ __forceinline__ void vfma_lo(Acc2& acc, float w, float v) {
+    asm volatile("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 l, %1, %2, l;\n\tmov.b64 %0, {l, h};\n\t}" : "+l"(acc) : "f"(w), "f"(v));
+}
+__device__ __forceinline__ void vfma_hi(Acc2& acc, float w, float v) {
+    asm volatile("{\n\t.reg .f32 l, h;\n\tmov.b64 {l, h}, %0;\n\tfma.rn.f32 h, %1, %2, h;\n\tmov.b64 %0, {l, h};\n\t}" : "+l"(acc) : "f"(w), "f"(v));
+}
+
+// One input row's taps into the 2R+1 accumulator rows of a lane's 4 outputs,
+// register-renamed by the row phase PH (no accumulator moves): the
+// accumulator of output row o is acc[o mod K]; input row Y feeds output row
+// Y+R-d with tap row d, so acc[(PH+R) mod K] starts (d = 0) and
+// acc[(PH-R) mod K] completes (d = 2R) with this row.
+template <int R, int PH>
+__device__ __forceinline__ void taps_ph(Acc2 (&acc)[2 * R + 1][2], const float (&b)[2 * R + 4],
+                                        unsigned long long cwq, unsigned long long cw) {
     constexpr int K = 2 * R + 1;
+    constexpr int NEW = (PH + R) % K;
+    acc[NEW][0] = acc[NEW][1] = 0ull;  // (+0.0f, +0.0f): the oracle's acc = 0
 #pragma unroll
-    for (int d = K - 1; d > 0; --d) {
-        acc[d][0] = acc[d - 1][0];
-        acc[d][1] = acc[d - 1][1];
-    }
-    acc[0][0] = acc[0][1] = 0ull;  // (+0.0f, +0.0f): a new output row starts
+    for (int d = 0; d < K; ++d) {
+        const int ph = (PH + R - d + K) % K;
 #pragma unroll
-    for (int m = 0; m <= K; ++m) {
-#pragma unroll
-        for (int d = 0; d < K; ++d) {
-            if (m == 0 || m == K) {
-                const float w = ldc_one(cw + 4 * (d * K + (m == 0 ? 0 : K - 1)));
+        for (int s = 0; s <= K; ++s) {
+            if (s == 0 || s == K) {
+                const float wv = ldc_one(cw + 4 * (d * K + (s == 0 ? 0 : K - 1)));
 #pragma unroll
                 for (int jp = 0; jp < 2; ++jp) {
-                    const float v = b[4 - R + 2 * jp + m];
-                    if (m == 0) fma_hi(acc[d][jp], w, v);
-                    else fma_lo(acc[d][jp], w, v);
+                    if (s == 0) vfma_lo(acc[ph][jp], wv, b[2 * jp + s]);
+                    else vfma_hi(acc[ph][jp], wv, b[2 * jp + s]);
                 }
             } else {
-                const unsigned long long w = ldc_pair(cwp + 8 * (d * (K - 1) + m - 1));
+                const unsigned long long wq = ldc_pair(cwq + 8 * (d * (K - 1) + s - 1));
 #pragma unroll
-                for (int jp = 0; jp < 2; ++jp) fma_pair(acc[d][jp], b[4 - R + 2 * jp + m], w);
+                for (int jp = 0; jp < 2; ++jp) vfma_pair(acc[ph][jp], b[2 * jp + s], wq);
             }
         }
     }
 }
 
-__device__ __forceinline__ float4 acc_row(const Acc2 (&a)[2]) {
-    return make_float4(acc_hi(a[0]), acc_lo(a[0]), acc_hi(a[1]), acc_lo(a[1]));
+template <int I>
+using ic = std::integral_constant<int, I>;
+
+template <typename F, int... Is>
+__device__ __forceinline__ void unroll_seq(F& f, int j0, std::integer_sequence<int, Is...>) {
+    (f(ic<Is>(), j0 + Is), ...);
 }
 
-template <int R, int NC, int NS, int CM>
-__global__ void __launch_bounds__((NC + 2) * 32, 1) conv_tb2_kernel(const __grid_constant__ ConvTb2Params pp) {
-    constexpr int K = 2 * R + 1;
-    constexpr int S = NC * 128;                         // strip width (floats)
-    constexpr int SB = (S + 2 * kTbMargin) * 4;         // stage bytes
-    constexpr int L1W = S + 8;                          // level-1 row: [4 ghost | S | 4 ghost]
+__device__ __forceinline__ void st_shared_pairs(float* dst, Acc2 a, Acc2 b) {
+    asm volatile("st.shared.v2.b64 [%0], {%1, %2};" ::"r"(tma::smem_u32(dst)), "l"(a), "l"(b) : "memory");
+}
+__device__ __forceinline__ void st_shared_f4(float* dst, float v) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %1, %1, %1};" ::"r"(tma::smem_u32(dst)), "f"(v) : "memory");
+}
+__device__ __forceinline__ void st_global_pairs(float* dst, Acc2 a, Acc2 b) {
+    asm volatile("st.global.v2.b64 [%0], {%1, %2};" ::"l"(dst), "l"(a), "l"(b) : "memory");
+}
+
+// ---- shared-memory access by 32-bit shared addresses (the whole layout is
+// compile-time offsets from one base, so per-step addresses are immediates)
+__device__ __forceinline__ void mbar_wait_s(uint32_t bar, uint32_t parity) {
+    // suspends the warp in hardware (up to the hint, ns) instead of re-polling:
+    // the waits of a pipeline stage that runs ahead would otherwise spend
+    // issue slots of their SM sub-partition
+    uint32_t done = 0;
+    do {
+        asm volatile(
+            "{\n\t.reg .pred p;\n\t"
+            "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2, %3;\n\t"
+            "selp.u32 %0, 1, 0, p;\n\t}"
+            : "=r"(done)
+            : "r"(bar), "r"(parity), "r"(0x989680)
+            : "memory");
+    } while (!done);
+}
+__device__ __forceinline__ void mbar_arrive_s(uint32_t bar) {
+    asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(bar) : "memory");
+}
+__device__ __forceinline__ bool elect_one() {
+    uint32_t pred;
+    asm volatile("{\n\t.reg .pred p;\n\telect.sync _|p, 0xffffffff;\n\tselp.u32 %0, 1, 0, p;\n\t}" : "=r"(pred));
+    return pred != 0;
+}
+// every lane's shared stores / loads of this step are done, then one lane arrives
+__device__ __forceinline__ void warp_arrive(uint32_t bar) {
+    __syncwarp();
+    if (elect_one()) mbar_arrive_s(bar);
+}
+
+// The 2R+4 floats of columns [c0-R, c0+4+R) of a row at shared address `a`
+// (= the row's column c0): the inputs of the 4-column vector at c0.
+template <int R>
+__device__ __forceinline__ void window_s(uint32_t a, float (&b)[2 * R + 4]) {
+    static_assert(R == 1 || R == 2, "two-generation kernel: R = 1, 2");
+    asm volatile("ld.shared.v4.f32 {%0, %1, %2, %3}, [%4];"
+                 : "=f"(b[R]), "=f"(b[R + 1]), "=f"(b[R + 2]), "=f"(b[R + 3])
+                 : "r"(a)
+                 : "memory");
+    if (R == 2) {
+        asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(b[0]), "=f"(b[1]) : "r"(a - 8) : "memory");
+        asm volatile("ld.shared.v2.f32 {%0, %1}, [%2];" : "=f"(b[R + 4]), "=f"(b[R + 5]) : "r"(a + 16) : "memory");
+    } else {
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(b[0]) : "r"(a - 4) : "memory");
+        asm volatile("ld.shared.f32 %0, [%1];" : "=f"(b[R + 4]) : "r"(a + 16) : "memory");
+    }
+}
+__device__ __forceinline__ void st_shared_pairs_s(uint32_t a, Acc2 x, Acc2 y) {
+    asm volatile("st.shared.v2.b64 [%0], {%1, %2};" ::"r"(a), "l"(x), "l"(y) : "memory");
+}
+__device__ __forceinline__ void st_shared_f4_s(uint32_t a, float v) {
+    asm volatile("st.shared.v4.f32 [%0], {%1, %1, %1, %1};" ::"r"(a), "f"(v) : "memory");
+}
+
+constexpr int kTbWarps = 13;  // level-1 (= level-2) warps: 2 * 13 + ghost + producer = 28 warps
+constexpr int kTbL1Margin = 8;
+
+// Ring bookkeeping.  Both rings (the TMA input ring and the generation-t+1
+// ring) have 2K slots, K = 2R+1, and are indexed by the segment's input-row
+// step j: step j uses slot j mod 2K of both.  Every segment is padded to a
+// multiple of 2K steps (the padding steps move no data but keep every slot's
+// mbarrier phases in step), so a group of K steps j0 .. j0+K-1 uses slots
+// h*K + J (h = the group's half, J = 0..K-1 a compile-time offset) and
+// accumulator phase J: nothing is recomputed per step.  Step j:
+//   level 1: input row ys - 2R + j (j < n_in) into the accumulators; for
+//     2R <= j < n_in the completed generation-t+1 row ys - 3R + j goes to the
+//     ring slot (after its previous occupant was released).
+//   level 2: for 2R <= j < n_in, feed k = j - 2R: that same row (or, past a
+//     global CLAMP edge, the edge row; past a ZERO edge, a zero row); for
+//     j >= 4R the output row ys - 4R + j completes.  Level 2 waits for every
+//     slot occupant (data or padding) before releasing it, so a slot's full
+//     and empty phases alternate strictly.  The bottom CLAMP edge row, which
+//     the last R feeds read again, is released after the last feed.
+// Deadlock-free: a level-1 write waits only for the release of the occupant
+// 2K steps earlier, and level 2 never waits for a row more than R steps
+// ahead of its own.
+template <int R, int NW>
+struct TbLayout {
+    static constexpr int K = 2 * R + 1, NS = 2 * K, S = NW * 128;
+    static constexpr int SB = (S + 2 * kTbMargin) * 4;  // TMA stage bytes: [8 | S | 8] floats
+    static constexpr int L1B = (S + 2 * kTbL1Margin) * 4;  // generation-t+1 row bytes: [8 | S | 8]
+    static constexpr int OFF_L1 = NS * SB;
+    static constexpr int OFF_ZERO = OFF_L1 + NS * L1B;
+    static constexpr int OFF_FULL = OFF_ZERO + L1B;
+    static constexpr int OFF_EMPTY = OFF_FULL + 8 * NS;
+    static constexpr int OFF_L1FULL = OFF_EMPTY + 8 * NS;
+    static constexpr int OFF_L1EMPTY = OFF_L1FULL + 8 * NS;
+    static constexpr int BYTES = OFF_L1EMPTY + 8 * NS;
+};
+
+// Producer: the segment's n_in input rows, then empty rounds up to P steps.
+template <int NS>
+__device__ __forceinline__ void tb2_produce_seg(const tma::RowStream& p, const tma::Seg& t, uint8_t* smem,
+                                                int stage_bytes, uint64_t* full, uint64_t* empty, int64_t y_first,
+                                                int n_in, int P, tma::RingPos& r, bool wrap_cols) {
+    tb2_produce<NS>(p, t, smem, stage_bytes, full, empty, y_first, n_in, r, wrap_cols);
+    for (int j = n_in; j < P; ++j) {
+        if (r.count >= NS) mbar_wait_s(tma::smem_u32(&empty[r.stage]), r.phase ^ 1u);
+        tma::mbar_arrive(&full[r.stage]);
+        r.advance(NS);
+    }
+}
+
+template <int K, typename F>
+__device__ __forceinline__ void group_steps(F&& f) {
+    unroll_seq(f, 0, std::make_integer_sequence<int, K>());
+}
+
+template <int R, int NW, int NS_, int CM>
+__global__ void __launch_bounds__((2 * NW + 2) * 32, 1) conv_tb2_kernel(const __grid_constant__ ConvTb2Params pp) {
+    using Ly = TbLayout<R, NW>;
+    constexpr int K = Ly::K, NS = Ly::NS, S = Ly::S;
+    static_assert(NS_ == NS, "ring size");
     const tma::RowStream& p = pp.s;
     extern __shared__ __align__(128) uint8_t smem[];
-    float* l1 = reinterpret_cast<float*>(smem + NS * SB);          // 2 rows
-    uint64_t* full = reinterpret_cast<uint64_t*>(l1 + 2 * L1W);
-    uint64_t* empty = full + NS;
-    tma::init_barriers<NS>(full, empty, NC + 1);
-    const unsigned long long cwp = to_const(&c_conv_wp[pp.slot][0]);
-    const unsigned long long cw = to_const(&c_conv_w[pp.slot][0]);
+    const uint32_t sb = tma::smem_u32(smem);
+    uint64_t* full = reinterpret_cast<uint64_t*>(smem + Ly::OFF_FULL);
+    uint64_t* empty = reinterpret_cast<uint64_t*>(smem + Ly::OFF_EMPTY);
+    for (int i = threadIdx.x; i < Ly::L1B / 4; i += blockDim.x)
+        reinterpret_cast<float*>(smem + Ly::OFF_ZERO)[i] = 0.f;
+    if (threadIdx.x == 0)
+        for (int s = 0; s < NS; ++s) {
+            tma::mbar_init(reinterpret_cast<uint64_t*>(smem + Ly::OFF_L1FULL) + s, NW + 1);
+            tma::mbar_init(reinterpret_cast<uint64_t*>(smem + Ly::OFF_L1EMPTY) + s, NW);
+        }
+    tma::init_barriers<NS>(full, empty, NW + 1);
     const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
     tma::SegIter it = tma::seg_iter(p);
     tma::Seg sg;
-    tma::RingPos ring;
 
-    if (warp == NC + 1) {  // producer
+    if (warp == 2 * NW + 1) {  // producer
         if (lane == 0) {
-            while (tma::seg_next<NC, 4>(p, it, sg)) {
-                tma::produce_align<NS, 1>(full, empty, ring, 0);
-                tb2_produce<NS>(p, sg, smem, SB, full, empty, sg.ys - 2 * R, sg.ye - sg.ys + 4 * R, ring,
-                                CM == COL_WRAP);
+            tma::RingPos ring;
+            while (tma::seg_next<NW, 4>(p, it, sg)) {
+                const int n_in = (int)(sg.ye - sg.ys) + 4 * R;
+                const int P = (n_in + NS - 1) / NS * NS;
+                tb2_produce_seg<NS>(p, sg, smem, Ly::SB, full, empty, sg.ys - 2 * R, n_in, P, ring,
+                                    CM == COL_WRAP);
             }
         }
         return;
     }
-    const bool ghost = warp == NC;  // lanes 0 / 1: the level-1 vectors left / right of the strip
-    const int v = ghost ? (lane == 0 ? -1 : NC * 32) : warp * 32 + lane;  // level-1 vector (strip columns 4v..4v+3)
-    const bool l1_on = !ghost || lane < 2;
-    const bool clamp_top = p.top_map == ROWMAP_CLAMP, clamp_bot = p.bot_map == ROWMAP_CLAMP;
-    const bool edge_top = clamp_top || pp.zero_top, edge_bot = clamp_bot || pp.zero_bot;
-    Acc2 a1[K][2], a2[K][2];
+    const unsigned long long cwq = to_const(&c_tb_wq[pp.slot][0]);
+    const unsigned long long cw = to_const(&c_conv_w[pp.slot][0]);
+    Acc2 a[K][2];
 #pragma unroll
-    for (int d = 0; d < K; ++d) a1[d][0] = a1[d][1] = a2[d][0] = a2[d][1] = 0ull;
+    for (int d = 0; d < K; ++d) a[d][0] = a[d][1] = 0ull;
+    uint32_t h = 0, ph = 0;  // the group's half and the round's phase parity
+    auto next_group = [&]() {
+        h ^= 1u;
+        ph ^= (h ^ 1u);
+    };
 
-    while (tma::seg_next<NC, 4>(p, it, sg)) {
-        tma::consume_align<NS>(full, empty, ring, lane);
-        const int seg = (int)sg.seg;
-        const int64_t ys = sg.ys, ye = sg.ye;
-        const int n_in = (int)(ye - ys) + 4 * R;
-        // lanes whose 12-float windows reach past a grid edge (CLAMP / ZERO synthesis)
-        const bool edge1 = (sg.first_strip && 4 * v - 4 < 0) || (sg.last_strip && 4 * v + 8 > seg);
-        const bool active = !ghost && 4 * v < seg;  // stores level 2
-        float* out0 = reinterpret_cast<float*>(p.out) + sg.e0 + 4 * v;
-        int feeds = 0;
-        // level 2: consume one generation-t+1 row (or a zero row), store the completed row
-        auto feed = [&](const float* row) {
-            if (ghost) return;
-            float b[12];
-            if (row) {
-                window12<CM>(row, 4 * v, sg.e0, p.n, edge1, b);
-            } else {
+    if (warp < NW || warp == 2 * NW) {
+        // ---- level 1; the ghost warp's lanes 0 / 1: the vectors left / right of the strip
+        const bool ghost = warp == 2 * NW;
+        const int v = ghost ? (lane == 0 ? -1 : NW * 32) : warp * 32 + lane;
+        const bool on = !ghost || lane < 2;
+        const uint32_t lo4 = (uint32_t)(16 * v);  // the lane's byte offset in a row (column 4v)
+        while (tma::seg_next<NW, 4>(p, it, sg)) {
+            const int seg = (int)sg.seg;
+            const int n_in = (int)(sg.ye - sg.ys) + 4 * R;
+            const int P = (n_in + NS - 1) / NS * NS;
+            const bool lf = CM != COL_WRAP && on && sg.first_strip && v == 0;
+            const bool rf = CM != COL_WRAP && on && sg.last_strip && 4 * v + 4 == seg;
+            // vectors outside the grid under CLAMP / ZERO are not stored (lf / rf write those margins)
+            const bool store = on && !(CM != COL_WRAP && ((sg.first_strip && v < 0) || (sg.last_strip && 4 * v >= seg)));
+            const bool wedge = __any_sync(0xffffffffu, lf || rf);
+            auto step = [&](auto JC, int j, auto fullc) {
+                constexpr int J = decltype(JC)::value;
+                constexpr bool FULL = decltype(fullc)::value;
+                const uint32_t hs = h * K;  // slot of J = 0
+                const uint32_t st = sb + hs * Ly::SB + J * Ly::SB + kTbMargin * 4;  // stage column 0
+                const uint32_t rw = sb + Ly::OFF_L1 + hs * Ly::L1B + J * Ly::L1B + kTbL1Margin * 4;  // ring row column 0
+                // every lane runs the taps of every step, padding included: an
+                // accumulator is zeroed when its row starts and completes 2R
+                // steps later, so stale stage data never reaches a stored row
+                // (and no lane-dependent control flow doubles the accumulators)
+                mbar_wait_s(sb + Ly::OFF_FULL + (hs + J) * 8, ph);
+                float b[2 * R + 4];
+                window_s<R>(st + lo4, b);
+                warp_arrive(sb + Ly::OFF_EMPTY + (hs + J) * 8);
+                if (wedge) {
 #pragma unroll
-                for (int m = 0; m < 12; ++m) b[m] = 0.f;
-            }
-            rot_taps<R>(a2, b, cwp, cw);
-            if (feeds >= 2 * R && active) {
-                const int64_t o = ys + feeds - 2 * R;
-                *reinterpret_cast<float4*>(out0 + o * p.pitch) = acc_row(a2[K - 1]);
-            }
-            ++feeds;
-        };
-        int stg = ring.stage;
-        uint32_t phs = ring.phase;
+                    for (int t = 0; t < R; ++t) b[t] = lf ? (CM == COL_CLAMP ? b[R] : 0.f) : b[t];
+#pragma unroll
+                    for (int t = R + 4; t < 2 * R + 4; ++t) b[t] = rf ? (CM == COL_CLAMP ? b[R + 3] : 0.f) : b[t];
+                }
+                taps_ph<R, J % K>(a, b, cwq, cw);
+                // the slot's previous occupant released (first round: parity 1 of a fresh barrier passes)
+                mbar_wait_s(sb + Ly::OFF_L1EMPTY + (hs + J) * 8, ph ^ 1u);
+                if (FULL || (j >= 2 * R && j < n_in)) {
+                    constexpr int DONE = (J - R + K) % K;
+                    if (store) st_shared_pairs_s(rw + lo4, a[DONE][0], a[DONE][1]);
+                    if (wedge) {
+                        if (lf) st_shared_f4_s(rw - 16, CM == COL_CLAMP ? __uint_as_float((unsigned)a[DONE][0]) : 0.f);
+                        if (rf)
+                            st_shared_f4_s(rw + lo4 + 16,
+                                           CM == COL_CLAMP ? __uint_as_float((unsigned)(a[DONE][1] >> 32)) : 0.f);
+                    }
+                }
+                warp_arrive(sb + Ly::OFF_L1FULL + (hs + J) * 8);
+            };
 #pragma unroll 1
-        for (int j = 0; j < n_in; ++j) {
-            // ---- level 1: input row Y = ys - 2R + j
-            tma::mbar_wait(&full[stg], phs);
-            const float* st = reinterpret_cast<const float*>(smem + stg * SB) + kTbMargin;  // strip column 0
-            float b[12];
-            if (l1_on) window12<CM>(st, 4 * v, sg.e0, p.n, edge1, b);
-            __syncwarp();
-            if (lane == 0) tma::mbar_arrive(&empty[stg]);
-            if (++stg == NS) {
-                stg = 0;
-                phs ^= 1u;
+            for (int j0 = 0; j0 < P; j0 += K) {
+                if (j0 >= 2 * R && j0 + K <= n_in)
+                    group_steps<K>([&](auto JC, int) { step(JC, j0 + decltype(JC)::value, std::true_type()); });
+                else
+                    group_steps<K>([&](auto JC, int) { step(JC, j0 + decltype(JC)::value, std::false_type()); });
+                next_group();
             }
-            if (l1_on) rot_taps<R>(a1, b, cwp, cw);
-            if (j < 2 * R) continue;  // generation-t+1 rows before ys - R are not needed
-            // ---- the generation-t+1 row y1 = Y - R completed
-            const int64_t y1 = ys - 3 * R + j;
-            float* lrow = l1 + (j & 1) * L1W + 4;  // strip column 0 of the level-1 row buffer
-            if (l1_on) *reinterpret_cast<float4*>(lrow + 4 * v) = acc_row(a1[K - 1]);
-            asm volatile("bar.sync 1, %0;" ::"r"((NC + 1) * 32) : "memory");
-            // ---- level 2
-            if (edge_top && y1 < 0) continue;          // replaced (below) when row 0 is fed
-            if (edge_bot && y1 >= p.rows) continue;    // replaced (below) after row rows-1
-            if (edge_top && y1 == 0)
-                for (int k = 0; k < R - (int)ys; ++k) feed(clamp_top ? lrow : nullptr);
-            feed(lrow);
-            if (edge_bot && y1 == p.rows - 1)
-                for (int k = 0; k < (int)(ye + R - p.rows); ++k) feed(clamp_bot ? lrow : nullptr);
         }
-        ring.stage = stg;
-        ring.phase = phs;
-        ring.count += n_in;
+    } else {
+        // ---- level 2
+        const int v = (warp - NW) * 32 + lane;
+        const uint32_t lo4 = (uint32_t)(16 * v);
+        const bool clamp_top = p.top_map == ROWMAP_CLAMP, clamp_bot = p.bot_map == ROWMAP_CLAMP;
+        const bool edge_top = clamp_top || pp.zero_top, edge_bot = clamp_bot || pp.zero_bot;
+        while (tma::seg_next<NW, 4>(p, it, sg)) {
+            const int n_in = (int)(sg.ye - sg.ys) + 4 * R;
+            const int P = (n_in + NS - 1) / NS * NS;
+            const int64_t ys = sg.ys;
+            const bool active = 4 * v < (int)sg.seg;
+            // steps whose fed row needs the row map: top j < jt, bottom j >= jb
+            const int jt = edge_top ? (int)(3 * R - ys) : 0;
+            const int jb = edge_bot ? (int)(p.rows - ys + 3 * R) : n_in;
+            const int jhold = (clamp_bot && jb < n_in) ? jb - 1 : -1;  // the bottom CLAMP edge row's step
+            float* outp = reinterpret_cast<float*>(p.out) + sg.e0 + 4 * v + (ys - 4 * R) * p.pitch;
+            const int64_t pitch = p.pitch;
+            const int lo = jt > 4 * R ? jt : 4 * R, hi = jb < n_in ? jb : n_in;
+            auto step = [&](auto JC, int j, auto fullc) {
+                constexpr int J = decltype(JC)::value;
+                constexpr bool FULL = decltype(fullc)::value;
+                const uint32_t hs = h * K;
+                const uint32_t slot = hs + J;
+                mbar_wait_s(sb + Ly::OFF_L1FULL + slot * 8, ph);
+                if (FULL || (j >= 2 * R && j < n_in)) {
+                    uint32_t src = sb + Ly::OFF_L1 + slot * Ly::L1B + kTbL1Margin * 4;
+                    int relh = -1;
+                    if (!FULL) {
+                        const int64_t y = ys - 3 * R + j;  // generation-t+1 row fed by step j
+                        int jm = j;
+                        if (y < 0 && edge_top) jm = clamp_top ? j - (int)y : -1;                       // row 0
+                        else if (y >= p.rows && edge_bot) jm = clamp_bot ? j - (int)(y - (p.rows - 1)) : -1;  // row rows-1
+                        if (jm < 0) {
+                            src = sb + Ly::OFF_ZERO + kTbL1Margin * 4;
+                        } else if (jm != j) {
+                            // the mapped row's slot / phase (within R steps: same or adjacent round)
+                            int ms = (int)slot + (jm - j);
+                            uint32_t mph = ph;
+                            if (ms >= NS) {
+                                ms -= NS;
+                                mph ^= 1u;
+                            } else if (ms < 0) {
+                                ms += NS;
+                                mph ^= 1u;
+                            }
+                            mbar_wait_s(sb + Ly::OFF_L1FULL + ms * 8, mph);
+                            src = sb + Ly::OFF_L1 + ms * Ly::L1B + kTbL1Margin * 4;
+                            if (jm == jhold && j == n_in - 1) relh = ms;
+                        }
+                    }
+                    float b[2 * R + 4];
+                    window_s<R>(src + lo4, b);
+                    if (FULL || j != jhold) warp_arrive(sb + Ly::OFF_L1EMPTY + slot * 8);
+                    if (!FULL && relh >= 0) warp_arrive(sb + Ly::OFF_L1EMPTY + relh * 8);  // after its last read
+                    constexpr int PH = ((J - 2 * R) % K + K) % K;
+                    taps_ph<R, PH>(a, b, cwq, cw);
+                    if ((FULL || j >= 4 * R) && active) {
+                        constexpr int DONE = (PH - R + K) % K;
+                        st_global_pairs(outp, a[DONE][0], a[DONE][1]);
+                    }
+                } else {
+                    warp_arrive(sb + Ly::OFF_L1EMPTY + slot * 8);
+                }
+                outp += pitch;
+            };
+#pragma unroll 1
+            for (int j0 = 0; j0 < P; j0 += K) {
+                if (j0 >= lo && j0 + K <= hi)
+                    group_steps<K>([&](auto JC, int) { step(JC, j0 + decltype(JC)::value, std::true_type()); });
+                else
+                    group_steps<K>([&](auto JC, int) { step(JC, j0 + decltype(JC)::value, std::false_type()); });
+                next_group();
+            }
+        }
     }
+    (void)S;
 }
 
 template <int R, int NC, int NS, int CM>
@@ -254,7 +492,7 @@ cudaError_t launch_conv_tb2_t(const StencilGeom& g, const RowBands& b, int zero_
     if (g.wslot < 0 || g.wslot >= kConvWeightSlots) return cudaErrorInvalidValue;
     tma_set_link(p, nullptr, R);
     constexpr int S = NC * 128;
-    const int smem = NS * (S + 2 * kTbMargin) * 4 + 2 * (S + 8) * 4 + 2 * NS * 8;
+    const int smem = TbLayout<R, NC>::BYTES;
     static bool attr = false;
     if (!attr) {
         cudaError_t e = cudaFuncSetAttribute(conv_tb2_kernel<R, NC, NS, CM>,
@@ -263,16 +501,16 @@ cudaError_t launch_conv_tb2_t(const StencilGeom& g, const RowBands& b, int zero_
         attr = true;
     }
     const int64_t ctas = tma_plan_grid(p, b, num_sms, 1, S);
-    tma_record(g.rec, LK_CONV_TB2, p, ctas, (NC + 2) * 32, smem, NS, 1, NC, 2);
+    tma_record(g.rec, LK_CONV_TB2, p, ctas, (2 * NC + 2) * 32, smem, NS, 1, NC, 2);
     if (ctas == 0) return cudaSuccess;
-    conv_tb2_kernel<R, NC, NS, CM><<<(unsigned)ctas, (NC + 2) * 32, smem, s>>>(pp);
+    conv_tb2_kernel<R, NC, NS, CM><<<(unsigned)ctas, (2 * NC + 2) * 32, smem, s>>>(pp);
     return cudaGetLastError();
 }
 
 template <int R>
 cudaError_t launch_conv_tb2_r(const StencilGeom& g, const RowBands& b, int zero_top, int zero_bot, int num_sms,
                               cudaStream_t s) {
-    constexpr int NS = 12;
+    constexpr int NS = 2 * (2 * R + 1);  // both rings: 2K slots (conv_tb2_kernel)
     const int64_t nvec = g.w / 4;
     auto go = [&](auto nc_tag) -> cudaError_t {
         constexpr int NC = decltype(nc_tag)::value;
@@ -282,7 +520,7 @@ cudaError_t launch_conv_tb2_r(const StencilGeom& g, const RowBands& b, int zero_
             default: return launch_conv_tb2_t<R, NC, NS, COL_ZERO>(g, b, zero_top, zero_bot, num_sms, s);
         }
     };
-    if (nvec > 4 * 32) return go(std::integral_constant<int, 16>());
+    if (nvec > 4 * 32) return go(std::integral_constant<int, kTbWarps>());
     return go(std::integral_constant<int, 4>());
 }
 

@@ -66,7 +66,7 @@ for b in ("wrap", "clamp", "zero"):
         check(f"conv deep halo K=3 local g=3 {b}", g.gather(), oracle.conv(f0, W, 7, b))
     for r in (1, 2):  # fused two-generation conv kernel (conv_tb.cuh)
         W = mi.weights_f32(16 + r, r)
-        for (w, h) in ((516, 21), (12, 9)):
+        for (w, h) in ((516, 21), (12, 14)):
             f0 = mi.field_f32(18, w, h)
             with M.Grid(loc, w, h, "conv", r, b, W, deep_halo=2) as g:
                 g.bind(f0)
