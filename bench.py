@@ -519,9 +519,11 @@ def host_input(env, wl, rows, y0):
     return t
 
 
-def roofline_of(env, name, wl, kernel, cells_launch, t_launch_s, clocks, launch_unit):
+def roofline_of(env, name, wl, kernel, cells_launch, t_launch_s, clocks, launch_unit, gens=1):
     """The dominant kernel's roofline: algorithmic work of one launch over the
-    average launch duration in the timed region."""
+    average launch duration in the timed region.  `gens`:
+    generations one launch computes with one HBM read and one write of the
+    field (conv_tb2_kernel: 2), which multiplies the arithmetic, not the bytes."""
     peak_gbs, peak_src = load_peaks()
     bcell = wl["bcell"]
     hbm_ach = bcell * cells_launch / t_launch_s / 1e9
@@ -549,7 +551,8 @@ def roofline_of(env, name, wl, kernel, cells_launch, t_launch_s, clocks, launch_
                                                   "fraction is not a bound (it can exceed 1)"}}
     if wl["op"] == "conv":
         fma_cell = (2 * wl["r"] + 1) ** (3 if wl.get("d") else 2)
-        if fma_cell / bcell > 5.7:  # above the FMA/HBM balance (37.2 TFMA/s / 6.5 TB/s): FP32-FMA bound
+        if fma_cell * gens / bcell > 5.7:  # above the FMA/HBM balance (37.2 TFMA/s / 6.5 TB/s): FP32-FMA bound
+            fma_cell *= gens
             ach = 2.0 * fma_cell * cells_launch / t_launch_s / 1e12
             peak = 148 * 128 * 2 * mhz * 1e6 / 1e12
             return {"bound": "alu", **base, "achieved": ach, "peak": peak, "unit": "TFLOP/s", "frac": ach / peak,
@@ -751,6 +754,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         dclocks = env.sampler.region(dt0, dt1)
         dinfo = dg.info()
         dl = (dinfo.launches - dl0) // steps
+        dkernel = M.KERNEL_NAMES.get(dg.launch(0).kernel, "?")
         dg.close()
         d_ms = env.max_over_ranks(d_ms)
         d_value = units_per_step * steps / (d_ms / 1e3)
@@ -759,14 +763,56 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         if op == "life":
             droof = roofline_of(env, name, wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
                                 f"one pass = {K} generations ({dl} launches per step)")
+        elif dkernel == "conv_tb2_kernel":  # one launch = the two generations of a pass
+            droof = roofline_of(env, name + "_tb2", wl, dkernel, slab_cells, t_pass, dclocks,
+                                f"one pass = {K} generations in one launch ({dl} launches per step)", gens=K)
         else:
-            droof = roofline_of(env, name, wl, kernel, slab_cells, t_pass / K, dclocks,
+            droof = roofline_of(env, name, wl, dkernel, slab_cells, t_pass / K, dclocks,
                                 f"one generation (a pass = {K} launches; {dl} launches per step)")
         deep = {"generations_per_pass": int(dinfo.gens_per_pass), "halo_rows": int(dinfo.halo_rows),
                 "value": d_value, "unit": metric_of(wl)[1], "ms_per_step": d_ms / steps,
                 "vs_per_generation_path": d_value / value, "roofline": droof, "clocks": dclocks,
-                "hbm_bytes_per_cell_update": 0.25 / K if op == "life" else wl["bcell"],
+                "kernel": dkernel,
+                "hbm_bytes_per_cell_update": (0.25 / K if op == "life" else
+                                              wl["bcell"] / K if dkernel == "conv_tb2_kernel" else wl["bcell"]),
                 "exchanged_rows_per_pass": K * wl["r"]}
+
+    ring = None
+    if extras and world == 1 and op != "histogram" and wl["b"] == "wrap" and not d:
+        # The NCCL data plane on one GPU (include/mapsm.h, one-rank NCCL
+        # context): the WRAP row ring closes through ncclSend/ncclRecv to
+        # itself every generation — boundary rows first, the exchange group on
+        # the side stream, interior overlapped, all inside the CUDA graphs — so
+        # the multi-process path runs on hardware; exposure = the same steps
+        # with the exchange switched off.
+        rctx = M.mapsm_ctx_create(0, 1, env.local_rank, M.mapsm_nccl_unique_id(), env.stream.cuda_stream)
+        try:
+            rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W)
+            rg.bind(h_in)
+            for _ in range(warmup):
+                rg.iterate(n)
+            x0, l0 = rg.info().exchanges, rg.info().launches
+            r_ms, rt0, rt1 = env.timed(lambda: rg.iterate(n), steps)
+            rclocks = env.sampler.region(rt0, rt1)
+            rinfo = rg.info()
+            rg.set_option(M.OPT_NO_EXCHANGE, 1)
+            rg.iterate(n)
+            ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
+            rg.close()
+        finally:
+            M.mapsm_ctx_destroy(rctx)
+        r_step = r_ms / steps
+        ring = {"how": "one-rank NCCL communicator (mapsm_ctx_create with world 1 and an id): per generation a "
+                       "boundary-row launch, one NCCL group (send-up, send-down, recv-bottom, recv-top to rank 0) "
+                       "on the side stream, the interior launch overlapped; CUDA graphs",
+                "value": units_per_step * steps / (r_ms / 1e3), "unit": metric_of(wl)[1], "ms_per_step": r_step,
+                "vs_plain_path": (units_per_step * steps / (r_ms / 1e3)) / value,
+                "launches_per_step": (rinfo.launches - l0) // steps,
+                "halo_messages_per_step": (rinfo.exchanges - x0) // steps,
+                "halo_bytes_per_message": wl["r"] * int(info0.pitch_bytes),
+                "halo_exposure": {"ms_per_step_no_exchange": ne_ms / 2,
+                                  "exposed_pct": 100.0 * (r_step - ne_ms / 2) / r_step},
+                "clocks": rclocks}
 
     metric, unit_name = metric_of(wl)
     nbuf = 1 if op == "histogram" else 2
@@ -797,6 +843,8 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         line["halo_exposure"] = exposure
     if deep is not None:
         line["deep_halo"] = deep
+    if ring is not None:
+        line["nccl_ring"] = ring
     if chained is not None:
         line["chained_task"] = chained
     return line

@@ -202,7 +202,17 @@ mapsm_status mapsm_locmon_copied(mapsm_locmon m, int datum, int nops, const maps
 
 /* Multi-process mode: one process (rank of world) per GPU.  `nccl_unique_id`
  * is the 128-byte ncclUniqueId from mapsm_nccl_unique_id() on rank 0,
- * broadcast by the caller (e.g. torch.distributed); NULL iff world == 1.
+ * broadcast by the caller (e.g. torch.distributed); required when world > 1.
+ * world == 1 with an id (from mapsm_nccl_unique_id() in the same process)
+ * creates a one-rank NCCL communicator: the WRAP row ring then closes
+ * through NCCL, every pass sending the slab's first and last halo rows to
+ * itself and receiving its halos with ncclSend / ncclRecv in the order of
+ * mapsm_exchange_plan (send-up, send-down, recv-bottom, recv-top, peer 0) —
+ * the data plane of the multi-process mode (boundary rows first, exchange on
+ * the side stream, interior overlapped, CUDA graphs) executed on one GPU.
+ * Results are identical to world == 1 without an id (which maps the halo
+ * rows on the read side, no exchange); CLAMP / ZERO have no exchanged edge
+ * at world == 1 and are unaffected.  ENCCL if NCCL fails to initialise.
  * `cuda_stream` (a cudaStream_t, e.g. torch.cuda.current_stream().cuda_stream)
  * becomes the compute stream; NULL -> the library creates its own.  The
  * exchange runs on a library-owned side stream.                             */

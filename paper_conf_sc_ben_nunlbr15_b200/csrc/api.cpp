@@ -191,6 +191,25 @@ static char* row_ptr(const mapsm_grid_s* g, const Slab& s, int b, int64_t y) {
     return s.base[b] + (y + g->halo) * g->pitch;
 }
 
+// The partition of slab k of a grid.  A one-rank NCCL context (world == 1
+// with a communicator, mapsm.h) closes the WRAP row ring through NCCL: its
+// halos are exchanged with itself (up == down == 0, send-up / send-down /
+// recv-bottom / recv-top to rank 0, matched in issue order as between two
+// ranks) instead of the local read-side row map.
+static mapsm_status slab_plan(const mapsm_grid_s* g, int64_t halo, mapsm_boundary b, int k, mapsm_slab_plan* p) {
+    const mapsm_ctx c = g->ctx;
+    mapsm_status st = compute_plan(g->units(), c->g, (int)halo, b, k, p);
+    if (st != MAPSM_OK) return st;
+    if (!c->local && c->world == 1 && c->comm && b == MAPSM_WRAP && halo > 0) {
+        p->up = p->down = 0;
+        p->top_kind = p->bottom_kind = MAPSM_HALO_EXCHANGE;
+        p->top_src_row = g->units() - halo;
+        p->bottom_src_row = 0;
+        p->n_send = p->n_recv = 2;
+    }
+    return MAPSM_OK;
+}
+
 static bool has_exchange(const Slab& s) {
     return s.plan.top_kind == MAPSM_HALO_EXCHANGE || s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
 }
@@ -220,8 +239,7 @@ extern "C" mapsm_status mapsm_ctx_create(int rank, int world, int device, const 
     if (!out) return fail(MAPSM_EINVAL, "out is NULL");
     *out = nullptr;
     if (world < 1 || rank < 0 || rank >= world) return fail(MAPSM_EINVAL, "bad rank %d / world %d", rank, world);
-    if ((world > 1) != (nccl_unique_id != nullptr))
-        return fail(MAPSM_EINVAL, "nccl_unique_id must be given iff world > 1");
+    if (world > 1 && !nccl_unique_id) return fail(MAPSM_EINVAL, "nccl_unique_id must be given when world > 1");
     int ndev = 0;
     CK(cudaGetDeviceCount(&ndev));
     if (device < 0 || device >= ndev) return fail(MAPSM_EINVAL, "device %d out of range (%d devices)", device, ndev);
@@ -235,7 +253,7 @@ extern "C" mapsm_status mapsm_ctx_create(int rank, int world, int device, const 
     c->first_slab = rank;
     c->devices = {device};
     c->user_stream = static_cast<cudaStream_t>(cuda_stream);
-    if (world > 1) {
+    if (nccl_unique_id) {  // world == 1 with an id: the one-rank NCCL ring (mapsm.h)
         mapsm_status s = nccl_load();
         if (s != MAPSM_OK) {
             delete c;
@@ -374,7 +392,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
     // validate the partition for every slab before allocating anything
     for (int k = 0; k < c->g; ++k) {
         mapsm_slab_plan p;
-        if (compute_plan(g->units(), c->g, (int)halo, boundary, k, &p) != MAPSM_OK)
+        if (slab_plan(g, halo, boundary, k, &p) != MAPSM_OK)
             return fail(MAPSM_EINVAL, "cannot split %lld rows over %d slabs with %lld halo rows (need >= that many rows each)",
                         (long long)g->units(), c->g, (long long)halo);
     }
@@ -398,7 +416,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
         s.device = c->devices[c->local ? i : 0];
         // the plan's kinds / neighbours / rows do not depend on the halo
         // depth; alloc_rows does (rows + 2 * halo)
-        compute_plan(g->units(), c->g, (int)halo, boundary, s.rank, &s.plan);
+        slab_plan(g, halo, boundary, s.rank, &s.plan);
         CK(cudaSetDevice(s.device));
         CK(cudaDeviceGetAttribute(&s.num_sms, cudaDevAttrMultiProcessorCount, s.device));
         const size_t bytes = (size_t)s.plan.alloc_rows * (size_t)g->pitch;
@@ -779,7 +797,7 @@ static bool fused_now(const mapsm_grid_s* g) {
 static mapsm_status p2p_link(mapsm_grid_s* g) {
     if (g->p2p_linked) return MAPSM_OK;
     mapsm_ctx c = g->ctx;
-    if (c->local) {
+    if (c->local || c->world == 1) {  // (world == 1: the one-rank NCCL ring links to itself)
         for (auto& s : g->slabs) {
             if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
                 Slab& u = g->slabs[s.plan.up];

@@ -209,15 +209,18 @@ __global__ void __launch_bounds__(kThreads, 1) life_resident_kernel(const __grid
     const int up = (b - 1 + G) % G, down = (b + 1) % G;
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
 
-    // lane geometry: column chunk cx of 32 * kV words, row group rg
+    // lane geometry: column chunk cx of 32 * kV words, row group rg.  Rows
+    // wider than kWarps chunks (w > kWarps * 32 * kV * 32 cells = 32768 at
+    // 512 threads) give every warp the chunks cx, cx + kWarps, ... of all rows.
     const int nvec = nw / kV;
     const int ncx = (nvec + 31) / 32;
     const int ngr = kWarps / ncx > 0 ? kWarps / ncx : 1;
     const int cx = warp % ncx, rg = warp / ncx;
+    const int cstep = ncx > kWarps ? kWarps : ncx;  // (cx < ncx: one chunk when ncx <= kWarps)
     const bool has_work = warp < ncx * ngr;
-    Lane c;
-    {
-        const int vi = cx * 32 + lane;
+    auto lane_of = [&](int cxi) {
+        Lane c;
+        const int vi = cxi * 32 + lane;
         c.active = vi < nvec;
         c.w0 = c.active ? vi * kV : 0;
         const bool first = c.w0 == 0, last = c.w0 + kV == nw;
@@ -227,7 +230,8 @@ __global__ void __launch_bounds__(kThreads, 1) life_resident_kernel(const __grid
         c.rsh = (CM == COL_CLAMP && last) ? 31 : 0;
         c.lmask = (CM == COL_ZERO && first) ? 0u : ~0u;
         c.rmask = (CM == COL_ZERO && last) ? 0u : ~0u;
-    }
+        return c;
+    };
 
     // generation 0: rows [-K, R+K) on the torus; at a CLAMP / ZERO global edge
     // rows [-1, R+1) with row -1 / R the replicated / zero row (both buffers
@@ -259,7 +263,9 @@ __global__ void __launch_bounds__(kThreads, 1) life_resident_kernel(const __grid
         const int rr = rg - g0;
         if (!has_work || nr <= 0 || rr < 0 || rr >= ng) return;
         const int ys = a + rr * nr / ng, ye = a + (rr + 1) * nr / ng;
-        if (ys < ye) warp_gen<CM>(c, bcur + K * nw, bnxt + K * nw, nw, ys, ye, R, top_edge, bot_edge);
+        if (ys < ye)
+            for (int cxi = cx; cxi < ncx; cxi += cstep)
+                warp_gen<CM>(lane_of(cxi), bcur + K * nw, bnxt + K * nw, nw, ys, ye, R, top_edge, bot_edge);
     };
     auto two_bands = [&](int a0, int a1, int b0, int b1) {
         if (ngr >= 2) {

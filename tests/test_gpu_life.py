@@ -137,6 +137,28 @@ def test_resident_vs_oracle(ctx, b, shape, n):
     assert np.array_equal(out, oracle.life(g0, n, b))
 
 
+@pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
+@pytest.mark.parametrize("shape", [(65536, 256), (65536, 1024), (32768 + 4096, 300), (131072, 64), (32768, 500)])
+@pytest.mark.parametrize("persistent", [True, 2])
+def test_persistent_wide_rows_vs_oracle(ctx, b, shape, persistent):
+    """Rows wider than the resident kernel's warps cover in one chunk
+    (w > 512 threads x 64 cells = 32768): every warp then takes several
+    column chunks of each row.  Found by the one-rank NCCL ring test (its
+    65536 x 1024 grid disagreed with the plain context, whose resident kernel
+    left columns >= 32768 uncomputed).  Also the grid-barrier kernel (2)."""
+    w, h = shape
+    n = 5
+    g0 = mi.life_u8(4100 + w + h, w, h)
+    with M.Grid(ctx, w, h, "life", 1, b) as g:
+        g.set_option(M.OPT_PERSISTENT, persistent)
+        g.bind(g0)
+        g.iterate(n)
+        li = g.launch()
+        out = g.gather()
+    assert li.kernel == (M.KERNEL_LIFE_TB_PERSIST if persistent is True else M.KERNEL_LIFE_PERSIST)
+    assert np.array_equal(out, oracle.life(g0, n, b))
+
+
 def test_resident_split_calls_and_parity(ctx):
     """Several iterate calls (odd and even n) keep the buffer parity right."""
     g0 = mi.life_u8(17, 8192, 1024)

@@ -1,0 +1,122 @@
+"""GPU parity of the NCCL data plane on one B200: a one-rank NCCL communicator
+(mapsm_ctx_create(0, 1, dev, id, stream), include/mapsm.h) closes the WRAP row
+ring through ncclSend / ncclRecv to itself, so every pass runs exactly what a
+rank of the multi-process mode runs (boundary rows
+first, the exchange list of mapsm_exchange_plan issued in one NCCL group on
+the side stream, interior rows overlapped, CUDA graphs capturing the NCCL
+group) — the two-line boundary exchange of P:L461 §5.1 — with the peer being
+the rank itself.  Results are compared bit for bit with the CPU oracle
+(oracle/oracle.c) and with the same grid on the plain one-GPU context (which
+maps the halo rows on the read side and exchanges nothing).  Every case
+asserts that halo messages were actually exchanged."""
+import numpy as np
+import pytest
+
+import mapsm_inputs as mi
+import oracle
+from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def ring_ctx():
+    import torch
+
+    torch.cuda.set_device(0)
+    c = M.mapsm_ctx_create(0, 1, 0, M.mapsm_nccl_unique_id(), None)
+    yield c
+    M.mapsm_ctx_destroy(c)
+
+
+def run(c, op, w, h, r, b, x0, steps, W=None, K=1, graphs=True, p2p=False):
+    with M.Grid(c, w, h, op, r, b, W, deep_halo=K) as g:
+        if not graphs:
+            g.set_option(M.OPT_GRAPHS, 0)
+        if p2p:
+            g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
+        g.bind(x0)
+        for n in steps:
+            g.iterate(n)
+        out = g.gather()
+        info = g.info()
+    return out, info
+
+
+@pytest.mark.parametrize("graphs", [True, False])
+@pytest.mark.parametrize("w,h,n", [(256, 64, 9), (4096, 2048, 20), (1024 + 64, 333, 7)])
+def test_life_ring_vs_oracle(ring_ctx, graphs, w, h, n):
+    x0 = mi.life_u8(7100 + w + h, w, h)
+    out, info = run(ring_ctx, "life", w, h, 1, "wrap", x0, [n], graphs=graphs)
+    assert info.exchanges >= 2 * n, info.exchanges  # two halo receives per generation
+    assert np.array_equal(out, oracle.life(x0, n, "wrap"))
+
+
+@pytest.mark.parametrize("b", ["clamp", "zero"])
+def test_life_ring_non_wrap_unchanged(ring_ctx, b):
+    """No exchanged edge at world == 1 under CLAMP / ZERO: same result, no messages."""
+    x0 = mi.life_u8(7200, 512, 96)
+    out, info = run(ring_ctx, "life", 512, 96, 1, b, x0, [6])
+    assert info.exchanges == 0
+    assert np.array_equal(out, oracle.life(x0, 6, b))
+
+
+@pytest.mark.parametrize("r", [1, 2, 4, 6])
+def test_conv_ring_vs_oracle(ring_ctx, r):
+    w, h, n = 512 + 4, 8 * r + 37, 5
+    f0 = mi.field_f32(7300 + r, w, h)
+    W = mi.weights_f32(7310 + r, r)
+    out, info = run(ring_ctx, "conv", w, h, r, "wrap", f0, [2, n - 2], W=W)
+    assert info.exchanges >= 2 * n
+    assert np.array_equal(out.view(np.uint32), oracle.conv(f0, W, n, "wrap").view(np.uint32))
+
+
+@pytest.mark.parametrize("K", [2, 4, 8])
+def test_life_ring_deep_halo(ring_ctx, K):
+    """Deep halos over the NCCL ring: K rows exchanged once per pass."""
+    w, h, n = 2048, 4 * K + 50, 3 * K + 1
+    x0 = mi.life_u8(7400 + K, w, h)
+    out, info = run(ring_ctx, "life", w, h, 1, "wrap", x0, [n], K=K)
+    assert info.gens_per_pass == K and info.halo_rows == K
+    assert info.exchanges >= 2 * (n // K)
+    assert np.array_equal(out, oracle.life(x0, n, "wrap"))
+
+
+@pytest.mark.parametrize("r,K", [(2, 2), (1, 2), (2, 3)])
+def test_conv_ring_deep_halo(ring_ctx, r, K):
+    """conv deep halos over the NCCL ring (K = 2, r <= 2: the fused two-generation kernel)."""
+    w, h, n = 1024, 4 * K * r + 29, 2 * K + 1
+    f0 = mi.field_f32(7500 + 10 * r + K, w, h)
+    W = mi.weights_f32(7510 + r, r)
+    out, info = run(ring_ctx, "conv", w, h, r, "wrap", f0, [n], W=W, K=K)
+    assert info.halo_rows == K * r
+    assert info.exchanges >= 2 * (n // K)
+    assert np.array_equal(out.view(np.uint32), oracle.conv(f0, W, n, "wrap").view(np.uint32))
+
+
+@pytest.mark.parametrize("op,r", [("life", 1), ("conv", 2)])
+def test_ring_fused_p2p_self_link(ring_ctx, op, r):
+    """MAPSM_OPT_EXCHANGE = P2P on the one-rank ring: the boundary CTAs store their rows
+    into the slab's own halos and signal its own mailbox (no NCCL per pass)."""
+    w, h, n = 2048, 300, 11
+    if op == "life":
+        x0 = mi.life_u8(7600, w, h)
+        exp = oracle.life(x0, n, "wrap")
+        out, info = run(ring_ctx, op, w, h, 1, "wrap", x0, [n], p2p=True)
+        assert np.array_equal(out, exp)
+    else:
+        x0 = mi.field_f32(7610, w, h)
+        W = mi.weights_f32(7611, r)
+        out, info = run(ring_ctx, op, w, h, r, "wrap", x0, [n], W=W, p2p=True)
+        assert np.array_equal(out.view(np.uint32), oracle.conv(x0, W, n, "wrap").view(np.uint32))
+    assert info.exchanges >= 2 * n
+
+
+def test_ring_equals_plain_context(ring_ctx, ctx):
+    """The ring and the read-side row map give the same generation (65536-wide rows, 3 full TMA trips)."""
+    w, h, n = 65536, 1024, 6
+    x0 = mi.life_u8(7700, w, h)
+    a, ia = run(ring_ctx, "life", w, h, 1, "wrap", x0, [n])
+    b, ib = run(ctx, "life", w, h, 1, "wrap", x0, [n])
+    assert ia.exchanges > 0 and ib.exchanges == 0
+    assert np.array_equal(a, b)
