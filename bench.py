@@ -795,6 +795,10 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
             r_ms, rt0, rt1 = env.timed(lambda: rg.iterate(n), steps)
             rclocks = env.sampler.region(rt0, rt1)
             rinfo = rg.info()
+            rg.set_option(M.OPT_EXCHANGE_SMS, 0)
+            rg.iterate(n)
+            ser_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
+            rg.set_option(M.OPT_EXCHANGE_SMS, -1)
             rg.set_option(M.OPT_NO_EXCHANGE, 1)
             rg.iterate(n)
             ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
@@ -802,9 +806,11 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         finally:
             M.mapsm_ctx_destroy(rctx)
         r_step = r_ms / steps
-        ring = {"how": "one-rank NCCL communicator (mapsm_ctx_create with world 1 and an id): per generation a "
-                       "boundary-row launch, one NCCL group (send-up, send-down, recv-bottom, recv-top to rank 0) "
-                       "on the side stream, the interior launch overlapped; CUDA graphs",
+        ring = {"how": "one-rank NCCL communicator (mapsm_ctx_create with world 1 and an id): per generation the "
+                       "boundary rows and one NCCL group (send-up, send-down, recv-bottom, recv-top to rank 0) on "
+                       "the side stream on a few SMs, the interior on the others (concurrent-boundary schedule, "
+                       "MAPSM_OPT_EXCHANGE_SMS default); CUDA graphs",
+                "serial_ms_per_step": ser_ms / 2,
                 "value": units_per_step * steps / (r_ms / 1e3), "unit": metric_of(wl)[1], "ms_per_step": r_step,
                 "vs_plain_path": (units_per_step * steps / (r_ms / 1e3)) / value,
                 "launches_per_step": (rinfo.launches - l0) // steps,
@@ -851,6 +857,9 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
 
 
 def main():
+    # NCCL's own log lines (e.g. the version banner under NCCL_DEBUG=VERSION)
+    # go to stdout by default; stdout carries only the JSON line
+    os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
     ap.add_argument("--steps", type=int, default=10)

@@ -473,6 +473,21 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         several grids of one ctx overlap (e.g. one grid's
  *                         upload with another's compute and a third's
  *                         download); 0 (default): the ctx stream
+ *   MAPSM_OPT_EXCHANGE_SMS  k in -1..64, one slab per process (multi-process
+ *                         NCCL mode or the one-rank ring).  k > 0: the
+ *                         concurrent-boundary schedule — generation t's
+ *                         boundary rows and their NCCL exchange run on the
+ *                         side stream on k SMs while the interior runs on
+ *                         the other SMs; the interior of t waits only for
+ *                         the boundary rows of t-1, the boundary rows of t
+ *                         for the interior and halos of t-1.  k = 0: serial
+ *                         (boundary, then exchange beside the interior — which
+ *                         fills every SM, so NCCL's kernel waits for it).
+ *                         -1 (default): 2 for Life, 4 for the 2-D conv r <= 4,
+ *                         0 otherwise (measured).  With
+ *                         MAPSM_EXCHANGE_P2P, k > 0 (explicit only) runs the
+ *                         boundary launch with the fused peer stores beside
+ *                         the interior instead of one fused launch.
  *   MAPSM_OPT_DEEP_HALO   K > 1 (1 = off, default): the grid keeps K*r halo
  *                         rows per side and exchanges them once per pass of
  *                         K generations instead of r rows every generation
@@ -502,7 +517,8 @@ typedef enum {
     MAPSM_OPT_PERSISTENT = 5,
     MAPSM_OPT_EXCHANGE = 6,
     MAPSM_OPT_DEEP_HALO = 7,
-    MAPSM_OPT_OWN_STREAM = 8
+    MAPSM_OPT_OWN_STREAM = 8,
+    MAPSM_OPT_EXCHANGE_SMS = 9
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

@@ -92,6 +92,7 @@ struct Slab {
     cudaStream_t main = nullptr, side = nullptr;
     bool own_main = false;
     cudaEvent_t ev_b = nullptr, ev_h = nullptr;
+    cudaEvent_t ev_i = nullptr;  // interior launch done (concurrent-boundary schedule)
     cudaGraphExec_t graph[2] = {nullptr, nullptr};
     int64_t graph_iters = 0;
     cudaGraphExec_t graph_tb[2] = {nullptr, nullptr};  // deep-halo passes (K generations each)
@@ -140,6 +141,8 @@ struct mapsm_grid_s {
     int opt_persistent_mode = 1;  // 1: SMEM-resident kernel when the slab fits, 2: grid-barrier kernel only
     bool opt_own_stream = false;  // the grid's slabs use private streams instead of the ctx stream
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
+    int opt_exchange_sms = -1;  // SMs the interior launch leaves to the exchange in flight (-1: auto)
+    bool conc_open = false;     // concurrent-boundary schedule: the side stream is forked from main
     int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
     int64_t halo = 0;           // halo rows allocated above/below each slab (r, or K*r with deep halos)
     bool deep_valid = false;    // the current buffer's halos are valid to depth `halo` (else only r)
@@ -363,6 +366,7 @@ static void free_slab(Slab& s) {
     for (auto& t : s.t_bnd) { cudaEventDestroy(t.a); cudaEventDestroy(t.b); }
     if (s.ev_b) cudaEventDestroy(s.ev_b);
     if (s.ev_h) cudaEventDestroy(s.ev_h);
+    if (s.ev_i) cudaEventDestroy(s.ev_i);
     if (s.side) cudaStreamDestroy(s.side);
     if (s.own_main && s.main) cudaStreamDestroy(s.main);
     s = Slab();
@@ -449,6 +453,7 @@ static mapsm_status alloc_slabs(mapsm_grid_s* g, int radius, mapsm_boundary boun
         CK(cudaStreamCreateWithFlags(&s.side, cudaStreamNonBlocking));
         CK(cudaEventCreateWithFlags(&s.ev_b, cudaEventDisableTiming));
         CK(cudaEventCreateWithFlags(&s.ev_h, cudaEventDisableTiming));
+        CK(cudaEventCreateWithFlags(&s.ev_i, cudaEventDisableTiming));
     }
     // slabs sharing a device split its SMs (their kernels run concurrently)
     for (auto& s : g->slabs) {
@@ -627,7 +632,9 @@ static bool conv_tb2_ok(const mapsm_grid_s* g) {
 }
 
 static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBands& bands, bool bulk,
-                                const FusedLink* link = nullptr, int K = 1) {
+                                const FusedLink* link = nullptr, int K = 1, cudaStream_t on = nullptr,
+                                int sms = 0) {
+    cudaStream_t st = on ? on : s.main;
     StencilGeom geom;
     geom.in = row_ptr(g, s, b_in, 0);
     geom.out = row_ptr(g, s, b_in ^ 1, 0);
@@ -652,23 +659,25 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
             vec.push_back(t);
         }
         tp = &vec[used++];
-        CK(cudaEventRecord(tp->a, s.main));
+        CK(cudaEventRecord(tp->a, st));
     }
     cudaError_t e;
+    int nsm = sms > 0 ? sms : s.num_sms;
+
     if (g->op == MAPSM_OP_CONV && K == 2 && conv_tb2_ok(g))
         e = launch_conv_tb2(geom, bands, g->r, s.plan.top_kind == MAPSM_HALO_ZERO, s.plan.bottom_kind == MAPSM_HALO_ZERO,
-                            s.num_sms, s.main);
+                            nsm, st);
     else if (g->op == MAPSM_OP_LIFE && K > 1)
         e = launch_life_tb(geom, bands, K, s.plan.top_kind == MAPSM_HALO_ZERO, s.plan.bottom_kind == MAPSM_HALO_ZERO,
-                           s.num_sms, s.main);
+                           nsm, st);
     else if (g->op == MAPSM_OP_LIFE)
-        e = launch_life_step(geom, bands, s.num_sms, s.main, link);
+        e = launch_life_step(geom, bands, nsm, st, link);
     else if (g->d)
-        e = launch_conv3d(geom, bands, g->r, g->wt, s.num_sms, s.main);
+        e = launch_conv3d(geom, bands, g->r, g->wt, nsm, st);
     else
-        e = launch_conv_step(geom, bands, g->r, g->wt, s.num_sms, s.main, link);
+        e = launch_conv_step(geom, bands, g->r, g->wt, nsm, st, link);
     if (e != cudaSuccess) return fail(MAPSM_ECUDA, "stencil launch: %s", cudaGetErrorString(e));
-    if (tp) CK(cudaEventRecord(tp->b, s.main));
+    if (tp) CK(cudaEventRecord(tp->b, st));
     g->launches++;
     return MAPSM_OK;
 }
@@ -695,11 +704,79 @@ static void split_bands(const Slab& s, int64_t r, RowBands& bnd, RowBands& inner
 // depth K*r, exchanged once per pass).
 static mapsm_status pass_conv_deep(mapsm_grid_s* g, int b_in, int K);
 
+// Concurrent-boundary schedule (NCCL mode, MAPSM_OPT_EXCHANGE_SMS = k > 0):
+// generation t's boundary rows B(t) and its NCCL exchange X(t) run on the
+// side stream on k SMs while the interior I(t) runs on the main stream on the
+// other SMs.  B(t) reads I(t-1)'s rows and the halos X(t-1) delivered (side
+// stream order); I(t) reads B(t-1)'s rows (not the halos).  So the chain
+// I(t-1) -> I(t) -> ... is never held up by an exchange as long as B + X
+// fit under I: per generation
+//     side: wait I(t-1); B(t); record ev_b; X(t)
+//     main: wait B(t-1);  I(t); record ev_i
+// (issued main-wait first, so each wait sees the previous generation's
+// record).  The side stream is forked from main on first use and joined back
+// at the end of mapsm_iterate / of a captured graph (join_side).
+static mapsm_status fork_side(mapsm_grid_s* g) {
+    if (g->conc_open) return MAPSM_OK;
+    Slab& s = g->slabs[0];
+    CK(cudaEventRecord(s.ev_i, s.main));
+    CK(cudaEventRecord(s.ev_b, s.main));
+    CK(cudaStreamWaitEvent(s.side, s.ev_i, 0));
+    g->conc_open = true;
+    return MAPSM_OK;
+}
+
+static mapsm_status join_side(mapsm_grid_s* g) {
+    if (!g->conc_open) return MAPSM_OK;
+    Slab& s = g->slabs[0];
+    DeviceGuard dg;
+    CK(cudaSetDevice(s.device));
+    CK(cudaEventRecord(s.ev_h, s.side));
+    CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
+    g->conc_open = false;
+    return MAPSM_OK;
+}
+
+// MAPSM_OPT_EXCHANGE_SMS, resolved: -1 (default) = measured choice for the
+// 2-D TMA kernels (Life 2, conv r <= 4: 4), 0 elsewhere.
+static int exchange_sms(const mapsm_grid_s* g) {
+    if (g->opt_exchange_sms >= 0) return g->opt_exchange_sms;
+    if (g->d) return 0;
+    if (g->op == MAPSM_OP_LIFE) return 2;
+    if (g->op == MAPSM_OP_CONV && g->r <= 4) return 4;
+    return 0;
+}
+
+static bool concurrent_boundary(const mapsm_grid_s* g) {
+    return exchange_sms(g) > 0 && !g->ctx->local && !g->opt_timing && !g->opt_no_exchange && !g->opt_p2p &&
+           g->slabs.size() == 1 && has_exchange(g->slabs[0]) && g->slabs[0].num_sms > exchange_sms(g);
+}
+
+static mapsm_status iterate_concurrent(mapsm_grid_s* g, int b_in, int K, int64_t depth) {
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    TRY(fork_side(g));
+    RowBands bnd, inner;
+    split_bands(s, depth, bnd, inner);
+    CK(cudaStreamWaitEvent(s.main, s.ev_b, 0));  // I(t) after B(t-1)
+    CK(cudaStreamWaitEvent(s.side, s.ev_i, 0));  // B(t) after I(t-1)
+    const int k = exchange_sms(g);
+    TRY(launch_step(g, s, b_in, bnd, false, nullptr, K, s.side, k));
+    CK(cudaEventRecord(s.ev_b, s.side));
+    TRY(exchange_nccl(g, b_in ^ 1, depth));
+    if (inner.nbands > 0 && inner.end[0] > inner.begin[0])
+        TRY(launch_step(g, s, b_in, inner, true, nullptr, K, s.main, s.num_sms - k));
+    CK(cudaEventRecord(s.ev_i, s.main));
+    return MAPSM_OK;
+}
+
 // xdepth > 0: exchange that many rows (the last generation of a conv deep-halo pass)
 static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1, int64_t xdepth = 0) {
     if (K > 1 && g->op == MAPSM_OP_CONV && !conv_tb2_ok(g)) return pass_conv_deep(g, b_in, K);
     mapsm_ctx c = g->ctx;
     const int64_t depth = xdepth > 0 ? xdepth : (int64_t)g->r * K;
+    if (xdepth == 0 && concurrent_boundary(g)) return iterate_concurrent(g, b_in, K, depth);
+    TRY(join_side(g));  // (a trapezoid pass after concurrent generations)
     const bool exch = !g->opt_no_exchange;
     bool any_exchange = false;
     for (auto& s : g->slabs) any_exchange |= has_exchange(s);
@@ -757,6 +834,7 @@ static mapsm_status iterate_once(mapsm_grid_s* g, int b_in, int K = 1, int64_t x
 // computed by the same kernel as in K single generations: bit-identical.
 static mapsm_status pass_conv_deep(mapsm_grid_s* g, int b_in, int K) {
     const int64_t r = g->r;
+    TRY(join_side(g));
     int b = b_in;
     for (int j = 1; j < K; ++j) {
         for (auto& s : g->slabs) {
@@ -866,6 +944,22 @@ static mapsm_status p2p_link(mapsm_grid_s* g) {
     return MAPSM_OK;
 }
 
+// The peer-memory link of slab s for a launch writing buffer bo: the
+// neighbours' halo rows of bo and their mailboxes.
+static FusedLink fused_link(const mapsm_grid_s* g, const Slab& s, int bo) {
+    const int r = g->r;
+    const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+    FusedLink L;
+    L.mailbox = s.mailbox;
+    L.dst_up = top ? s.up_base[bo] + (s.up_rows + g->halo) * g->pitch : nullptr;  // up's row up_rows (bottom halo)
+    L.dst_down = bot ? s.down_base[bo] + (g->halo - r) * g->pitch : nullptr;      // down's row -r (top halo)
+    L.sig_up = top ? reinterpret_cast<unsigned int*>(s.up_mail + 16) : nullptr;      // recv_bot
+    L.sig_down = bot ? reinterpret_cast<unsigned int*>(s.down_mail + 12) : nullptr;  // recv_top
+    L.wait_top = top;
+    L.wait_bot = bot;
+    return L;
+}
+
 // One fused iteration: per slab ONE launch with bands [top boundary rows,
 // bottom boundary rows, interior]; the boundary CTAs deliver their rows into
 // the neighbours' halos of the output buffer and signal their mailboxes.
@@ -883,22 +977,47 @@ static mapsm_status iterate_fused(mapsm_grid_s* g, int b_in) {
         bands.begin[bands.nbands] = top ? r : 0;
         bands.end[bands.nbands] = bot ? rows - r : rows;
         bands.nbands++;
-        FusedLink L;
-        L.mailbox = s.mailbox;
-        L.dst_up = top ? s.up_base[bo] + (s.up_rows + g->halo) * g->pitch : nullptr;  // up's row up_rows (bottom halo)
-        L.dst_down = bot ? s.down_base[bo] + (g->halo - r) * g->pitch : nullptr;      // down's row -r (top halo)
-        L.sig_up = top ? reinterpret_cast<unsigned int*>(s.up_mail + 16) : nullptr;      // recv_bot
-        L.sig_down = bot ? reinterpret_cast<unsigned int*>(s.down_mail + 12) : nullptr;  // recv_top
-        L.wait_top = top;
-        L.wait_bot = bot;
+        const FusedLink L = fused_link(g, s, bo);
         TRY(launch_step(g, s, b_in, bands, true, &L));
         g->exchanges += s.plan.n_recv;
     }
     return MAPSM_OK;
 }
 
+// The concurrent-boundary schedule with the exchange fused into the boundary
+// launch (MAPSM_OPT_EXCHANGE = P2P with MAPSM_OPT_EXCHANGE_SMS = k > 0): B(t)
+// on the side stream on k SMs computes the boundary rows, stores them into
+// the neighbours' halos (NVLink peer stores / same-process stores) and
+// signals their mailboxes — its producers wait for the neighbours' B(t-1)
+// deliveries before loading halo rows — while I(t) runs on the other SMs.
+// No NCCL kernel on the chain: per generation it is B alone beside I.
+static bool concurrent_p2p(const mapsm_grid_s* g) {
+    return g->opt_exchange_sms > 0 && fused_now(g) && !g->ctx->local && !g->opt_timing && g->slabs.size() == 1 &&
+           g->slabs[0].num_sms > g->opt_exchange_sms;
+}
+
+static mapsm_status iterate_concurrent_p2p(mapsm_grid_s* g, int b_in) {
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    TRY(fork_side(g));
+    RowBands bnd, inner;
+    split_bands(s, g->r, bnd, inner);
+    const FusedLink L = fused_link(g, s, b_in ^ 1);
+    CK(cudaStreamWaitEvent(s.main, s.ev_b, 0));  // I(t) after B(t-1)
+    CK(cudaStreamWaitEvent(s.side, s.ev_i, 0));  // B(t) after I(t-1)
+    const int k = g->opt_exchange_sms;
+    TRY(launch_step(g, s, b_in, bnd, false, &L, 1, s.side, k));
+    CK(cudaEventRecord(s.ev_b, s.side));
+    g->exchanges += s.plan.n_recv;
+    if (inner.nbands > 0 && inner.end[0] > inner.begin[0])
+        TRY(launch_step(g, s, b_in, inner, true, nullptr, 1, s.main, s.num_sms - k));
+    CK(cudaEventRecord(s.ev_i, s.main));
+    return MAPSM_OK;
+}
+
 static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
-    return fused_now(g) ? iterate_fused(g, b_in) : iterate_once(g, b_in);
+    if (fused_now(g)) return concurrent_p2p(g) ? iterate_concurrent_p2p(g, b_in) : iterate_fused(g, b_in);
+    return iterate_once(g, b_in);
 }
 
 // Deep-halo passes apply: Life with TMA-kernel rows (w % 128 == 0), every slab
@@ -951,6 +1070,7 @@ static int pass_flips(const mapsm_grid_s* g, int K) {
 
 static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64_t iters, int K = 1) {
     CK(cudaSetDevice(s.device));
+    TRY(join_side(g));
     const int64_t l0 = g->launches, x0 = g->exchanges;
     CK(cudaStreamBeginCapture(s.main, cudaStreamCaptureModeThreadLocal));
     mapsm_status st = MAPSM_OK;
@@ -959,6 +1079,8 @@ static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64
         st = K > 1 ? iterate_once(g, cur, K) : step_all(g, cur);
         cur ^= K > 1 ? pass_flips(g, K) : 1;
     }
+    if (st == MAPSM_OK) st = join_side(g);
+    g->conc_open = false;
     cudaGraph_t graph = nullptr;
     cudaError_t e = cudaStreamEndCapture(s.main, &graph);
     g->launches = l0;
@@ -978,8 +1100,16 @@ static mapsm_status capture_graph(mapsm_grid_s* g, Slab& s, int start_cur, int64
     return MAPSM_OK;
 }
 
+static mapsm_status iterate_impl(mapsm_grid_s* g, int64_t n);
+
 extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
     if (!g) return fail(MAPSM_EINVAL, "grid is NULL");
+    mapsm_status st = iterate_impl(g, n);
+    mapsm_status sj = join_side(g);
+    return st != MAPSM_OK ? st : sj;
+}
+
+static mapsm_status iterate_impl(mapsm_grid_s* g, int64_t n) {
     if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "iterate before bind");
     if (n < 0) return fail(MAPSM_EINVAL, "n < 0");
     if (n == 0) return MAPSM_OK;
@@ -1105,7 +1235,7 @@ extern "C" mapsm_status mapsm_iterate(mapsm_grid g, int64_t n) {
             // launches per iteration (for the counters; graphs replay them)
             RowBands bnd, inner;
             split_bands(s, g->r, bnd, inner);
-            per_graph_launches = (has_exchange(s) && !fused_now(g))
+            per_graph_launches = (has_exchange(s) && (!fused_now(g) || concurrent_p2p(g)))
                                      ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0))
                                      : 1;
             per_graph_exch = (has_exchange(s) && !g->opt_no_exchange) ? s.plan.n_recv : 0;
@@ -1762,6 +1892,11 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
         case MAPSM_OPT_TIMING:
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;
+            break;
+        case MAPSM_OPT_EXCHANGE_SMS:
+            if (v < -1 || v > 64) return fail(MAPSM_EINVAL, "exchange SMs %lld (-1..64)", (long long)v);
+            g->opt_exchange_sms = (int)v;
+            drop_graphs(g);
             break;
         case MAPSM_OPT_OWN_STREAM: {
             g->opt_own_stream = v != 0;

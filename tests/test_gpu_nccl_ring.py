@@ -120,3 +120,50 @@ def test_ring_equals_plain_context(ring_ctx, ctx):
     b, ib = run(ctx, "life", w, h, 1, "wrap", x0, [n])
     assert ia.exchanges > 0 and ib.exchanges == 0
     assert np.array_equal(a, b)
+
+
+@pytest.mark.parametrize("p2p", [False, True])
+@pytest.mark.parametrize("k", [1, 2, 4])
+@pytest.mark.parametrize("op,r,w,h", [("life", 1, 65536, 300), ("life", 1, 2048, 77), ("conv", 2, 4096, 90),
+                                      ("conv", 4, 1024 + 4, 61)])
+@pytest.mark.parametrize("graphs", [True, False])
+def test_ring_concurrent_boundary(ring_ctx, p2p, k, op, r, w, h, graphs):
+    """MAPSM_OPT_EXCHANGE_SMS = k: the boundary rows (and the NCCL group, or
+    the fused peer stores) on the side stream on k SMs while the interior runs
+    on the others; generation t's interior waits only for t-1's boundary rows
+    and t's boundary rows for t-1's interior and halos.  Odd / even n over
+    several calls (the side stream is forked and joined per call)."""
+    W = mi.weights_f32(7800 + r, r) if op == "conv" else None
+    x0 = mi.field_f32(7810 + w, w, h) if op == "conv" else mi.life_u8(7810 + w, w, h)
+    steps = [5, 20, 1]
+    n = sum(steps)
+    with M.Grid(ring_ctx, w, h, op, r, "wrap", W) as g:
+        if not graphs:
+            g.set_option(M.OPT_GRAPHS, 0)
+        if p2p:
+            g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
+        g.set_option(M.OPT_EXCHANGE_SMS, k)
+        g.bind(x0)
+        for s in steps:
+            g.iterate(s)
+        out = g.gather()
+        info = g.info()
+    exp = oracle.conv(x0, W, n, "wrap") if op == "conv" else oracle.life(x0, n, "wrap")
+    assert info.exchanges >= 2 * n and info.launches == 2 * n
+    assert np.array_equal(out.view(np.uint8), exp.view(np.uint8))
+
+
+@pytest.mark.parametrize("op,r,K", [("life", 1, 4), ("life", 1, 8), ("conv", 2, 2), ("conv", 1, 2)])
+def test_ring_concurrent_deep_halo(ring_ctx, op, r, K):
+    """The concurrent schedule on deep-halo passes (boundary band K*r rows)."""
+    w, h = 4096, 6 * K * r + 31
+    W = mi.weights_f32(7900 + r, r) if op == "conv" else None
+    x0 = mi.field_f32(7910, w, h) if op == "conv" else mi.life_u8(7910, w, h)
+    n = 5 * K + 1
+    with M.Grid(ring_ctx, w, h, op, r, "wrap", W, deep_halo=K) as g:
+        g.set_option(M.OPT_EXCHANGE_SMS, 2)
+        g.bind(x0)
+        g.iterate(n)
+        out = g.gather()
+    exp = oracle.conv(x0, W, n, "wrap") if op == "conv" else oracle.life(x0, n, "wrap")
+    assert np.array_equal(out.view(np.uint8), exp.view(np.uint8))
