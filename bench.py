@@ -803,6 +803,15 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
             rg.iterate(n)
             ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
             rg.close()
+            dring = None
+            if op == "life" and args.deep_halo > 1:  # deep halos over the same ring: one exchange per K generations
+                rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W, deep_halo=args.deep_halo)
+                rg.bind(h_in)
+                rg.iterate(n)
+                dr_ms, _, _ = env.timed(lambda: rg.iterate(n), 3)
+                dring = {"generations_per_pass": args.deep_halo, "ms_per_step": dr_ms / 3,
+                         "value": units_per_step * 3 / (dr_ms / 1e3)}
+                rg.close()
         finally:
             M.mapsm_ctx_destroy(rctx)
         r_step = r_ms / steps
@@ -819,6 +828,8 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                 "halo_exposure": {"ms_per_step_no_exchange": ne_ms / 2,
                                   "exposed_pct": 100.0 * (r_step - ne_ms / 2) / r_step},
                 "clocks": rclocks}
+        if dring is not None:
+            ring["deep_halo"] = dring
 
     metric, unit_name = metric_of(wl)
     nbuf = 1 if op == "histogram" else 2

@@ -508,7 +508,7 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         per-generation kernels.  EUNSUPPORTED for non-Life
  *                         grids or other K; not combined with EXCHANGE_P2P
  *                         (the fused path then runs per generation).         */
-typedef enum { MAPSM_EXCHANGE_COPY = 0, MAPSM_EXCHANGE_P2P = 1 } mapsm_exchange;
+typedef enum { MAPSM_EXCHANGE_COPY = 0, MAPSM_EXCHANGE_P2P = 1, MAPSM_EXCHANGE_CE = 2 } mapsm_exchange;
 typedef enum {
     MAPSM_OPT_GRAPHS = 1,
     MAPSM_OPT_GRAPH_ITERS = 2,

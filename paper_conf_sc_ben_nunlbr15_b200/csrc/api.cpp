@@ -141,6 +141,7 @@ struct mapsm_grid_s {
     int opt_persistent_mode = 1;  // 1: SMEM-resident kernel when the slab fits, 2: grid-barrier kernel only
     bool opt_own_stream = false;  // the grid's slabs use private streams instead of the ctx stream
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
+    bool opt_ce = false;        // ... with the rows moved by copy-engine peer copies (MAPSM_EXCHANGE_CE)
     int opt_exchange_sms = -1;  // SMs the interior launch leaves to the exchange in flight (-1: auto)
     bool conc_open = false;     // concurrent-boundary schedule: the side stream is forked from main
     int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
@@ -748,7 +749,7 @@ static int exchange_sms(const mapsm_grid_s* g) {
 }
 
 static bool concurrent_boundary(const mapsm_grid_s* g) {
-    return exchange_sms(g) > 0 && !g->ctx->local && !g->opt_timing && !g->opt_no_exchange && !g->opt_p2p &&
+    return exchange_sms(g) > 0 && !g->ctx->local && !g->opt_timing && !g->opt_p2p &&
            g->slabs.size() == 1 && has_exchange(g->slabs[0]) && g->slabs[0].num_sms > exchange_sms(g);
 }
 
@@ -763,7 +764,7 @@ static mapsm_status iterate_concurrent(mapsm_grid_s* g, int b_in, int K, int64_t
     const int k = exchange_sms(g);
     TRY(launch_step(g, s, b_in, bnd, false, nullptr, K, s.side, k));
     CK(cudaEventRecord(s.ev_b, s.side));
-    TRY(exchange_nccl(g, b_in ^ 1, depth));
+    if (!g->opt_no_exchange) TRY(exchange_nccl(g, b_in ^ 1, depth));
     if (inner.nbands > 0 && inner.end[0] > inner.begin[0])
         TRY(launch_step(g, s, b_in, inner, true, nullptr, K, s.main, s.num_sms - k));
     CK(cudaEventRecord(s.ev_i, s.main));
@@ -1015,7 +1016,56 @@ static mapsm_status iterate_concurrent_p2p(mapsm_grid_s* g, int b_in) {
     return MAPSM_OK;
 }
 
+// Host-initiated peer copies (MAPSM_EXCHANGE_CE; the paper's P2P copies,
+// P:L51 §2.1 "large host-initiated P2P copies"), in the concurrent-boundary
+// schedule: B(t) on the side stream on k SMs — its producers wait until the
+// neighbours' generation counts (in my mailbox) reach mine, i.e. their
+// B(t-1) rows have landed in my halos — then the copy engines move my r
+// first / last rows into the neighbours' halos (cudaMemcpyAsync over NVLink
+// through the CUDA-IPC mappings) followed by my generation count into their
+// mailboxes, while I(t) runs on the other SMs.  No NCCL kernel and no SM
+// time for the transfer.  Ordering: a generation count is the number of
+// completed B launches.  A neighbour's copy at t (into my halos of buffer
+// (t+1) % 2, which my B(t-1) read) follows its B(t), whose producers waited
+// for its count of me to reach t — written only after my B(t-1) finished;
+// so a sender is at most one generation ahead and never overwrites halos
+// still being read.
+static mapsm_status iterate_concurrent_ce(mapsm_grid_s* g, int b_in) {
+    Slab& s = g->slabs[0];
+    CK(cudaSetDevice(s.device));
+    TRY(fork_side(g));
+    const int r = g->r;
+    const int bo = b_in ^ 1;
+    RowBands bnd, inner;
+    split_bands(s, r, bnd, inner);
+    FusedLink L = fused_link(g, s, bo);
+    L.dst_up = L.dst_down = nullptr;  // no peer stores in the kernel
+    L.sig_up = L.sig_down = nullptr;
+    L.ce = 1;
+    const int k = exchange_sms(g) > 0 ? exchange_sms(g) : 2;
+    CK(cudaStreamWaitEvent(s.main, s.ev_b, 0));  // I(t) after B(t-1)
+    CK(cudaStreamWaitEvent(s.side, s.ev_i, 0));  // B(t) after I(t-1)
+    TRY(launch_step(g, s, b_in, bnd, false, &L, 1, s.side, k));
+    CK(cudaEventRecord(s.ev_b, s.side));
+    const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+    const size_t rb = (size_t)r * (size_t)g->pitch;
+    if (top)
+        CK(cudaMemcpyAsync(s.up_base[bo] + (s.up_rows + g->halo) * g->pitch, row_ptr(g, s, bo, 0), rb,
+                           cudaMemcpyDefault, s.side));
+    if (bot)
+        CK(cudaMemcpyAsync(s.down_base[bo] + (g->halo - r) * g->pitch, row_ptr(g, s, bo, s.plan.rows - r), rb,
+                           cudaMemcpyDefault, s.side));
+    if (top) CK(cudaMemcpyAsync(s.up_mail + 16, s.mailbox, 4, cudaMemcpyDefault, s.side));   // -> up's recv_bot
+    if (bot) CK(cudaMemcpyAsync(s.down_mail + 12, s.mailbox, 4, cudaMemcpyDefault, s.side)); // -> down's recv_top
+    g->exchanges += s.plan.n_recv;
+    if (inner.nbands > 0 && inner.end[0] > inner.begin[0])
+        TRY(launch_step(g, s, b_in, inner, true, nullptr, 1, s.main, s.num_sms - k));
+    CK(cudaEventRecord(s.ev_i, s.main));
+    return MAPSM_OK;
+}
+
 static mapsm_status step_all(mapsm_grid_s* g, int b_in) {
+    if (fused_now(g) && g->opt_ce) return iterate_concurrent_ce(g, b_in);
     if (fused_now(g)) return concurrent_p2p(g) ? iterate_concurrent_p2p(g, b_in) : iterate_fused(g, b_in);
     return iterate_once(g, b_in);
 }
@@ -1235,7 +1285,7 @@ static mapsm_status iterate_impl(mapsm_grid_s* g, int64_t n) {
             // launches per iteration (for the counters; graphs replay them)
             RowBands bnd, inner;
             split_bands(s, g->r, bnd, inner);
-            per_graph_launches = (has_exchange(s) && (!fused_now(g) || concurrent_p2p(g)))
+            per_graph_launches = (has_exchange(s) && (!fused_now(g) || concurrent_p2p(g) || g->opt_ce))
                                      ? (1 + ((inner.nbands > 0 && inner.end[0] > inner.begin[0]) ? 1 : 0))
                                      : 1;
             per_graph_exch = (has_exchange(s) && !g->opt_no_exchange) ? s.plan.n_recv : 0;
@@ -1884,10 +1934,14 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             g->opt_persistent_mode = v == 2 ? 2 : 1;
             break;
         case MAPSM_OPT_EXCHANGE:
-            if (v != MAPSM_EXCHANGE_COPY && v != MAPSM_EXCHANGE_P2P) return fail(MAPSM_EINVAL, "exchange mode %lld", (long long)v);
-            if (g->state >= ST_BOUND && (v == MAPSM_EXCHANGE_P2P) != g->opt_p2p)
+            if (v != MAPSM_EXCHANGE_COPY && v != MAPSM_EXCHANGE_P2P && v != MAPSM_EXCHANGE_CE)
+                return fail(MAPSM_EINVAL, "exchange mode %lld", (long long)v);
+            if (v == MAPSM_EXCHANGE_CE && g->ctx->local)
+                return fail(MAPSM_EUNSUPPORTED, "MAPSM_EXCHANGE_CE needs one slab per process (NCCL context)");
+            if (g->state >= ST_BOUND && ((v != MAPSM_EXCHANGE_COPY) != g->opt_p2p || (v == MAPSM_EXCHANGE_CE) != g->opt_ce))
                 return fail(MAPSM_ESTATE, "set MAPSM_OPT_EXCHANGE before bind");
-            g->opt_p2p = v == MAPSM_EXCHANGE_P2P;
+            g->opt_p2p = v != MAPSM_EXCHANGE_COPY;
+            g->opt_ce = v == MAPSM_EXCHANGE_CE;
             break;
         case MAPSM_OPT_TIMING:
             g->opt_timing = v != 0;

@@ -79,6 +79,8 @@ struct FusedLink {
     unsigned int* sig_up;   // up neighbour's mailbox.recv_bot
     unsigned int* sig_down; // down neighbour's mailbox.recv_top
     int wait_top, wait_bot;
+    int ce = 0;             // copy-engine exchange: the halos arrive by peer memcpy; the mailbox
+                            // counters hold the sender's generation count (wait until >= mine)
 };
 
 // Life (bit-packed: bit j of 32-bit word m of a row = column 32m + j).

@@ -99,6 +99,8 @@ struct HaloLink {
     unsigned int* sig_down;  // &down.mailbox.recv_top
     int wait_top, wait_bot;  // my top / bottom halo is delivered by a neighbour
     int r;                   // rows per delivery
+    int ce;                  // copy-engine exchange (MAPSM_EXCHANGE_CE): recv_top / recv_bot are the
+                             // neighbours' generation counts, copied after their rows; wait for >= gen
 };
 
 struct RowStream {
@@ -345,6 +347,14 @@ inline void tma_set_link(tma::RowStream& p, const FusedLink* l, int r) {
     p.link.wait_top = l ? l->wait_top : 0;
     p.link.wait_bot = l ? l->wait_bot : 0;
     p.link.r = r;
+    p.link.ce = l ? l->ce : 0;
+}
+
+// The producer's wait target for halo rows: rows delivered since bind
+// (peer stores) or the neighbour's generation count (copy engine).
+__device__ __forceinline__ unsigned int halo_wait_target(const tma::HaloLink& L, int64_t nstrips) {
+    const unsigned long long gen = L.mine->gen;
+    return L.ce ? (unsigned int)gen : (unsigned int)(gen * (unsigned long long)(L.r * nstrips));
 }
 
 // Host side: fill the band table of a RowStream for a launch of

@@ -167,3 +167,36 @@ def test_ring_concurrent_deep_halo(ring_ctx, op, r, K):
         out = g.gather()
     exp = oracle.conv(x0, W, n, "wrap") if op == "conv" else oracle.life(x0, n, "wrap")
     assert np.array_equal(out.view(np.uint8), exp.view(np.uint8))
+
+
+@pytest.mark.parametrize("k", [-1, 1, 3])
+@pytest.mark.parametrize("op,r,w,h", [("life", 1, 65536, 300), ("life", 1, 2048, 77), ("conv", 2, 4096, 90),
+                                      ("conv", 4, 1024 + 4, 61), ("conv", 1, 516, 40)])
+@pytest.mark.parametrize("graphs", [True, False])
+def test_ring_copy_engine_exchange(ring_ctx, k, op, r, w, h, graphs):
+    """MAPSM_EXCHANGE_CE: the boundary launch waits on the mailbox for the
+    neighbours' generation counts; the rows move by copy-engine peer copies
+    (here: to the rank itself), followed by the count; interior beside it."""
+    W = mi.weights_f32(8000 + r, r) if op == "conv" else None
+    x0 = mi.field_f32(8010 + w, w, h) if op == "conv" else mi.life_u8(8010 + w, w, h)
+    steps = [7, 16, 2]
+    n = sum(steps)
+    with M.Grid(ring_ctx, w, h, op, r, "wrap", W) as g:
+        if not graphs:
+            g.set_option(M.OPT_GRAPHS, 0)
+        g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_CE)
+        g.set_option(M.OPT_EXCHANGE_SMS, k)
+        g.bind(x0)
+        for s in steps:
+            g.iterate(s)
+        out = g.gather()
+        info = g.info()
+    exp = oracle.conv(x0, W, n, "wrap") if op == "conv" else oracle.life(x0, n, "wrap")
+    assert info.exchanges >= 2 * n and info.launches == 2 * n
+    assert np.array_equal(out.view(np.uint8), exp.view(np.uint8))
+
+
+def test_copy_engine_exchange_needs_nccl_context(local_ctx):
+    with M.Grid(local_ctx(2), 256, 64, "life", 1, "wrap") as g:
+        with pytest.raises(M.MapsmError):
+            g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_CE)
