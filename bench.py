@@ -761,7 +761,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         passes = n // K
         t_pass = (d_ms / steps / 1e3) / max(1, passes)
         if op == "life":
-            droof = roofline_of(env, name, wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
+            droof = roofline_of(env, f"{name}_tb{K}", wl, "life_tb_kernel", slab_cells * K, t_pass, dclocks,
                                 f"one pass = {K} generations ({dl} launches per step)")
         elif dkernel == "conv_tb2_kernel":  # one launch = the two generations of a pass
             droof = roofline_of(env, name + "_tb2", wl, dkernel, slab_cells, t_pass, dclocks,
