@@ -676,7 +676,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
     e2e_value, e2e_how = seq_value, ("mapsm_bind(pinned host) + mapsm_histogram(-> host bins) per step"
                                      if op == "histogram" else
                                      "mapsm_bind(pinned host) + mapsm_iterate(n) + mapsm_read(pinned host) per step")
-    pipe = None
+    pipe = packed_e2e = None
     if op != "histogram" and args.e2e_pipeline > 1 and world == 1:
         # (N = 1 only: with N > 1 every Bind is a collective; several grids'
         # NCCL exchanges on different streams of one communicator are not
@@ -730,6 +730,42 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         e2e_how = (f"{P} grids on their own streams, each step mapsm_bind_async(pinned host input) + "
                    f"mapsm_iterate(n) + mapsm_read_async(pinned host output) on the next grid; {k_steps} steps "
                    "timed end to end (device events, all grid streams joined)")
+        if op == "life" and w % 32 == 0:
+            # The same pipeline with bit-packed host rows (MAPSM_OPT_HOST_PACKED:
+            # the device row format, 1/8 of the u8 bytes over PCIe).
+            import numpy as np
+
+            hp_in = torch.from_numpy(np.packbits(h_in.numpy() != 0, axis=1, bitorder="little")).pin_memory()
+            hp_outs = [torch.empty_like(hp_in, pin_memory=True) for _ in range(P)]
+            for pg in pgrids:
+                pg.set_option(M.OPT_HOST_PACKED, 1)
+                M.mapsm_bind(pg.handle, hp_in)
+                pg.iterate(n)
+                pg.sync()
+            env.barrier()
+            e0.record(env.stream)
+            for gs in gstreams:
+                gs.wait_event(e0)
+            for k in range(k_steps):
+                pg = pgrids[k % P]
+                M.mapsm_bind_async(pg.handle, hp_in)
+                pg.iterate(n)
+                M.mapsm_read_async(pg.handle, hp_outs[k % P])
+            for gs in gstreams:
+                ev = torch.cuda.Event()
+                ev.record(gs)
+                env.stream.wait_event(ev)
+            e1.record(env.stream)
+            e1.synchronize()
+            for pg in pgrids:
+                pg.sync()
+            pk_ms = env.max_over_ranks(e0.elapsed_time(e1))
+            packed_e2e = {"value": units_per_step * k_steps / (pk_ms / 1e3), "ms_per_step": pk_ms / k_steps,
+                          "h2d_bytes_per_step": int(hp_in.numel()), "d2h_bytes_per_step": int(hp_in.numel()),
+                          "how": "as `how`, with MAPSM_OPT_HOST_PACKED: host rows bit-packed (w/32 uint32 "
+                                 "words, bit j of word k = column 32k+j), the device row format"}
+            for pg in pgrids:
+                pg.set_option(M.OPT_HOST_PACKED, 0)
         for pg in pgrids[1:]:
             pg.close()
     elem = 4 if op == "conv" else 1
@@ -851,7 +887,8 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                                                 "ring_stages": int(li.ring_stages)}},
         "e2e": {"value": e2e_value, "unit": unit_name, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "how": e2e_how, "sequential_value": seq_value,
-                "sequential_how": "one step: mapsm_bind + mapsm_iterate + mapsm_read, host waits between steps"},
+                "sequential_how": "one step: mapsm_bind + mapsm_iterate + mapsm_read, host waits between steps",
+                **({"packed_host": packed_e2e} if packed_e2e else {})},
         "gpu_launches": total_launches,
         "roofline": roofline,
         "clocks": clocks,

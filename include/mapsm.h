@@ -488,6 +488,14 @@ mapsm_status mapsm_get_info(mapsm_grid grid, mapsm_grid_info* out);
  *                         MAPSM_EXCHANGE_P2P, k > 0 (explicit only) runs the
  *                         boundary launch with the fused peer stores beside
  *                         the interior instead of one fused launch.
+ *   MAPSM_OPT_HOST_PACKED 1: Life grids (w % 32 == 0, else EUNSUPPORTED): the
+ *                         host rows of mapsm_bind / mapsm_read / mapsm_gather
+ *                         (and their _async forms) are bit-packed — w / 32
+ *                         little-endian uint32 words per row, bit j of word k =
+ *                         column 32k + j, nonzero bit = alive — i.e. the
+ *                         device row format: one 2-D copy each way, 1/8 of
+ *                         the u8 bytes over PCIe, no pack / unpack kernel.
+ *                         Row pitch >= w / 8 bytes.  0 (default): u8 cells.
  *   MAPSM_OPT_DEEP_HALO   K > 1 (1 = off, default): the grid keeps K*r halo
  *                         rows per side and exchanges them once per pass of
  *                         K generations instead of r rows every generation
@@ -518,7 +526,8 @@ typedef enum {
     MAPSM_OPT_EXCHANGE = 6,
     MAPSM_OPT_DEEP_HALO = 7,
     MAPSM_OPT_OWN_STREAM = 8,
-    MAPSM_OPT_EXCHANGE_SMS = 9
+    MAPSM_OPT_EXCHANGE_SMS = 9,
+    MAPSM_OPT_HOST_PACKED = 10
 } mapsm_option;
 
 mapsm_status mapsm_set_option(mapsm_grid grid, mapsm_option opt, int64_t value);

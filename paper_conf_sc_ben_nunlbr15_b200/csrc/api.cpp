@@ -141,7 +141,8 @@ struct mapsm_grid_s {
     int opt_persistent_mode = 1;  // 1: SMEM-resident kernel when the slab fits, 2: grid-barrier kernel only
     bool opt_own_stream = false;  // the grid's slabs use private streams instead of the ctx stream
     bool opt_p2p = false;       // fused compute + peer-memory halo exchange
-    bool opt_ce = false;        // ... with the rows moved by copy-engine peer copies (MAPSM_EXCHANGE_CE)
+    bool opt_ce = false;
+    bool opt_host_packed = false;  // Life: host rows are bit-packed (the device row format)        // ... with the rows moved by copy-engine peer copies (MAPSM_EXCHANGE_CE)
     int opt_exchange_sms = -1;  // SMs the interior launch leaves to the exchange in flight (-1: auto)
     bool conc_open = false;     // concurrent-boundary schedule: the side stream is forked from main
     int tb_k = 1;               // generations per pass (MAPSM_OPT_DEEP_HALO); 1 = per-generation path
@@ -1398,10 +1399,14 @@ static mapsm_status xfer_end(mapsm_grid_s* g, Slab& s, bool h2d) {
     return MAPSM_OK;
 }
 
+// Bytes of one host row: w cells of elem bytes, or (MAPSM_OPT_HOST_PACKED)
+// w / 32 little-endian u32 words of cells, bit j of word k = column 32k + j.
+static int64_t host_row_bytes(const mapsm_grid_s* g) { return g->opt_host_packed ? g->w / 8 : g->w * g->elem; }
+
 static mapsm_status bind_impl(mapsm_grid_s* g, const void* ptr, int64_t pitch, bool async) {
     if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
     if (g->state < ST_OP) return fail(MAPSM_ESTATE, "bind before window_set/op_set");
-    if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch %lld < row bytes", (long long)pitch);
+    if (pitch < host_row_bytes(g)) return fail(MAPSM_EINVAL, "row pitch %lld < row bytes", (long long)pitch);
     DeviceGuard dg;
     int pdev = -1;
     const bool on_dev = is_device_ptr(ptr, &pdev);
@@ -1417,6 +1422,8 @@ static mapsm_status bind_impl(mapsm_grid_s* g, const void* ptr, int64_t pitch, b
         if (!g->packed()) {  // planes of a 3-D slab are rows_per_unit contiguous device rows each
             CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->rpitch, src, pitch, g->w * g->elem, rows * g->rows_per_unit(),
                                  cudaMemcpyDefault, s.main));
+        } else if (g->opt_host_packed) {  // already the device row format: one 2-D copy
+            CK(cudaMemcpy2DAsync(row_ptr(g, s, 0, 0), g->pitch, src, pitch, g->w / 8, rows, cudaMemcpyDefault, s.main));
         } else if (on_dev && pdev == s.device) {
             CK(launch_pack_life(reinterpret_cast<const uint8_t*>(src), pitch, row_ptr(g, s, 0, 0), g->pitch, rows,
                                 g->w, s.main));
@@ -1497,6 +1504,11 @@ static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitc
                              rows * g->rows_per_unit(), cudaMemcpyDefault, s.main));
         return MAPSM_OK;
     }
+    if (g->opt_host_packed) {
+        CK(cudaMemcpy2DAsync(dst, dpitch, row_ptr(g, s, g->cur, 0), g->pitch, g->w / 8, rows, cudaMemcpyDefault,
+                             s.main));
+        return MAPSM_OK;
+    }
     if (dst_on_dev) {
         CK(launch_unpack_life(row_ptr(g, s, g->cur, 0), g->pitch, reinterpret_cast<uint8_t*>(dst), dpitch, rows, g->w,
                               s.main));
@@ -1519,7 +1531,7 @@ static mapsm_status read_slab(mapsm_grid_s* g, Slab& s, char* dst, int64_t dpitc
 static mapsm_status read_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, bool async) {
     if (!g || !ptr) return fail(MAPSM_EINVAL, "NULL argument");
     if (g->state < ST_BOUND) return fail(MAPSM_ESTATE, "read before bind");
-    if (pitch < g->w * g->elem) return fail(MAPSM_EINVAL, "row pitch too small");
+    if (pitch < host_row_bytes(g)) return fail(MAPSM_EINVAL, "row pitch too small");
     DeviceGuard dg;
     int pdev = -1;
     const bool on_dev = is_device_ptr(ptr, &pdev);
@@ -1551,7 +1563,7 @@ static mapsm_status gather_impl(mapsm_grid_s* g, void* ptr, int64_t pitch, int r
         if (!ptr) return fail(MAPSM_EINVAL, "ptr is NULL");
         return read_impl(g, ptr, pitch, async);
     }
-    if (c->rank == root && (!ptr || pitch < g->w * g->elem)) return fail(MAPSM_EINVAL, "root needs ptr and pitch");
+    if (c->rank == root && (!ptr || pitch < host_row_bytes(g))) return fail(MAPSM_EINVAL, "root needs ptr and pitch");
     DeviceGuard dg;
     Slab& s = g->slabs[0];
     CK(cudaSetDevice(s.device));
@@ -1946,6 +1958,11 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
         case MAPSM_OPT_TIMING:
             g->opt_timing = v != 0;
             for (auto& s : g->slabs) s.t_bulk_used = s.t_bnd_used = 0;
+            break;
+        case MAPSM_OPT_HOST_PACKED:
+            if (v != 0 && (!g->packed() || g->w % 32 != 0))
+                return fail(MAPSM_EUNSUPPORTED, "host-packed rows: Life grids with w %% 32 == 0");
+            g->opt_host_packed = v != 0;
             break;
         case MAPSM_OPT_EXCHANGE_SMS:
             if (v < -1 || v > 64) return fail(MAPSM_EINVAL, "exchange SMs %lld (-1..64)", (long long)v);

@@ -163,12 +163,14 @@ __device__ __forceinline__ void warp_gen(const Lane& c, const uint32_t* src, uin
             else if constexpr (kV == 2) *reinterpret_cast<uint2*>(o) = make_uint2(r[0], r[1]);
             else *o = r[0];
             if constexpr (CM == COL_CLAMP) {
-                if ((top_clamp && y == 0) || (bot_clamp && y == R - 1)) {
-                    uint32_t* e = o + (y == 0 ? -nw : nw);
+                // (a one-row slab is both edges: row -1 AND row 1 get the copy)
+                auto put = [&](uint32_t* e) {
                     if constexpr (kV == 4) *reinterpret_cast<uint4*>(e) = make_uint4(r[0], r[1], r[2], r[3]);
                     else if constexpr (kV == 2) *reinterpret_cast<uint2*>(e) = make_uint2(r[0], r[1]);
                     else *e = r[0];
-                }
+                };
+                if (top_clamp && y == 0) put(o - nw);
+                if (bot_clamp && y == R - 1) put(o + nw);
             }
         }
         o += nw;

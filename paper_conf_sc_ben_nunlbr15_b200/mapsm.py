@@ -26,6 +26,7 @@ HALO_EXCHANGE, HALO_WRAP_LOCAL, HALO_CLAMP, HALO_ZERO = 0, 1, 2, 3
 OPT_GRAPHS, OPT_GRAPH_ITERS, OPT_NO_EXCHANGE, OPT_TIMING, OPT_PERSISTENT, OPT_EXCHANGE, OPT_DEEP_HALO = 1, 2, 3, 4, 5, 6, 7
 OPT_OWN_STREAM = 8
 OPT_EXCHANGE_SMS = 9
+OPT_HOST_PACKED = 10
 EXCHANGE_COPY, EXCHANGE_P2P, EXCHANGE_CE = 0, 1, 2
 
 BOUNDARY = {"wrap": WRAP, "clamp": CLAMP, "zero": ZERO, "no_checks": NO_CHECKS}

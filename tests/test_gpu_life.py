@@ -120,7 +120,7 @@ def test_persistent_long_run_many_chunks(ctx):
 
 @pytest.mark.parametrize("b", ["wrap", "clamp", "zero"])
 @pytest.mark.parametrize("shape", [(128, 16), (256, 96), (1024, 333), (4096, 1000), (8192, 1200), (2048, 4096),
-                                   (128, 9)])
+                                   (128, 9), (2048, 1), (128, 1), (4096, 2)])
 @pytest.mark.parametrize("n", [1, 7, 8, 9, 33])
 def test_resident_vs_oracle(ctx, b, shape, n):
     """One cooperative launch, all generations in shared memory, K generations
