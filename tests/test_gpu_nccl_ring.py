@@ -200,3 +200,63 @@ def test_copy_engine_exchange_needs_nccl_context(local_ctx):
     with M.Grid(local_ctx(2), 256, 64, "life", 1, "wrap") as g:
         with pytest.raises(M.MapsmError):
             g.set_option(M.OPT_EXCHANGE, M.EXCHANGE_CE)
+
+
+def test_ring_config2_full_grid_two_generations(ring_ctx):
+    """BASELINE configs[2] (65536^2 WRAP, seed 0x5EED0003) through the NCCL
+    ring in the bench's nccl_ring configuration (default concurrent-boundary
+    schedule, CUDA graphs): generations 1 and 2, every cell."""
+    import torch
+
+    w = h = 65536
+    g0 = np.empty((h, w), np.uint8)
+    mi.life_u8(mi.SEED_LIFE_64K, w, h, out=g0)
+    dev = torch.empty((h, w), dtype=torch.uint8, device="cuda")
+    with M.Grid(ring_ctx, w, h, "life", 1, "wrap") as g:
+        g.bind(g0)
+        g.iterate(1)
+        M.mapsm_read(g.handle, dev)
+        torch.cuda.synchronize()
+        exp = oracle.life(g0, 1, "wrap")
+        del g0
+        assert torch.equal(dev, torch.from_numpy(exp).cuda()), "generation 1"
+        g.iterate(1)
+        M.mapsm_read(g.handle, dev)
+        torch.cuda.synchronize()
+        assert g.info().exchanges >= 4
+    exp = oracle.life(exp, 1, "wrap")
+    assert torch.equal(dev, torch.from_numpy(exp).cuda()), "generation 2"
+
+
+def test_ring_life_slab_deep_halo_full_grid():
+    """One GPU's slab at N = 8 (65536 x 8192) with deep halos K = 8 over the
+    ring, 16 generations in 2 passes (the E(8) prediction's path), every cell."""
+    import torch
+
+    torch.cuda.set_device(0)
+    c = M.mapsm_ctx_create(0, 1, 0, M.mapsm_nccl_unique_id(), None)
+    try:
+        w, h, n = 65536, 8192, 16
+        g0 = mi.life_u8(mi.SEED_LIFE_64K, w, h)
+        with M.Grid(c, w, h, "life", 1, "wrap", deep_halo=8) as g:
+            g.bind(g0)
+            g.iterate(n)
+            out = g.gather()
+            assert g.info().exchanges >= 4
+    finally:
+        M.mapsm_ctx_destroy(c)
+    assert np.array_equal(out, oracle.life(g0, n, "wrap"))
+
+
+@pytest.mark.parametrize("K", [1, 2])
+def test_ring_conv5_full_grid(ring_ctx, K):
+    """The 5x5 16384^2 field (seeds 0x5EED0004 / 0x5EED0044) under WRAP through
+    the ring: per generation (K = 1) and the two-generation kernel (K = 2)."""
+    w = h = 16384
+    f0 = mi.field_f32(mi.SEED_CONV5_FIELD, w, h)
+    W = mi.weights_f32(mi.SEED_CONV5_W, 2)
+    with M.Grid(ring_ctx, w, h, "conv", 2, "wrap", W, deep_halo=K) as g:
+        g.bind(f0)
+        g.iterate(2)
+        got = g.gather()
+    assert np.array_equal(got.view(np.uint32), oracle.conv(f0, W, 2, "wrap").view(np.uint32))
