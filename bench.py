@@ -691,7 +691,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         # end after every grid stream's last read).  The library orders the
         # own-stream grids' host transfers FIFO per direction (xfer_begin).
         P = args.e2e_pipeline
-        k_steps = max(e2e_steps, 4 * P)
+        k_steps = max(e2e_steps, 8 * P)
         pgrids = [grid]
         grid.set_option(M.OPT_OWN_STREAM, 1)
         for _ in range(P - 1):
