@@ -47,6 +47,22 @@
 namespace mapsm {
 namespace conv_detail {
 
+// Weight loads of the two-generation kernel: plain (not volatile) constant
+// loads at uniform addresses, so ptxas keeps the 5x5 pairs in uniform
+// registers across input rows instead of re-issuing an LDCU per tap and row
+// (static LDCU 3746 -> 1171; 934 -> 1008 G cell-updates/s on 16384^2,
+// profiles/r02_conv5_tb2_variants.txt).
+__device__ __forceinline__ unsigned long long ldc_pair_u(unsigned long long a) {
+    unsigned long long r;
+    asm("ld.const.b64 %0, [%1];" : "=l"(r) : "l"(a));
+    return r;
+}
+__device__ __forceinline__ float ldc_one_u(unsigned long long a) {
+    float r;
+    asm("ld.const.f32 %0, [%1];" : "=f"(r) : "l"(a));
+    return r;
+}
+
 constexpr int kTbMargin = 8;  // input stage margin (floats) each side
 
 struct ConvTb2Params {
@@ -150,14 +166,14 @@ __device__ __forceinline__ void taps_ph(Acc2 (&acc)[2 * R + 1][2], const float (
 #pragma unroll
         for (int s = 0; s <= K; ++s) {
             if (s == 0 || s == K) {
-                const float wv = ldc_one(cw + 4 * (d * K + (s == 0 ? 0 : K - 1)));
+                const float wv = ldc_one_u(cw + 4 * (d * K + (s == 0 ? 0 : K - 1)));
 #pragma unroll
                 for (int jp = 0; jp < 2; ++jp) {
                     if (s == 0) vfma_lo(acc[ph][jp], wv, b[2 * jp + s]);
                     else vfma_hi(acc[ph][jp], wv, b[2 * jp + s]);
                 }
             } else {
-                const unsigned long long wq = ldc_pair(cwq + 8 * (d * (K - 1) + s - 1));
+                const unsigned long long wq = ldc_pair_u(cwq + 8 * (d * (K - 1) + s - 1));
 #pragma unroll
                 for (int jp = 0; jp < 2; ++jp) vfma_pair(acc[ph][jp], b[2 * jp + s], wq);
             }
