@@ -62,6 +62,41 @@ __global__ void tma_copy(const char* a, char* b, size_t nrows) {
     asm volatile("cp.async.bulk.wait_group 0;" ::: "memory");
 }
 
+// TMA loads into the ring; 16 consumer warps copy each stage to global memory
+// with 16-byte st.global (the Life interior's store path), 544 threads.
+__global__ void tma_ld_st(const char* a, char* b, size_t nrows) {
+    extern __shared__ __align__(128) char sm[];
+    uint64_t* full = reinterpret_cast<uint64_t*>(sm + NS * ROW);
+    uint64_t* empty = full + NS;
+    const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+    if (threadIdx.x == 0) {
+        for (int i = 0; i < NS; ++i) { mbar_init(&full[i], 1); mbar_init(&empty[i], 16); }
+        asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+    }
+    __syncthreads();
+    size_t r0 = blockIdx.x * nrows / gridDim.x, r1 = (blockIdx.x + 1) * nrows / gridDim.x;
+    if (warp == 16) {
+        if (lane == 0)
+            for (size_t r = r0; r < r1; ++r) {
+                int s = (r - r0) % NS; unsigned ph = ((r - r0) / NS) & 1;
+                if (r - r0 >= NS) mbar_wait(&empty[s], ph ^ 1);
+                mbar_expect(&full[s], ROW);
+                asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];"
+                             ::"r"((unsigned)__cvta_generic_to_shared(sm + s * ROW)), "l"(a + r * ROW), "r"(ROW),
+                               "r"((unsigned)__cvta_generic_to_shared(&full[s])) : "memory");
+            }
+        return;
+    }
+    for (size_t r = r0; r < r1; ++r) {
+        int s = (r - r0) % NS; unsigned ph = ((r - r0) / NS) & 1;
+        mbar_wait(&full[s], ph);
+        const uint4 v = reinterpret_cast<const uint4*>(sm + s * ROW)[warp * 32 + lane];
+        __syncwarp();
+        if (lane == 0) asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"((unsigned)__cvta_generic_to_shared(&empty[s])) : "memory");
+        reinterpret_cast<uint4*>(b + r * ROW)[warp * 32 + lane] = v;
+    }
+}
+
 __global__ void side(int mode, long long ns, unsigned int* flag) {
     long long t0 = clock64();
     const long long cyc = ns * 19 / 10;
@@ -82,6 +117,7 @@ int main(int argc, char** argv) {
     cudaMalloc(&flag, 64); cudaMemset(flag, 0, 64); cudaMemset(a, 1, bytes);
     const int smem = NS * ROW + NS * 8;
     cudaFuncSetAttribute(tma_copy, cudaFuncAttributeMaxDynamicSharedMemorySize, smem);
+    cudaFuncSetAttribute(tma_ld_st, cudaFuncAttributeMaxDynamicSharedMemorySize, smem + NS * 8);
     cudaStream_t m, s;
     cudaStreamCreateWithFlags(&m, cudaStreamNonBlocking);
     cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking);
@@ -97,19 +133,25 @@ int main(int argc, char** argv) {
     cudaEvent_t e0, e1, go;
     cudaEventCreate(&e0); cudaEventCreate(&e1); cudaEventCreateWithFlags(&go, cudaEventDisableTiming);
     const char* names[] = {"none", "spin+threadfence_system", "spin+threadfence(gpu)", "spin+ld.acquire.sys",
-                           "NCCL self send/recv 2x8KB", "spin only"};
-    printf("TMA grid, working set 2 x %zu MiB\n", bytes >> 20);
-    for (int mode = 0; mode <= 5; ++mode) {
+                           "NCCL self send/recv 2x8KB", "spin only", "2-CTA ring kernel, then NCCL",
+                           "2-CTA ring kernel only"};
+    printf("%s grid, working set 2 x %zu MiB\n", getenv("PROBE_LDST") ? "TMA-load / st.global" : "TMA", bytes >> 20);
+    for (int mode = 0; mode <= 7; ++mode) {
         float tot = 0;
         const int reps = 40;
         for (int r = 0; r < reps + 5; ++r) {
             cudaEventRecord(go, m);
             cudaStreamWaitEvent(s, go, 0);
             cudaEventRecord(e0, m);
-            tma_copy<<<146, 32, smem, m>>>(a, b, bytes / ROW);
+            if (getenv("PROBE_LDST"))
+                tma_ld_st<<<146, 544, smem + NS * 8, m>>>(a, b, bytes / ROW);
+            else
+                tma_copy<<<146, 32, smem, m>>>(a, b, bytes / ROW);
             if (mode >= 1 && mode <= 3) side<<<1, 128, 0, s>>>(mode, 10000, flag);
             if (mode == 5) side<<<1, 128, 0, s>>>(0, 10000, flag);
-            if (mode == 4) {
+            if (mode == 7) tma_ld_st<<<2, 544, smem + NS * 8, s>>>(a, s1, 2);
+            if (mode == 4 || mode == 6) {
+                if (mode == 6) tma_ld_st<<<2, 544, smem + NS * 8, s>>>(a, s1, 2);  // a 2-row "boundary" launch first
                 ncclGroupStart();
                 ncclSend(s0, 8192, ncclUint8, 0, comm, s); ncclSend(s0 + 8192, 8192, ncclUint8, 0, comm, s);
                 ncclRecv(s1, 8192, ncclUint8, 0, comm, s); ncclRecv(s1 + 8192, 8192, ncclUint8, 0, comm, s);
