@@ -68,7 +68,7 @@ int main(int argc, char** argv) {
     ncclComm_t comm;
     int dev0 = 0;
     ncclCommInitAll(&comm, 1, &dev0);
-    printf("working set 2 x %zu MiB\n", bytes >> 20);
+    printf("working set 2 x %zu MiB%s\n", bytes >> 20, getenv("PROBE_PINGPONG") ? " (ping-pong)" : "");
     for (int mode = 0; mode <= 10; ++mode) {
         float tot = 0;
         const int reps = 40;
@@ -76,7 +76,10 @@ int main(int argc, char** argv) {
             cudaEventRecord(go, m);
             cudaStreamWaitEvent(s, go, 0);
             cudaEventRecord(e0, m);
-            copy_grid<<<146, 1024, 0, m>>>(a, b, n);
+            if (getenv("PROBE_PINGPONG") && (r & 1))
+                copy_grid<<<146, 1024, 0, m>>>(b, a, n);  // ping-pong: read what the last launch wrote
+            else
+                copy_grid<<<146, 1024, 0, m>>>(a, b, n);
             if (mode >= 1 && mode <= 7) side<<<1, 128, 0, s>>>(mode, 10000, flag, scratch);
             if (mode == 9) {
                 ncclGroupStart();
