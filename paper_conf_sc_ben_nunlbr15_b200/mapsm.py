@@ -238,6 +238,9 @@ def mapsm_nccl_unique_id() -> bytes:
 
 def mapsm_ctx_create(rank: int, world: int, device: int, nccl_unique_id: bytes | None = None,
                      cuda_stream: int | None = None) -> int:
+    """One rank of `world` (include/mapsm.h).  world > 1 needs the rank-0
+    mapsm_nccl_unique_id(); world == 1 with an id = the one-rank NCCL ring
+    (WRAP halos through ncclSend/ncclRecv to the rank itself)."""
     out = ctypes.c_void_p()
     uid = ctypes.create_string_buffer(nccl_unique_id, 128) if nccl_unique_id is not None else None
     _check(lib().mapsm_ctx_create(rank, world, device, uid, cuda_stream, ctypes.byref(out)), "mapsm_ctx_create")
