@@ -10,7 +10,10 @@
 #include <cstdint>
 #include <cstdlib>
 
-constexpr int NS = 16, ROW = 8192;  // stages x bytes
+#ifndef PROBE_NS
+#define PROBE_NS 16
+#endif
+constexpr int NS = PROBE_NS, ROW = 8192;  // stages x bytes
 
 __device__ __forceinline__ void mbar_init(uint64_t* b, int n) {
     asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"((unsigned)__cvta_generic_to_shared(b)), "r"(n));
