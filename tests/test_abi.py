@@ -67,3 +67,27 @@ def test_no_cpu_fallback_symbols():
     out = subprocess.check_output(["cuobjdump", "--list-text", M._LIB_PATH]).decode()
     assert "life_step_kernel" in out and "conv_step_kernel" in out
     assert "pack_life_kernel" in out and "unpack_life_kernel" in out
+
+
+def test_binding_constants_match_header_enums():
+    """Every MAPSM_* enumerator of include/mapsm.h that the binding mirrors
+    (same name without the prefix) has the same value in mapsm.py."""
+    import re
+
+    from paper_conf_sc_ben_nunlbr15_b200 import mapsm as M
+
+    text = open(os.path.join(ROOT, "include", "mapsm.h")).read()
+    body = " ".join(re.findall(r"typedef enum\s*\{(.*?)\}", text, re.S))
+    enums = {k: int(v) for k, v in re.findall(r"MAPSM_([A-Z0-9_]+)\s*=\s*(-?\d+)", body)}
+    assert len(enums) > 40
+    aliases = {"LIFE_REG": "KERNEL_LIFE_REG"}
+    checked = 0
+    for name, value in enums.items():
+        py = name if hasattr(M, name) else aliases.get(name)
+        if py is None or not hasattr(M, py):
+            continue
+        assert getattr(M, py) == value, (name, getattr(M, py), value)
+        checked += 1
+    for must in ("OPT_EXCHANGE_SMS", "OPT_HOST_PACKED", "EXCHANGE_CE", "KERNEL_CONV_TB2", "OPT_DEEP_HALO"):
+        assert must in enums and getattr(M, must) == enums[must], must
+    assert checked >= 25, checked
