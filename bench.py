@@ -815,57 +815,61 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
 
     ring = None
     if extras and world == 1 and op != "histogram" and wl["b"] == "wrap" and not d:
-        # The NCCL data plane on one GPU (include/mapsm.h, one-rank NCCL
-        # context): the WRAP row ring closes through ncclSend/ncclRecv to
-        # itself every generation — boundary rows first, the exchange group on
-        # the side stream, interior overlapped, all inside the CUDA graphs — so
-        # the multi-process path runs on hardware; exposure = the same steps
-        # with the exchange switched off.
-        rctx = M.mapsm_ctx_create(0, 1, env.local_rank, M.mapsm_nccl_unique_id(), env.stream.cuda_stream)
-        try:
-            rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W)
-            rg.bind(h_in)
-            for _ in range(warmup):
-                rg.iterate(n)
-            x0, l0 = rg.info().exchanges, rg.info().launches
-            r_ms, rt0, rt1 = env.timed(lambda: rg.iterate(n), steps)
-            rclocks = env.sampler.region(rt0, rt1)
-            rinfo = rg.info()
-            rg.set_option(M.OPT_EXCHANGE_SMS, 0)
-            rg.iterate(n)
-            ser_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
-            rg.set_option(M.OPT_EXCHANGE_SMS, -1)
-            rg.set_option(M.OPT_NO_EXCHANGE, 1)
-            rg.iterate(n)
-            ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
-            rg.close()
-            dring = None
-            if op == "life" and args.deep_halo > 1:  # deep halos over the same ring: one exchange per K generations
-                rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W, deep_halo=args.deep_halo)
+        try:  # (an NCCL failure here must not cost the bench line)
+            # The NCCL data plane on one GPU (include/mapsm.h, one-rank NCCL
+            # context): the WRAP row ring closes through ncclSend/ncclRecv to
+            # itself every generation — boundary rows first, the exchange group on
+            # the side stream, interior overlapped, all inside the CUDA graphs — so
+            # the multi-process path runs on hardware; exposure = the same steps
+            # with the exchange switched off.
+            rctx = M.mapsm_ctx_create(0, 1, env.local_rank, M.mapsm_nccl_unique_id(), env.stream.cuda_stream)
+            try:
+                rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W)
                 rg.bind(h_in)
+                for _ in range(warmup):
+                    rg.iterate(n)
+                x0, l0 = rg.info().exchanges, rg.info().launches
+                r_ms, rt0, rt1 = env.timed(lambda: rg.iterate(n), steps)
+                rclocks = env.sampler.region(rt0, rt1)
+                rinfo = rg.info()
+                rg.set_option(M.OPT_EXCHANGE_SMS, 0)
                 rg.iterate(n)
-                dr_ms, _, _ = env.timed(lambda: rg.iterate(n), 3)
-                dring = {"generations_per_pass": args.deep_halo, "ms_per_step": dr_ms / 3,
-                         "value": units_per_step * 3 / (dr_ms / 1e3)}
+                ser_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
+                rg.set_option(M.OPT_EXCHANGE_SMS, -1)
+                rg.set_option(M.OPT_NO_EXCHANGE, 1)
+                rg.iterate(n)
+                ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
                 rg.close()
-        finally:
-            M.mapsm_ctx_destroy(rctx)
-        r_step = r_ms / steps
-        ring = {"how": "one-rank NCCL communicator (mapsm_ctx_create with world 1 and an id): per generation the "
-                       "boundary rows and one NCCL group (send-up, send-down, recv-bottom, recv-top to rank 0) on "
-                       "the side stream on a few SMs, the interior on the others (concurrent-boundary schedule, "
-                       "MAPSM_OPT_EXCHANGE_SMS default); CUDA graphs",
-                "serial_ms_per_step": ser_ms / 2,
-                "value": units_per_step * steps / (r_ms / 1e3), "unit": metric_of(wl)[1], "ms_per_step": r_step,
-                "vs_plain_path": (units_per_step * steps / (r_ms / 1e3)) / value,
-                "launches_per_step": (rinfo.launches - l0) // steps,
-                "halo_messages_per_step": (rinfo.exchanges - x0) // steps,
-                "halo_bytes_per_message": wl["r"] * int(info0.pitch_bytes),
-                "halo_exposure": {"ms_per_step_no_exchange": ne_ms / 2,
-                                  "exposed_pct": 100.0 * (r_step - ne_ms / 2) / r_step},
-                "clocks": rclocks}
-        if dring is not None:
-            ring["deep_halo"] = dring
+                dring = None
+                if op == "life" and args.deep_halo > 1:  # deep halos over the same ring: one exchange per K generations
+                    rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W, deep_halo=args.deep_halo)
+                    rg.bind(h_in)
+                    rg.iterate(n)
+                    dr_ms, _, _ = env.timed(lambda: rg.iterate(n), 3)
+                    dring = {"generations_per_pass": args.deep_halo, "ms_per_step": dr_ms / 3,
+                             "value": units_per_step * 3 / (dr_ms / 1e3)}
+                    rg.close()
+            finally:
+                M.mapsm_ctx_destroy(rctx)
+            r_step = r_ms / steps
+            ring = {"how": "one-rank NCCL communicator (mapsm_ctx_create with world 1 and an id): per generation the "
+                           "boundary rows and one NCCL group (send-up, send-down, recv-bottom, recv-top to rank 0) on "
+                           "the side stream on a few SMs, the interior on the others (concurrent-boundary schedule, "
+                           "MAPSM_OPT_EXCHANGE_SMS default); CUDA graphs",
+                    "serial_ms_per_step": ser_ms / 2,
+                    "value": units_per_step * steps / (r_ms / 1e3), "unit": metric_of(wl)[1], "ms_per_step": r_step,
+                    "vs_plain_path": (units_per_step * steps / (r_ms / 1e3)) / value,
+                    "launches_per_step": (rinfo.launches - l0) // steps,
+                    "halo_messages_per_step": (rinfo.exchanges - x0) // steps,
+                    "halo_bytes_per_message": wl["r"] * int(info0.pitch_bytes),
+                    "halo_exposure": {"ms_per_step_no_exchange": ne_ms / 2,
+                                      "exposed_pct": 100.0 * (r_step - ne_ms / 2) / r_step},
+                    "clocks": rclocks}
+            if dring is not None:
+                ring["deep_halo"] = dring
+
+        except Exception as e:  # noqa: BLE001
+            ring = {"error": f"{type(e).__name__}: {e}"[:300]}
 
     metric, unit_name = metric_of(wl)
     nbuf = 1 if op == "histogram" else 2
