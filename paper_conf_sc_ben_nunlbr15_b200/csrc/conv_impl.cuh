@@ -406,7 +406,11 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
     static_assert(EPL % 2 == 0, "pairs of outputs");
     float acc[PAIR ? 1 : K][EPL];
     Acc2 acc2[PAIR ? K : 1][EPL / 2];
-    while (tma::seg_next<NC, EPL>(p, it, sg)) {
+    // Per segment: the linked body (boundary rows also stored into the
+    // neighbours' halos, then signalled) only for segments with boundary
+    // rows; interior segments of a fused launch run the plain body.
+    auto seg_body = [&](auto link_tag) {
+        constexpr bool LINK = decltype(link_tag)::value;
         tma::consume_align<NS>(full, empty, ring, lane);
         uint32_t ph = ring.phase;  // segment starts at stage 0
         const int n_out = (int)(sg.ye - sg.ys);
@@ -523,7 +527,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                         else
                             ov = make_float2(res[0], res[1]);
                         *reinterpret_cast<OT*>(out0 + (int64_t)o * p.pitch) = ov;
-                        if constexpr (FUSED) {  // boundary rows also go to the neighbours' halos
+                        if constexpr (LINK) {  // boundary rows also go to the neighbours' halos
                             const int64_t yo = sg.ys + o;
                             if (Lk.dst_up && yo < R)
                                 *reinterpret_cast<OT*>(reinterpret_cast<float*>(Lk.dst_up) + yo * p.pitch + sg.e0 +
@@ -571,7 +575,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         ring.stage = n_in % NS;
         ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
         ring.count += n_in;
-        if constexpr (FUSED) {
+        if constexpr (LINK) {
             if (Lk.dst_up && sg.ys < R) {
                 const int64_t e = sg.ye < R ? sg.ye : R;
                 tma::publish_delivery(Lk.sig_up, (unsigned int)(e - sg.ys), NC);
@@ -581,6 +585,15 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                 tma::publish_delivery(Lk.sig_down, (unsigned int)(sg.ye - b0), NC);
             }
         }
+    };
+    while (tma::seg_next<NC, EPL>(p, it, sg)) {
+        if constexpr (FUSED) {
+            if (sg.ys < R || sg.ye > p.rows - R) {
+                seg_body(std::true_type{});
+                continue;
+            }
+        }
+        seg_body(std::false_type{});
     }
     }
     if constexpr (FUSED) tma::finish_launch_consumers(Lk.mine, (NC + 1) * 32);

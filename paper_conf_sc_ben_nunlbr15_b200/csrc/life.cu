@@ -24,6 +24,8 @@
 #include <cuda_runtime.h>
 #include <stdint.h>
 
+#include <type_traits>
+
 #include "kernels.h"
 #include "tma_rows.cuh"
 
@@ -370,7 +372,13 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
         static_assert(NS % 3 == 0, "NS must be a multiple of 3");
         const int t = warp * 32 + lane;  // vector index within the strip
         uint32_t r0[3][4], r1[3][4], xs[3][4];  // row sums and raw words of 3 rows
-        while (tma::seg_next<NC>(p, it, sg)) {
+        // Per segment: the linked body (stores into the neighbours' halos and
+        // signals them) only for segments that contain boundary rows; the
+        // interior segments of a fused launch run the plain body, so they
+        // cost what the unfused kernel costs (measured: one body for all
+        // segments made the fused 65536^2 generation 212 us instead of 165).
+        auto seg_body = [&](auto link_tag) {
+            constexpr bool LINK = decltype(link_tag)::value;
             tma::consume_align<NS>(full, empty, ring, lane);
             uint32_t ph = ring.phase;  // segment starts at stage 0
             const int n_in = (int)(sg.ye - sg.ys + 2);  // input rows ys-1 .. ye
@@ -418,7 +426,7 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
                 if (active) {
                     const uint4 ov = make_uint4(o[0], o[1], o[2], o[3]);
                     *reinterpret_cast<uint4*>(out_row) = ov;
-                    if constexpr (FUSED) {  // boundary rows also go to the neighbours' halos
+                    if constexpr (LINK) {  // boundary rows also go to the neighbours' halos
                         if (L.dst_up && yo < L.r)
                             *reinterpret_cast<uint4*>(L.dst_up + yo * p.pitch + sg.e0 + t * 4) = ov;
                         if (L.dst_down && yo >= p.rows - L.r)
@@ -460,7 +468,7 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
             ring.stage = n_in % NS;
             ring.phase = ph0 ^ (uint32_t)((n_in / NS) & 1);
             ring.count += n_in;
-            if constexpr (FUSED) {
+            if constexpr (LINK) {
                 if (L.dst_up && sg.ys < L.r) {
                     const int64_t e = sg.ye < L.r ? sg.ye : L.r;
                     tma::publish_delivery(L.sig_up, (unsigned int)(e - sg.ys), NC);
@@ -470,6 +478,15 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
                     tma::publish_delivery(L.sig_down, (unsigned int)(sg.ye - b0), NC);
                 }
             }
+        };
+        while (tma::seg_next<NC>(p, it, sg)) {
+            if constexpr (FUSED) {
+                if (sg.ys < L.r || sg.ye > p.rows - L.r) {
+                    seg_body(std::true_type{});
+                    continue;
+                }
+            }
+            seg_body(std::false_type{});
         }
     }
     if constexpr (FUSED) tma::finish_launch_consumers(L.mine, (NC + 1) * 32);
