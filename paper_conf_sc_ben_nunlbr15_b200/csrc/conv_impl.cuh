@@ -390,8 +390,10 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
     if (warp == NC) {
         constexpr int PL = R <= 2 ? 2 : MAPSM_CONV_BIG_PL;  // producer lanes (see tma_rows.cuh)
         if (lane < PL) {
-            const unsigned int halo_target = FUSED ? halo_wait_target(Lk, p.nstrips) : 0u;
             while (tma::seg_next<NC, EPL>(p, it, sg)) {
+                // (the mailbox is read only by segments that load halo rows)
+                const unsigned int halo_target =
+                    FUSED && (sg.ys < R || sg.ye + R > p.rows) ? halo_wait_target(Lk, p.nstrips) : 0u;
                 tma::produce_align<NS, PL>(full, empty, ring, lane);
                 tma::produce<NC, NS, CM == COL_WRAP, EPL, PL>(p, sg, smem, full, empty, sg.ys - R, sg.ye - sg.ys + 2 * R,
                                                          ring, halo_target, lane);

@@ -353,8 +353,10 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
 
     if (warp == NC) {
         if (lane == 0) {
-            const unsigned int halo_target = FUSED ? halo_wait_target(L, p.nstrips) : 0u;
             while (tma::seg_next<NC>(p, it, sg)) {
+                // (the mailbox is read only by segments that load halo rows)
+                const unsigned int halo_target =
+                    FUSED && (sg.ys < 1 || sg.ye + 1 > p.rows) ? halo_wait_target(L, p.nstrips) : 0u;
                 tma::produce_align<NS, 1>(full, empty, ring, lane);
                 tma::produce<NC, NS, CM == COL_WRAP, 4, 1>(p, sg, smem, full, empty, sg.ys - 1, sg.ye - sg.ys + 2, ring,
                                                      halo_target, lane);
