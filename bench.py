@@ -840,6 +840,14 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                 rg.iterate(n)
                 ne_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
                 rg.close()
+                # the fused peer-store kernel over the same ring (MAPSM_EXCHANGE_P2P:
+                # boundary CTAs store their rows into the halos and signal the mailbox)
+                rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W)
+                rg.set_option(M.OPT_EXCHANGE, M.EXCHANGE_P2P)
+                rg.bind(h_in)
+                rg.iterate(n)
+                fp_ms, _, _ = env.timed(lambda: rg.iterate(n), 2)
+                rg.close()
                 dring = None
                 if op == "life" and args.deep_halo > 1:  # deep halos over the same ring: one exchange per K generations
                     rg = M.Grid(rctx, w, h, op, wl["r"], wl["b"], W, deep_halo=args.deep_halo)
@@ -857,6 +865,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                            "the side stream on a few SMs, the interior on the others (concurrent-boundary schedule, "
                            "MAPSM_OPT_EXCHANGE_SMS default); CUDA graphs",
                     "serial_ms_per_step": ser_ms / 2,
+                    "fused_p2p_ms_per_step": fp_ms / 2,
                     "value": units_per_step * steps / (r_ms / 1e3), "unit": metric_of(wl)[1], "ms_per_step": r_step,
                     "vs_plain_path": (units_per_step * steps / (r_ms / 1e3)) / value,
                     "launches_per_step": (rinfo.launches - l0) // steps,
