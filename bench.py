@@ -580,6 +580,9 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
     else:
         W = None
     grid = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, d=d)
+    if args.exchange != "nccl" and world > 1 and op != "histogram":
+        # (multi-process only: at N = 1 nothing is exchanged; the ring sub-line covers the modes)
+        grid.set_option(M.OPT_EXCHANGE, {"p2p": M.EXCHANGE_P2P, "ce": M.EXCHANGE_CE}[args.exchange])
     cpu_ = w * (h if d else 1)             # cells per partition unit (row or plane)
     cells_total = w * h * (d if d else 1)
     if args.graph_iters:
@@ -886,7 +889,10 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
     dtype = {"life": "u32 bit-sliced (1 bit/cell)", "conv": "f32", "histogram": "u8 in, u32/u64 counts"}[op]
     para = f"row-slab x{world}"
     if world > 1:
-        para += " + NCCL allreduce of bins" if op == "histogram" else " + NCCL halo exchange"
+        para += (" + NCCL allreduce of bins" if op == "histogram" else
+                 {"nccl": " + NCCL halo exchange (concurrent-boundary schedule)",
+                  "p2p": " + fused peer-store halo exchange (CUDA IPC)",
+                  "ce": " + copy-engine peer-copy halo exchange"}[args.exchange])
     line = {
         "metric": metric, "value": value, "unit": unit_name, "n_gpus": world, "steps": steps,
         "warmup": warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -933,6 +939,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="headline only (no BASELINE sub-configurations)")
     ap.add_argument("--graph-iters", type=int, default=0)
+    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p", "ce"],
+                    help="N > 1: halo exchange of the measured grids (nccl = NCCL send/recv with the "
+                         "concurrent-boundary schedule, the default; p2p = fused peer stores over CUDA IPC; "
+                         "ce = copy-engine peer copies)")
     ap.add_argument("--deep-halo", type=int, default=8,
                     help="Life 65536^2: also measure the deep-halo path with K generations per pass "
                          "(reported under 'deep_halo'; 0/1 = skip)")
