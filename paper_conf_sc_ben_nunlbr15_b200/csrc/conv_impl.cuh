@@ -399,7 +399,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
                                                          ring, halo_target, lane);
             }
         }
-        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32);
+        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32, p.link_ctas);
         return;
     }
     {
@@ -598,7 +598,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
         seg_body(std::false_type{});
     }
     }
-    if constexpr (FUSED) tma::finish_launch_consumers(Lk.mine, (NC + 1) * 32);
+    if constexpr (FUSED) tma::finish_launch_consumers(Lk.mine, (NC + 1) * 32, p.link_ctas);
 }
 
 template <int R, int NC, int NS, int CM, int EPL>

@@ -362,7 +362,7 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
                                                      halo_target, lane);
             }
         }
-        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32);
+        if constexpr (FUSED) tma::finish_launch_producer((NC + 1) * 32, p.link_ctas);
         return;
     }
     {
@@ -491,7 +491,7 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
             seg_body(std::false_type{});
         }
     }
-    if constexpr (FUSED) tma::finish_launch_consumers(L.mine, (NC + 1) * 32);
+    if constexpr (FUSED) tma::finish_launch_consumers(L.mine, (NC + 1) * 32, p.link_ctas);
 }
 
 template <int NC, int NS, int CM>

@@ -113,6 +113,7 @@ struct RowStream {
     int nbands;
     int64_t begin[kMaxBands], end[kMaxBands];  // output-row bands of this launch
     int cta_begin[kMaxBands + 1];              // CTAs [cta_begin[b], cta_begin[b+1]) work on band b
+    int link_ctas;                             // fused launches: CTAs [0, link_ctas) count the launch (gen)
     int top_map, bot_map;
     HaloLink link;
 };
@@ -195,19 +196,23 @@ __device__ __forceinline__ void publish_delivery(unsigned int* counter, unsigned
     }
 }
 
-// At exit the last CTA of the launch advances gen.  The producer warp only
-// arrives (named barrier 2) and leaves, so the consumer code stays free of
-// CTA-wide divergence; the consumers wait on barrier 2, then thread 0 counts.
-__device__ __forceinline__ void finish_launch_producer(int threads) {
+// At exit the last of the launch's boundary-band CTAs (CTAs [0, n_link):
+// the ones that read gen, at their start) advances gen; interior CTAs of a
+// fused launch leave without counting.  The producer warp only arrives
+// (named barrier 2) and leaves, so the consumer code stays free of CTA-wide
+// divergence; the consumers wait on barrier 2, then thread 0 counts.
+__device__ __forceinline__ void finish_launch_producer(int threads, int n_link) {
+    if ((int)blockIdx.x >= n_link) return;
     __syncwarp();
     asm volatile("bar.arrive 2, %0;" ::"r"(threads) : "memory");
 }
 
-__device__ __forceinline__ void finish_launch_consumers(Mailbox* mb, int threads) {
+__device__ __forceinline__ void finish_launch_consumers(Mailbox* mb, int threads, int n_link) {
+    if ((int)blockIdx.x >= n_link) return;
     asm volatile("bar.sync 2, %0;" ::"r"(threads) : "memory");
     if (threadIdx.x == 0) {
         __threadfence();
-        if (atomicAdd(&mb->done, 1u) == gridDim.x - 1) {
+        if (atomicAdd(&mb->done, 1u) == (unsigned)n_link - 1) {
             mb->done = 0;
             __threadfence();
             atomicAdd(&mb->gen, 1ull);
@@ -401,6 +406,9 @@ inline int64_t tma_plan_grid(tma::RowStream& p, const RowBands& b, int num_sms, 
         p.cta_begin[i + 1] = (int)total;
     }
     for (int i = b.nbands; i < tma::kMaxBands; ++i) p.cta_begin[i + 1] = (int)total;
+    // who counts a fused launch: the boundary bands' CTAs (all of them when
+    // the launch has no interior band)
+    p.link_ctas = boundary_first && b.nbands > 1 ? p.cta_begin[b.nbands - 1] : (int)total;
     return total;
 }
 
