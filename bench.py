@@ -579,20 +579,45 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         W = mi.weights3d_f32(wl["wseed"], wl["r"]) if d else mi.weights_f32(wl["wseed"], wl["r"])
     else:
         W = None
-    grid = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, d=d)
-    if args.exchange != "nccl" and world > 1 and op != "histogram":
-        # (multi-process only: at N = 1 nothing is exchanged; the ring sub-line covers the modes)
-        grid.set_option(M.OPT_EXCHANGE, {"p2p": M.EXCHANGE_P2P, "ce": M.EXCHANGE_CE}[args.exchange])
+    # Halo exchange of the multi-process run (at N = 1 nothing is exchanged;
+    # the nccl_ring sub-line covers the modes on one GPU): "auto" = the fused
+    # peer-store kernel (MAPSM_EXCHANGE_P2P, CUDA IPC over NVLink; the fastest
+    # exchange on the ring at the N = 8 slab sizes) where the
+    # grid allows it, else — or if the collective IPC linking fails on any
+    # rank — NCCL send/recv with the concurrent-boundary schedule.
+    xmode = args.exchange
+    if xmode == "auto":
+        xmode = "p2p" if (world > 1 and op in ("life", "conv") and not d and wl["r"] <= 4) else "nccl"
+    if world == 1 or op == "histogram":
+        xmode = "nccl"
+
+    def make_grid(mode):
+        gr = M.Grid(env.ctx, w, h, op, wl["r"], wl["b"], W, d=d)
+        if mode != "nccl":
+            gr.set_option(M.OPT_EXCHANGE, {"p2p": M.EXCHANGE_P2P, "ce": M.EXCHANGE_CE}[mode])
+        if args.graph_iters:
+            gr.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
+        return gr
+
+    grid = make_grid(xmode)
     cpu_ = w * (h if d else 1)             # cells per partition unit (row or plane)
     cells_total = w * h * (d if d else 1)
-    if args.graph_iters:
-        grid.set_option(M.OPT_GRAPH_ITERS, args.graph_iters)
     y0, rows = grid.local_rows()
     h_in = host_input(env, {**wl, "h": h}, rows, y0)
     h_out = torch.empty_like(h_in, pin_memory=True) if op != "histogram" else None
     d_bins = torch.zeros(256, dtype=torch.int64, device=env.dev)
     h_bins = torch.zeros(256, dtype=torch.int64, pin_memory=True)
-    grid.bind(h_in)
+    x_fallback = None
+    try:
+        grid.bind(h_in)
+    except M.MapsmError as e:  # (the same error on every rank: the linking agrees collectively)
+        if xmode == "nccl" or args.exchange != "auto":
+            raise
+        x_fallback = str(e)[:200]
+        grid.close()
+        xmode = "nccl"
+        grid = make_grid(xmode)
+        grid.bind(h_in)
     info0 = grid.info()
 
     def step():
@@ -892,7 +917,7 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
         para += (" + NCCL allreduce of bins" if op == "histogram" else
                  {"nccl": " + NCCL halo exchange (concurrent-boundary schedule)",
                   "p2p": " + fused peer-store halo exchange (CUDA IPC)",
-                  "ce": " + copy-engine peer-copy halo exchange"}[args.exchange])
+                  "ce": " + copy-engine peer-copy halo exchange"}[xmode])
     line = {
         "metric": metric, "value": value, "unit": unit_name, "n_gpus": world, "steps": steps,
         "warmup": warmup, "ms_per_step": ms_per_step, "higher_is_better": True,
@@ -903,7 +928,9 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
                          f"{ws_mib:.0f} MiB vs 126 MB L2", "cuda_graphs": used_graphs,
                    "kernel": kernel, "launch": {"ctas": int(li.ctas), "threads": int(li.threads),
                                                 "smem_bytes": int(li.smem_bytes),
-                                                "ring_stages": int(li.ring_stages)}},
+                                                "ring_stages": int(li.ring_stages)},
+                   **({"exchange": xmode} if world > 1 else {}),
+                   **({"exchange_fallback": x_fallback} if x_fallback else {})},
         "e2e": {"value": e2e_value, "unit": unit_name, "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
                 "how": e2e_how, "sequential_value": seq_value,
                 "sequential_how": "one step: mapsm_bind + mapsm_iterate + mapsm_read, host waits between steps",
@@ -939,9 +966,10 @@ def main():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-configs", action="store_true", help="headline only (no BASELINE sub-configurations)")
     ap.add_argument("--graph-iters", type=int, default=0)
-    ap.add_argument("--exchange", default="nccl", choices=["nccl", "p2p", "ce"],
-                    help="N > 1: halo exchange of the measured grids (nccl = NCCL send/recv with the "
-                         "concurrent-boundary schedule, the default; p2p = fused peer stores over CUDA IPC; "
+    ap.add_argument("--exchange", default="auto", choices=["auto", "nccl", "p2p", "ce"],
+                    help="N > 1: halo exchange of the measured grids (auto = p2p where the grid allows it, "
+                         "falling back to nccl if the CUDA-IPC linking fails; nccl = NCCL send/recv with the "
+                         "concurrent-boundary schedule; p2p = fused peer stores over CUDA IPC; "
                          "ce = copy-engine peer copies)")
     ap.add_argument("--deep-halo", type=int, default=8,
                     help="Life 65536^2: also measure the deep-halo path with K generations per pass "

@@ -896,51 +896,77 @@ static mapsm_status p2p_link(mapsm_grid_s* g) {
         g->p2p_linked = true;
         return MAPSM_OK;
     }
+    // Across processes: every step that can fail locally is followed by the
+    // same collectives on every rank (the handle all-gather, then an
+    // all-reduce of the outcome), so a failure on one rank (no IPC, no peer
+    // access) surfaces as the same error on all of them — never as a rank
+    // waiting in a collective the failed one skipped — and the caller can
+    // fall back to the NCCL exchange (bench.py does).
     Slab& s = g->slabs[0];
     CK(cudaSetDevice(s.device));
     const int W = c->world;
     const size_t hb = 3 * sizeof(cudaIpcMemHandle_t);
-    std::vector<char> mine(hb), all(hb * W);
-    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()), s.base[0]));
-    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()) + 1, s.base[1]));
-    CK(cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()) + 2, s.mailbox));
-    char* dev = nullptr;
-    CK(cudaMalloc(&dev, hb * (W + 1)));
-    CK(cudaMemcpyAsync(dev, mine.data(), hb, cudaMemcpyHostToDevice, s.main));
-    ncclResult_t nr = g_nccl.allGather(dev, dev + hb, hb, ncclUint8, c->comm, s.main);
-    cudaError_t ce = cudaMemcpyAsync(all.data(), dev + hb, hb * W, cudaMemcpyDeviceToHost, s.main);
+    std::vector<char> mine(hb, 0), all(hb * W);
+    cudaError_t le = cudaSuccess;  // first local failure
+    void* mem[3] = {s.base[0], s.base[1], s.mailbox};
+    for (int k = 0; k < 3 && le == cudaSuccess; ++k)
+        le = cudaIpcGetMemHandle(reinterpret_cast<cudaIpcMemHandle_t*>(mine.data()) + k, mem[k]);
+    if (le != cudaSuccess) cudaGetLastError();
+    int* dev = nullptr;
+    CK(cudaMalloc(&dev, hb * (W + 1) + 2 * sizeof(int)));
+    char* hbuf = reinterpret_cast<char*>(dev) + 2 * sizeof(int);
+    CK(cudaMemcpyAsync(hbuf, mine.data(), hb, cudaMemcpyHostToDevice, s.main));
+    ncclResult_t nr = g_nccl.allGather(hbuf, hbuf + hb, hb, ncclUint8, c->comm, s.main);
+    cudaError_t ce = cudaMemcpyAsync(all.data(), hbuf + hb, hb * W, cudaMemcpyDeviceToHost, s.main);
     cudaError_t se = cudaStreamSynchronize(s.main);
-    cudaFree(dev);
-    if (nr != ncclSuccess) return fail(MAPSM_ENCCL, "IPC handle all-gather: %s", g_nccl.errStr(nr));
-    if (ce != cudaSuccess || se != cudaSuccess) return fail(MAPSM_ECUDA, "IPC handle all-gather copy failed");
-    auto open = [&](int rank, int k, void** out) -> mapsm_status {
+    if (nr != ncclSuccess || ce != cudaSuccess || se != cudaSuccess) {
+        cudaFree(dev);
+        if (nr != ncclSuccess) return fail(MAPSM_ENCCL, "IPC handle all-gather: %s", g_nccl.errStr(nr));
+        return fail(MAPSM_ECUDA, "IPC handle all-gather copy failed");
+    }
+    auto open = [&](int rank, int k, void** out) -> cudaError_t {
         cudaIpcMemHandle_t h;
         memcpy(&h, all.data() + (size_t)rank * hb + k * sizeof(h), sizeof(h));
-        CK(cudaIpcOpenMemHandle(out, h, cudaIpcMemLazyEnablePeerAccess));
-        s.ipc_opened.push_back(*out);
-        return MAPSM_OK;
+        cudaError_t e = cudaIpcOpenMemHandle(out, h, cudaIpcMemLazyEnablePeerAccess);
+        if (e == cudaSuccess) s.ipc_opened.push_back(*out);
+        else cudaGetLastError();
+        return e;
     };
-    void* p[3];
-    if (s.plan.top_kind == MAPSM_HALO_EXCHANGE) {
-        for (int k = 0; k < 3; ++k) TRY(open(s.plan.up, k, &p[k]));
-        s.up_base[0] = static_cast<char*>(p[0]);
-        s.up_base[1] = static_cast<char*>(p[1]);
-        s.up_mail = static_cast<char*>(p[2]);
+    void* pu[3] = {nullptr, nullptr, nullptr};
+    void* pd[3] = {nullptr, nullptr, nullptr};
+    const bool top = s.plan.top_kind == MAPSM_HALO_EXCHANGE, bot = s.plan.bottom_kind == MAPSM_HALO_EXCHANGE;
+    const bool same = bot && top && s.plan.down == s.plan.up;  // g == 2 under WRAP: one peer, mapped once
+    for (int k = 0; k < 3 && le == cudaSuccess && top; ++k) le = open(s.plan.up, k, &pu[k]);
+    for (int k = 0; k < 3 && le == cudaSuccess && bot && !same; ++k) le = open(s.plan.down, k, &pd[k]);
+    // every rank learns whether every rank linked
+    int ok_h = le == cudaSuccess ? 1 : 0, all_ok = 0;
+    CK(cudaMemcpyAsync(dev, &ok_h, sizeof(int), cudaMemcpyHostToDevice, s.main));
+    nr = g_nccl.allReduce(dev, dev + 1, 1, ncclInt32, ncclMin, c->comm, s.main);
+    ce = cudaMemcpyAsync(&all_ok, dev + 1, sizeof(int), cudaMemcpyDeviceToHost, s.main);
+    se = cudaStreamSynchronize(s.main);
+    cudaFree(dev);
+    if (nr != ncclSuccess) return fail(MAPSM_ENCCL, "P2P link agreement: %s", g_nccl.errStr(nr));
+    if (ce != cudaSuccess || se != cudaSuccess) return fail(MAPSM_ECUDA, "P2P link agreement copy failed");
+    if (!all_ok) {
+        for (void* q : s.ipc_opened) cudaIpcCloseMemHandle(q);
+        s.ipc_opened.clear();
+        if (le != cudaSuccess)
+            return fail(MAPSM_EUNSUPPORTED, "P2P exchange: CUDA IPC linking failed here: %s", cudaGetErrorString(le));
+        return fail(MAPSM_EUNSUPPORTED, "P2P exchange: CUDA IPC linking failed on another rank");
+    }
+    if (top) {
+        s.up_base[0] = static_cast<char*>(pu[0]);
+        s.up_base[1] = static_cast<char*>(pu[1]);
+        s.up_mail = static_cast<char*>(pu[2]);
         mapsm_slab_plan up;
         compute_plan(g->units(), c->g, g->r, g->boundary, s.plan.up, &up);
         s.up_rows = up.rows;
     }
-    if (s.plan.bottom_kind == MAPSM_HALO_EXCHANGE) {
-        if (s.plan.down == s.plan.up && s.up_mail) {  // g == 2 under WRAP: one peer, mapped once
-            s.down_base[0] = s.up_base[0];
-            s.down_base[1] = s.up_base[1];
-            s.down_mail = s.up_mail;
-        } else {
-            for (int k = 0; k < 3; ++k) TRY(open(s.plan.down, k, &p[k]));
-            s.down_base[0] = static_cast<char*>(p[0]);
-            s.down_base[1] = static_cast<char*>(p[1]);
-            s.down_mail = static_cast<char*>(p[2]);
-        }
+    if (bot) {
+        void** q = same ? pu : pd;
+        s.down_base[0] = static_cast<char*>(q[0]);
+        s.down_base[1] = static_cast<char*>(q[1]);
+        s.down_mail = static_cast<char*>(q[2]);
     }
     g->p2p_linked = true;
     return MAPSM_OK;
@@ -1483,6 +1509,26 @@ static mapsm_status bind_impl(mapsm_grid_s* g, const void* ptr, int64_t pitch, b
             CK(cudaStreamWaitEvent(s.main, s.ev_h, 0));
         }
         g->exchanges = 0;
+    }
+    if (g->opt_p2p && !g->ctx->local && g->ctx->world > 1) {
+        // Across processes a neighbour's LAST launch of the previous run may
+        // still deliver into my halo and mailbox after my reset above (its
+        // kernels need not have finished when I entered this bind).  Every
+        // rank's previous launches precede its part of the initial exchange
+        // (stream order), so once that collective completed none is in
+        // flight: reset again, then a barrier so that no neighbour starts
+        // delivering the new run before every mailbox is clean.
+        Slab& s = g->slabs[0];
+        CK(cudaSetDevice(s.device));
+        CK(cudaStreamSynchronize(s.main));
+        CK(cudaMemsetAsync(s.mailbox, 0, kMailboxBytes, s.main));
+        int* flag = nullptr;
+        CK(cudaMallocAsync(reinterpret_cast<void**>(&flag), sizeof(int), s.main));
+        CK(cudaMemsetAsync(flag, 0, sizeof(int), s.main));
+        ncclResult_t nr = g_nccl.allReduce(flag, flag, 1, ncclInt32, ncclSum, g->ctx->comm, s.main);
+        cudaFreeAsync(flag, s.main);
+        if (nr != ncclSuccess) return fail(MAPSM_ENCCL, "P2P bind barrier: %s", g_nccl.errStr(nr));
+        CK(cudaStreamSynchronize(s.main));
     }
     g->deep_valid = true;
     return async ? MAPSM_OK : check_async(g);
