@@ -1985,7 +1985,10 @@ extern "C" mapsm_status mapsm_set_option(mapsm_grid g, mapsm_option opt, int64_t
             if (v < 2) return fail(MAPSM_EINVAL, "graph iters must be >= 2");
             g->opt_graph_iters = v;
             break;
-        case MAPSM_OPT_NO_EXCHANGE: g->opt_no_exchange = v != 0; break;
+        case MAPSM_OPT_NO_EXCHANGE:
+            if (g->opt_no_exchange != (v != 0)) drop_graphs(g);  // captured passes hold the old schedule
+            g->opt_no_exchange = v != 0;
+            break;
         case MAPSM_OPT_PERSISTENT:
             if (v < 0 || v > 2) return fail(MAPSM_EINVAL, "persistent mode %lld (0, 1, 2)", (long long)v);
             g->opt_persistent = v != 0;

@@ -260,3 +260,24 @@ def test_ring_conv5_full_grid(ring_ctx, K):
         g.iterate(2)
         got = g.gather()
     assert np.array_equal(got.view(np.uint32), oracle.conv(f0, W, 2, "wrap").view(np.uint32))
+
+
+def test_no_exchange_toggle_after_graph_capture(ring_ctx):
+    """MAPSM_OPT_NO_EXCHANGE set after CUDA graphs were captured must take
+    effect (the captured passes hold the old schedule and are dropped): with
+    the exchange off the halos go stale and the result leaves the oracle's;
+    with it back on and a fresh bind it matches again."""
+    w, h = 2048, 64
+    x0 = mi.life_u8(8100, w, h)
+    with M.Grid(ring_ctx, w, h, "life", 1, "wrap") as g:
+        g.bind(x0)
+        g.iterate(32)  # graphs captured with the exchange
+        assert np.array_equal(g.gather(), oracle.life(x0, 32, "wrap"))
+        g.set_option(M.OPT_NO_EXCHANGE, 1)
+        g.iterate(32)
+        stale = g.gather()
+        assert not np.array_equal(stale, oracle.life(x0, 64, "wrap"))
+        g.set_option(M.OPT_NO_EXCHANGE, 0)
+        g.bind(x0)
+        g.iterate(64)
+        assert np.array_equal(g.gather(), oracle.life(x0, 64, "wrap"))
