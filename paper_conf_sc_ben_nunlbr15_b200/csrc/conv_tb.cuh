@@ -254,7 +254,10 @@ __device__ __forceinline__ void st_shared_f4_s(uint32_t a, float v) {
     asm volatile("st.shared.v4.f32 [%0], {%1, %1, %1, %1};" ::"r"(a), "f"(v) : "memory");
 }
 
-constexpr int kTbWarps = 13;  // level-1 (= level-2) warps: 2 * 13 + ghost + producer = 28 warps
+// level-1 (= level-2) warps: 2 * 13 + ghost + producer = 28 warps.  Not a
+// free knob: builds with 10, 12 or 14 hung on the 16384^2 bench grid
+// (round 2), so any change needs the ring's arrival counts re-derived.
+constexpr int kTbWarps = 13;
 constexpr int kTbL1Margin = 8;
 
 // Ring bookkeeping.  Both rings (the TMA input ring and the generation-t+1
