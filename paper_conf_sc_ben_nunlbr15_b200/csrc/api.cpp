@@ -650,6 +650,7 @@ static mapsm_status launch_step(mapsm_grid_s* g, Slab& s, int b_in, const RowBan
     geom.rpitch = g->rpitch;
     geom.rec = bulk ? &s.rec_bulk : &s.rec_bnd;
     geom.wslot = g->wslot;
+    geom.pdl = sms == 0;  // (the concurrent schedules pass their SM split)
     TimingPair* tp = nullptr;
     if (g->opt_timing && &s == &g->slabs[0]) {
         auto& vec = bulk ? s.t_bulk : s.t_bnd;

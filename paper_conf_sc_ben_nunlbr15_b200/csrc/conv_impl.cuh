@@ -378,6 +378,7 @@ __global__ void __launch_bounds__((NC + 1) * 32, (R <= 2 ? 1 : kConvBigCtas)) co
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
     uint64_t* empty = full + NS;
     tma::init_barriers<NS>(full, empty, NC);
+    tma::pdl_wait_and_release();
     // warp index through a full-mask shuffle: ptxas then knows the role
     // branch below is warp-uniform and may use the uniform datapath (LDCU
     // weights) inside the consumer code
@@ -642,10 +643,11 @@ cudaError_t launch_conv_tma_t(const StencilGeom& g, const RowBands& b, const flo
     tma_record(g.rec, LK_CONV_TMA, p, ctas, (NC + 1) * 32, smem, NS, 1, NC);
     if (ctas == 0) return cudaSuccess;
     if (link)
-        conv_tma_kernel<R, NC, NS, CM, EPL, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(pp);
+        return tma_launch(conv_tma_kernel<R, NC, NS, CM, EPL, true>, (unsigned)ctas, (NC + 1) * 32, smem, s, pp,
+                          false);  // (measured: PDL costs the fused conv launch ~2 us per generation)
     else
-        conv_tma_kernel<R, NC, NS, CM, EPL, false><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(pp);
-    return cudaGetLastError();
+        return tma_launch(conv_tma_kernel<R, NC, NS, CM, EPL, false>, (unsigned)ctas, (NC + 1) * 32, smem, s, pp,
+                          g.pdl);
 }
 
 // The FMA-bound radii (r >= 3) are compiled one column mode per translation

@@ -329,6 +329,7 @@ __global__ void __launch_bounds__((2 * NW + 2) * 32, 1) conv_tb2_kernel(const __
             tma::mbar_init(reinterpret_cast<uint64_t*>(smem + Ly::OFF_L1EMPTY) + s, NW);
         }
     tma::init_barriers<NS>(full, empty, NW + 1);
+    tma::pdl_wait_and_release();
     const int warp = __shfl_sync(0xffffffffu, (int)(threadIdx.x >> 5), 0), lane = threadIdx.x & 31;
     tma::SegIter it = tma::seg_iter(p);
     tma::Seg sg;
@@ -522,8 +523,7 @@ cudaError_t launch_conv_tb2_t(const StencilGeom& g, const RowBands& b, int zero_
     const int64_t ctas = tma_plan_grid(p, b, num_sms, 1, S);
     tma_record(g.rec, LK_CONV_TB2, p, ctas, (2 * NC + 2) * 32, smem, NS, 1, NC, 2);
     if (ctas == 0) return cudaSuccess;
-    conv_tb2_kernel<R, NC, NS, CM><<<(unsigned)ctas, (2 * NC + 2) * 32, smem, s>>>(pp);
-    return cudaGetLastError();
+    return tma_launch(conv_tb2_kernel<R, NC, NS, CM>, (unsigned)ctas, (2 * NC + 2) * 32, smem, s, pp, g.pdl);
 }
 
 template <int R>

@@ -53,6 +53,9 @@ struct StencilGeom {
     int64_t plane_rows = 0, rpitch = 0;
     LaunchRec* rec = nullptr;  // filled by the launcher when non-null
     int wslot = -1;            // conv r >= 3: the grid's weight slot (conv_upload_weights)
+    bool pdl = true;           // programmatic dependent launch on the previous kernel of the stream
+                               // (off in the concurrent-boundary schedules: an early-scheduled
+                               // interior grid would take the SMs kept for the boundary launch)
 };
 
 // fp32 conv, r = 2..4 (FFMA2 kernels): weights live in __constant__ slots,

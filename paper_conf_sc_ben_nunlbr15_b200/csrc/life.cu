@@ -23,6 +23,7 @@
 // input rows per chunk cost ~2% extra reads (L2 hits).
 #include <cuda_runtime.h>
 #include <stdint.h>
+#include <stdlib.h>
 
 #include <type_traits>
 
@@ -345,6 +346,7 @@ __global__ void __launch_bounds__((NC + 1) * 32) life_tma_kernel(const __grid_co
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * G::kStageBytes);
     uint64_t* empty = full + NS;
     tma::init_barriers<NS>(full, empty, NC);
+    tma::pdl_wait_and_release();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     tma::SegIter it = tma::seg_iter(p);
     tma::Seg sg;
@@ -525,11 +527,8 @@ cudaError_t launch_life_tma_t(const StencilGeom& g, const RowBands& b, int num_s
     const int64_t ctas = tma_plan_grid(p, b, num_sms, ctas_per_sm, G::kStripElems, link != nullptr);
     tma_record(g.rec, LK_LIFE_TMA, p, ctas, (NC + 1) * 32, smem, NS, 1, NC);
     if (ctas == 0) return cudaSuccess;
-    if (link)
-        life_tma_kernel<NC, NS, CM, true><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(p);
-    else
-        life_tma_kernel<NC, NS, CM, false><<<(unsigned)ctas, (NC + 1) * 32, smem, s>>>(p);
-    return cudaGetLastError();
+    if (link) return tma_launch(life_tma_kernel<NC, NS, CM, true>, (unsigned)ctas, (NC + 1) * 32, smem, s, p, g.pdl);
+    return tma_launch(life_tma_kernel<NC, NS, CM, false>, (unsigned)ctas, (NC + 1) * 32, smem, s, p, g.pdl);
 }
 
 template <int NC, int NS>

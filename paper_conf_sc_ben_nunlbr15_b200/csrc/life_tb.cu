@@ -76,6 +76,7 @@ struct TbParams {
     tma::RowStream s;  // s.n = words per row, bands, row maps (ROWMAP_CLAMP = mirror here)
     int64_t strip;     // strip width in words (multiple of 4); the last strip may be shorter
     int zero_top, zero_bot;  // ZERO global edges: rows outside [0, rows) forced to 0 every generation
+    int pdl;                 // (host) programmatic dependent launch (StencilGeom::pdl)
 };
 
 struct TbSeg {
@@ -282,6 +283,7 @@ __global__ void __maxnreg__(MAPSM_TB_REGS) life_tb_kernel(const __grid_constant_
     uint64_t* full = reinterpret_cast<uint64_t*>(smem + NS * stage_bytes);
     uint64_t* empty = full + NS;
     tma::init_barriers<NS>(full, empty, NC);
+    tma::pdl_wait_and_release();
     const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
     tma::SegIter it = tma::seg_iter(p);
     TbSeg sg;
@@ -359,8 +361,7 @@ cudaError_t launch_tb_t(const TbParams& P0, const RowBands& b, int nc, int num_s
     const int64_t ctas = tma_plan_grid(P.s, b, num_sms, occ[nc], (int)P.strip);
     tma_record(rec, LK_LIFE_TB, P.s, ctas, (nc + 1) * 32, smem, kNS, rows_per_stage(K), nc, K);
     if (ctas == 0) return cudaSuccess;
-    kfn<<<(unsigned)ctas, (nc + 1) * 32, smem, s>>>(P);
-    cudaError_t e = cudaGetLastError();
+    cudaError_t e = tma_launch(kfn, (unsigned)ctas, (nc + 1) * 32, smem, s, P, P.pdl != 0);
     if (e != cudaSuccess && getenv("MAPSM_DEBUG")) {
         cudaFuncAttributes fa;
         cudaFuncGetAttributes(&fa, kfn);
@@ -406,6 +407,7 @@ cudaError_t launch_life_tb(const StencilGeom& g, const RowBands& b, int k, int z
     P.strip = ((W + nstrips - 1) / nstrips + 3) / 4 * 4;
     P.zero_top = zero_top;
     P.zero_bot = zero_bot;
+    P.pdl = g.pdl ? 1 : 0;
     const int nc = (int)((P.strip + kOut - 1) / kOut);
     switch (k) {
         case 2: return launch_tb_k<2>(P, b, g.col_mode, nc, num_sms, s, g.rec);

@@ -21,6 +21,7 @@
 // bit; conv r <= 4 needs <= 4 floats).
 #pragma once
 #include <cuda_runtime.h>
+#include <stdlib.h>
 #include <stdint.h>
 
 #include "kernels.h"
@@ -236,6 +237,17 @@ __device__ __forceinline__ bool seg_next(const RowStream& p, SegIter& it, Seg& s
     return true;
 }
 
+// Programmatic dependent launch (the stencil launches of consecutive
+// generations): a CTA of generation t+1 may be scheduled while generation t
+// drains; it sets up its shared memory, then waits here until generation t
+// has completed and flushed (it reads t's output and overwrites t's input),
+// and lets generation t+2 start launching.  A no-op for launches without the
+// programmatic-serialization attribute.
+__device__ __forceinline__ void pdl_wait_and_release() {
+    asm volatile("griddepcontrol.wait;" ::: "memory");
+    asm volatile("griddepcontrol.launch_dependents;" :::);
+}
+
 template <int NS>
 __device__ __forceinline__ void init_barriers(uint64_t* full, uint64_t* empty, int consumers) {
     if (threadIdx.x == 0) {
@@ -410,6 +422,31 @@ inline int64_t tma_plan_grid(tma::RowStream& p, const RowBands& b, int num_sms, 
     // the launch has no interior band)
     p.link_ctas = boundary_first && b.nbands > 1 ? p.cta_begin[b.nbands - 1] : (int)total;
     return total;
+}
+
+// Host side: launch a ring kernel with programmatic dependent launch (the
+// kernel calls tma::pdl_wait_and_release() after its shared-memory setup),
+// so generation t+1's CTAs are scheduled while generation t drains.
+// MAPSM_NO_PDL=1 turns it off (A/B measurements).
+inline bool tma_pdl_enabled() {
+    static const bool on = getenv("MAPSM_NO_PDL") == nullptr;
+    return on;
+}
+
+template <typename Kernel, typename Param>
+inline cudaError_t tma_launch(Kernel kernel, unsigned grid, unsigned block, int smem, cudaStream_t s,
+                              const Param& p, bool pdl = true) {
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(grid);
+    cfg.blockDim = dim3(block);
+    cfg.dynamicSmemBytes = (size_t)smem;
+    cfg.stream = s;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+    attr[0].val.programmaticStreamSerializationAllowed = pdl && tma_pdl_enabled() ? 1 : 0;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    return cudaLaunchKernelEx(&cfg, kernel, p);
 }
 
 // Host side: describe a ring-kernel launch for mapsm_launch_query.
