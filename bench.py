@@ -382,7 +382,7 @@ def run_sgemm(args, wl, rank, world, local_rank):
                 "clocks": clocks, "cpu_baseline": cb,
                 "paper_context": "Table 4 P:L503-508: single-GPU 8K multiplication 245-366 ms on GTX 780/Titan "
                                  "Black/GTX 980 (CUBLAS over MAPS-Multi 248.62 ms on GTX 980)"}
-        print(json.dumps(line), flush=True)
+        emit(line)
     if world > 1:
         dist.barrier(device_ids=[local_rank])
         dist.destroy_process_group()
@@ -417,7 +417,7 @@ def run_reference(args, wl, rank, world):
             "dtype": "f32" if wl["op"] in ("conv", "sgemm") else "u8", "data": "synthetic",
             "config": {"workload": wl["label"]}, "cpu_baseline": cb,
             "e2e": {"value": value, "unit": unit, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0}}
-    print(json.dumps(line), flush=True)
+    emit(line)
 
 
 # ------------------------------------------------------------------ GPU leg
@@ -950,9 +950,26 @@ def measure(env, name, wl, steps, warmup, e2e_steps, min_region_s=0.0, extras=Fa
     return line
 
 
+_JSON_OUT = None
+
+
+def emit(line):
+    """The one JSON line on stdout (everything else the process writes to
+    file descriptor 1 — NCCL's version banner, CUDA or library logs — is
+    redirected to stderr by main())."""
+    out = _JSON_OUT or sys.stdout
+    out.write(json.dumps(line) + "\n")
+    out.flush()
+
+
 def main():
-    # NCCL's own log lines (e.g. the version banner under NCCL_DEBUG=VERSION)
-    # go to stdout by default; stdout carries only the JSON line
+    # stdout carries only the JSON line: keep a private handle on the real
+    # stdout, then point file descriptor 1 at stderr for everything else
+    # (NCCL prints its version banner to stdout under NCCL_DEBUG=VERSION)
+    global _JSON_OUT
+    sys.stdout.flush()
+    _JSON_OUT = os.fdopen(os.dup(1), "w")
+    os.dup2(2, 1)
     os.environ.setdefault("NCCL_DEBUG_FILE", "/dev/stderr")
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
@@ -1011,7 +1028,7 @@ def main():
             head["configs"] = {name: {k: v for k, v in sub.items() if k not in ("n_gpus", "higher_is_better",
                                                                                   "vs_baseline", "data")}
                                for name, sub in subs.items()}
-        print(json.dumps(head), flush=True)
+        emit(head)
 
 
 if __name__ == "__main__":
